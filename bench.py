@@ -1,0 +1,345 @@
+#!/usr/bin/env python
+"""bench.py — headline benchmark of the B200-native heterogeneous float64 sort.
+
+Metric (BASELINE.json): end-to-end keys/s host->host (float64) at 1/2/4/8 B200; radix GB/s vs HBM.
+Workload at N=1: BASELINE.json configs[1] — n = 2^30 uniform float64 (8 GiB), one batch
+(b_s = n), one B200.  A "step" is one whole GPUSort of that batch (K1 + K2 + 8 onesweep passes,
+PAPER.md §III-B) with the input already resident in HBM -> ``value``; ``e2e`` is the same metric
+through the public C ABI hsort_sort() with pinned HOST buffers (HtoD + GPUSort + DtoH inside the
+timed region, BLINE workflow P:285-292).
+
+Multi-GPU (torchrun, one process per GPU): every rank sorts its own 2^30-key batch — batches are
+independent units, no data-path collective — so scaling is "weak" and
+value = (N * n) / max-over-ranks time.
+
+``--impl reference`` times the CPU oracle (oracle/, serial std::sort under IEEE totalOrder) on the
+host cores, on a bounded sample of the same workload per step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "end-to-end keys/s host->host (float64) at 1/2/4/8 B200; radix GB/s vs HBM"
+N_KEYS = 1 << 30
+SEED = 2
+WORKLOAD = "C2: n=2^30 uniform float64 (8 GiB), single batch b_s=n, 1 B200 per rank"
+ALG_BYTES_PER_KEY_PASS = 16  # one onesweep digit pass reads 8 B and writes 8 B per key
+ORACLE_SAMPLE = 1 << 26      # cpu_baseline sample (~15 s of serial CPU work)
+REF_STEP_SAMPLE = 1 << 24    # --impl reference: keys per step
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_traffic():
+    """Per-launch DRAM bytes of the onesweep pass from the committed ncu --set full capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        try:
+            d = json.load(open(p))
+            return d.get("onesweep_dram_bytes_per_launch"), d.get("n")
+        except Exception:
+            return None, None
+    return None, None
+
+
+class ClockSampler:
+    """Samples SM clocks and throttle reasons via NVML during the timed region."""
+
+    def __init__(self, dev_index: int):
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        names = {
+            getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8): "hw_slowdown",
+            getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40): "hw_thermal_slowdown",
+            getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20): "sw_thermal_slowdown",
+            getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4): "sw_power_cap",
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in names.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.nv:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        return {
+            "sm_mhz": statistics.median(self.samples) if self.samples else None,
+            "sm_max_mhz": self.max_mhz,
+            "reasons": sorted(self.reasons),
+            "samples": len(self.samples),
+        }
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def cpu_baseline_oracle(n_sample: int):
+    import hsort_inputs
+    import oracle
+    A = hsort_inputs.generate("uniform", n_sample, seed=SEED)
+    t = time.perf_counter()
+    oracle.sort_f64(A)
+    dt = time.perf_counter() - t
+    return {
+        "value": n_sample / dt, "unit": "keys/s", "cores": 1, "kind": "oracle",
+        "sample": f"first {n_sample} keys of the C2 workload (uniform seed {SEED}), serial "
+                  f"std::sort under IEEE totalOrder (oracle/oracle.cpp), {dt:.2f} s",
+    }
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    import hsort_inputs
+    import oracle
+    n = REF_STEP_SAMPLE
+    A = hsort_inputs.generate("uniform", n, seed=SEED)
+    for _ in range(args.warmup):
+        oracle.sort_f64(A[: n // 16])
+    times = []
+    for _ in range(args.steps):
+        t = time.perf_counter()
+        oracle.sort_f64(A)
+        times.append(time.perf_counter() - t)
+    tot = sum(times)
+    value = n * args.steps / tot
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "keys/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": WORKLOAD, "n": N_KEYS, "batch_elems": N_KEYS,
+                   "reference_sample_per_step": n},
+        "cpu_baseline": {"value": value, "unit": "keys/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{n} keys of the C2 workload per step (uniform seed {SEED})"},
+        "e2e": {"value": value, "unit": "keys/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=N_KEYS, help="keys per rank (default 2^30, config C2)")
+    ap.add_argument("--e2e-steps", type=int, default=None)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    args.warmup = max(args.warmup, 3)
+
+    import torch
+    import torch.distributed as dist
+
+    import hsort_inputs
+    import paper_conf_ipps_gowanlockk18a_b200 as hs
+
+    ws, rank, local = dist_env()
+    if ws > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.cuda.current_device()
+
+    def barrier():
+        if ws > 1:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if ws == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    n = args.n
+    hs.hsort_set_option("kernel_timing", 1)
+    t0 = time.perf_counter()
+    hs.hsort_init()
+    t_init = time.perf_counter() - t0
+
+    # inputs: pinned host A (generated in place), device copy for the resident arm
+    A_h = torch.empty(n, dtype=torch.float64).pin_memory()
+    hsort_inputs.generate("uniform", n, seed=SEED + rank, out=A_h.numpy())
+    B_h = torch.empty(n, dtype=torch.float64).pin_memory()
+    d_in = A_h.to(f"cuda:{dev}", non_blocking=False)
+    d_out = torch.empty_like(d_in)
+    stream = torch.cuda.current_stream()
+
+    # ---- device-resident arm (value): one step = one GPUSort of the whole batch ----------------
+    for _ in range(args.warmup):
+        hs.hsort_sort_device(d_in, d_out, stream)
+    torch.cuda.synchronize()
+    # sampled correctness guard on the benchmarked output (full parity lives in tests/)
+    o = d_out[:: max(1, n // (1 << 20))]
+    assert bool((o[1:] >= o[:-1]).all()), "device output not sorted"
+
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    pass_ms, hist_ms, other_ms = [], [], []
+    n_active = 8
+    sampler = ClockSampler(dev)
+    barrier()
+    torch.cuda.synchronize()
+    with sampler:
+        step_ms = []
+        for _ in range(args.steps):
+            ev0.record(stream)
+            hs.hsort_sort_device(d_in, d_out, stream)
+            ev1.record(stream)
+            ev1.synchronize()
+            step_ms.append(ev0.elapsed_time(ev1))
+            kt = hs.hsort_get_kernel_times()
+            n_active = kt["num_active"]
+            pass_ms.extend(kt["passes"][:n_active])
+            hist_ms.append(kt["hist"])
+            other_ms.append(kt["scan"] + kt["copy"] + sum(kt["passes"][n_active:]))
+    torch.cuda.synchronize()
+    barrier()
+    total_ms = max_over_ranks(sum(step_ms))
+    ms_per_step = total_ms / args.steps
+    value = ws * n * args.steps / (total_ms / 1e3)
+
+    # roofline of the dominant kernel (k_onesweep): algorithmic 16 B/key per pass
+    peak, peak_src = load_peaks()
+    avg_pass_ms = statistics.mean(pass_ms) if pass_ms else float("nan")
+    achieved = ALG_BYTES_PER_KEY_PASS * n / (avg_pass_ms / 1e3) / 1e9
+    traffic, traffic_n = load_traffic()
+    if traffic is not None and traffic_n and traffic_n != n:
+        traffic = traffic * n / traffic_n
+    share = sum(pass_ms) / sum(step_ms) if step_ms else None
+
+    # ---- end-to-end arm (e2e): public API, pinned host buffers, HtoD + sort + DtoH ------------
+    e2e_steps = args.e2e_steps or max(3, min(args.steps, 5))
+    hs.hsort_sort(A_h, B_h, batch_elems=0, n_gpus=1)  # warm (buffers cached)
+    barrier()
+    e2e_t = []
+    for _ in range(e2e_steps):
+        t = time.perf_counter()
+        hs.hsort_sort(A_h, B_h, batch_elems=0, n_gpus=1)
+        e2e_t.append(time.perf_counter() - t)
+    st = hs.hsort_get_stats()
+    Bv = B_h.numpy()[:: max(1, n // (1 << 20))]
+    assert bool((Bv[1:] >= Bv[:-1]).all()), "host output not sorted"
+    barrier()
+    e2e_total = max_over_ranks(sum(e2e_t))
+    e2e_value = ws * n * e2e_steps / e2e_total
+
+    line = {
+        "metric": METRIC,
+        "value": value,
+        "unit": "keys/s",
+        "n_gpus": ws,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": ms_per_step,
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f64",
+        "data": "synthetic",
+        "config": {
+            "workload": WORKLOAD,
+            "n": n,
+            "batch_elems": n,
+            "distribution": f"uniform U[0,1) 53-bit, splitmix64 seed {SEED}+rank",
+            "parallelism": f"independent batches, {ws} rank(s) x 1 GPU",
+            "l2": "input 8 GiB >> 126 MB L2: no flush needed between steps",
+        },
+        "roofline": {
+            "kernel": "k_onesweep (one 8-bit LSD digit pass)",
+            "bound": "hbm",
+            "achieved": achieved,
+            "peak": peak,
+            "peak_source": peak_src,
+            "unit": "GB/s",
+            "frac": achieved / peak,
+            "traffic": traffic,
+            "alg_bytes_per_launch": ALG_BYTES_PER_KEY_PASS * n,
+            "avg_launch_ms": avg_pass_ms,
+            "launches_per_step": n_active,
+            "share_of_step": share,
+            "hist_ms": statistics.mean(hist_ms) if hist_ms else None,
+        },
+        "e2e": {
+            "value": e2e_value,
+            "unit": "keys/s",
+            "h2d_bytes_per_step": n * 8,
+            "d2h_bytes_per_step": n * 8,
+            "api": "hsort_sort(A pinned, B pinned, n, batch_elems=0 -> BLINE, n_gpus=1)",
+            "ms_per_step": 1e3 * e2e_total / e2e_steps,
+            "t_h2d_s": st["t_h2d"], "t_gpu_sort_s": st["t_gpu_sort"], "t_d2h_s": st["t_d2h"],
+            "mode": st["mode_name"],
+        },
+        "gpu_launches": args.steps * 11,
+        "clocks": sampler.summary(),
+        "init_s": t_init,
+    }
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline_oracle(ORACLE_SAMPLE)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    hs.hsort_finalize()
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,220 @@
+/* include/hsort.h — C ABI of the B200-native heterogeneous float64 sort.
+ *
+ * The problem (§I): "given an unsorted input list, A, of n elements in main
+ * memory, generate a sorted output list, B, using the CPUs and GPU(s) on the platform".
+ * The method (§III): split A into n_b batches of b_s elements, sort each
+ * batch on the GPU, merge the sorted batches with a multiway merge,
+ * pipelining transfers through pinned staging buffers on CUDA streams (PIPEDATA) with
+ * parallel host copies (PARMEMCPY).  Table I names the parameters
+ * n, n_b, n_GPU, n_s, b_s, p_s used below.
+ *
+ * Result contract (readings A-1..A-4): B holds A's 64-bit patterns permuted into
+ * ascending IEEE 754 totalOrder (-NaNs < -inf < ... < -0 < +0 < ... < +inf < +NaNs).  No
+ * floating-point arithmetic touches a key; NaN payloads and the sign of zero are preserved.
+ * Equal keys are bit-identical, so the output is unique and checked bit-exactly.
+ *
+ * Conventions
+ *  - Every function returns HSORT_OK (0) or a negative hsort_status; none throws.
+ *  - hsort_last_error() returns a thread-local message for the last failing call.
+ *  - After a CUDA error the library is poisoned: later calls return HSORT_ERR_CUDA until
+ *    hsort_finalize().  B's contents are unspecified after an error; A is never written
+ *    unless B == A.
+ *  - The library is not re-entrant: a concurrent hsort_sort returns HSORT_ERR_BUSY.
+ *  - "host" pointers may be pageable or pinned (cudaHostAlloc / cudaHostRegister); pinned
+ *    buffers are DMA'd directly, pageable ones go through the pinned staging ring (Stage, MCpy).
+ *  - "device" pointers are CUDA global memory on the CURRENT device; "stream" is a cudaStream_t
+ *    (NULL = legacy default stream).  Device entry points are asynchronous on that stream
+ *    unless stated otherwise.
+ */
+#ifndef HSORT_H_
+#define HSORT_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  HSORT_OK = 0,
+  HSORT_ERR_INVALID = -1,          /* bad argument (null with n > 0, partial overlap, n_gpus) */
+  HSORT_ERR_NOT_INITIALIZED = -2,  /* hsort_init() not called */
+  HSORT_ERR_HOST_OOM = -3,         /* host allocation (W, pinned ring) failed */
+  HSORT_ERR_DEVICE_OOM = -4,       /* device allocation failed */
+  HSORT_ERR_CUDA = -5,             /* CUDA runtime error (library poisoned until finalize) */
+  HSORT_ERR_NCCL = -6,             /* reserved: NCCL exchange (multi-GPU resident mode) */
+  HSORT_ERR_BUSY = -7,             /* concurrent call, or hsort_init twice */
+  HSORT_ERR_INTERNAL = -8          /* invariant violated inside the library */
+} hsort_status;
+
+/* Merge/placement mode chosen by the planner (A1) for one hsort_sort call. */
+typedef enum {
+  HSORT_MODE_BLINE = 0,     /* n_b = 1: A -> HtoD -> GPUSort -> DtoH -> B */
+  HSORT_MODE_RESIDENT = 1,  /* n_b > 1, sorted runs stay in HBM, GPU merge-path merge, DtoH of
+                               merged chunks overlapped with the merge (B200 design) */
+  HSORT_MODE_STREAM = 2     /* n_b > 1, runs go to host working memory W, multiway merge on the
+                               CPU (+ optional GPU share f): PIPEDATA / BLINEMULTI */
+} hsort_mode;
+
+/* Per-call statistics (the paper reports per-component response times). Seconds are
+ * host wall-clock (steady_clock) unless marked "device". */
+typedef struct hsort_stats {
+  uint64_t n;              /* keys sorted */
+  uint64_t b_s;            /* batch size (elements) */
+  uint64_t n_b;            /* number of batches = ceil(n / b_s) */
+  int32_t n_gpus;          /* GPUs used */
+  int32_t n_s;             /* batch slots in flight per GPU (streams) */
+  int32_t mode;            /* hsort_mode */
+  int32_t passes_run;      /* radix digit passes run, summed over batches */
+  int32_t passes_skipped;  /* trivial digit passes skipped (one non-empty bin), summed */
+  int32_t direct_in;       /* 1 if A was DMA'd directly (pinned), 0 if staged */
+  int32_t direct_out;      /* 1 if B was written directly by DMA (pinned), 0 if staged */
+  int32_t merge_k;         /* runs merged (= n_b) */
+  double merge_gpu_fraction; /* share f of merge output produced by GPUs (A12) */
+  double t_total;          /* whole hsort_sort call */
+  double t_sort_phase;     /* from first HtoD to last run sorted (and, STREAM, landed in W) */
+  double t_merge_phase;    /* merge (+ its DtoH) after the sort phase */
+  double t_gpu_sort;       /* device: sum of GPUSort (K1+K2+K3) over batches (CUDA events) */
+  double t_h2d;            /* device: sum of HtoD copy time (CUDA events) */
+  double t_d2h;            /* device: sum of DtoH copy time (CUDA events) */
+  double t_stage;          /* host: sum of MCpy time into/out of pinned staging */
+  double t_merge_cpu;      /* host: CPU multiway merge time */
+  double t_merge_gpu;      /* device: GPU merge kernels (K4+K5) */
+  double t_init;           /* hsort_init() duration (pinned + device allocation) */
+  uint64_t bytes_h2d;      /* bytes moved host -> device */
+  uint64_t bytes_d2h;      /* bytes moved device -> host */
+} hsort_stats;
+
+/* Planner output (A1).  Pure host arithmetic; see hsort_plan(). */
+typedef struct hsort_plan_t {
+  uint64_t n, b_s, n_b;
+  int32_t n_gpus, n_s, mode;
+  uint64_t last_batch;            /* size of the ragged last batch (reading A-12) */
+  uint64_t device_bytes_per_gpu;  /* predicted device footprint */
+  uint64_t host_bytes;            /* predicted host working memory (W + staging) */
+  double batches_per_stream;      /* n_b / (n_s * n_GPU) */
+} hsort_plan_t;
+
+/* ---------------------------------------------------------------------------------------------
+ * Lifecycle
+ * ------------------------------------------------------------------------------------------- */
+
+/* Enumerate GPUs; create per-GPU streams (H2D / compute / D2H) and the pinned staging ring
+ * (n_ring slots of p_s bytes per GPU and direction; P:331-334 — pinned memory is expensive to
+ * allocate, so it is done once here).  Device batch buffers are allocated lazily by
+ * the first hsort_sort and cached.  A second call before hsort_finalize -> HSORT_ERR_BUSY. */
+int hsort_init(void);
+
+/* Free every library-owned resource.  Safe after errors and when not initialised. */
+int hsort_finalize(void);
+
+/* ---------------------------------------------------------------------------------------------
+ * The sort (host -> host).  Synchronous; retains no pointer.
+ *   A_host       n float64, 8-byte aligned host memory, read-only (unless B == A).
+ *   B_host       n float64 writable host memory; B == A allowed (in place); partial overlap of
+ *                A and B -> HSORT_ERR_INVALID.
+ *   n            number of keys; 0 -> HSORT_OK, no-op.
+ *   batch_elems  b_s; 0 -> auto (the largest batch with 2*b_s*n_s*8 bytes fitting in HBM,
+ *                P:864-870); > n -> clamped to n.  n_b = ceil(n / b_s).
+ *   n_gpus       1..visible devices; 0 -> all visible; > visible -> HSORT_ERR_INVALID.
+ * ------------------------------------------------------------------------------------------- */
+int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_elems, int n_gpus);
+
+/* Same, on raw uint64 keys (ascending unsigned order; no key transform). */
+int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_t batch_elems,
+                   int n_gpus);
+
+/* ---------------------------------------------------------------------------------------------
+ * Options, statistics, errors
+ *   keys: "n_s" (batch slots per GPU, default 2), "p_s" (pinned staging chunk bytes),
+ *         "n_ring" (pinned slots per direction), "memcpy_threads" (PARMEMCPY threads; 1 = serial
+ *         MCpy), "merge_threads" (CPU merge threads), "resident" (-1 auto, 0 force
+ *         STREAM, 1 force RESIDENT), "merge_gpu_permille" (A12 share f in 1/1000; -1 auto),
+ *         "pipeline" (1 = overlapped streams PIPEDATA, 0 = blocking BLINEMULTI ablation),
+ *         "merge_chunk" (GPU merge output chunk elements), "device_reserve_mb" (HBM left free),
+ *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times).
+ * ------------------------------------------------------------------------------------------- */
+int hsort_set_option(const char* key, int64_t value);
+int hsort_get_option(const char* key, int64_t* value);
+int hsort_get_stats(hsort_stats* out);      /* stats of the last successful hsort_sort */
+const char* hsort_last_error(void);          /* thread-local; never NULL */
+const char* hsort_version(void);
+
+/* Per-kernel device durations of the last GPUSort on the current device, recorded with CUDA
+ * events on the sort's stream when option "kernel_timing" = 1 (used by bench.py for the
+ * roofline).  ms[0] = K1 histograms, ms[1] = K2 scan/plan, ms[2+p] = K3 pass p (p = 0..7; passes
+ * p >= *num_active_passes are empty launches), ms[10] = final copy.  Returns the number of
+ * entries written (>= 0) or a negative hsort_status.  Call after synchronising the stream. */
+int hsort_get_kernel_times(float* ms, int max_entries, int* num_active_passes);
+
+/* Planner (A1): pure host arithmetic, no GPU needed.  device_bytes = usable HBM per GPU
+ * (0 -> query the current device).  Fills *out; HSORT_ERR_INVALID on bad arguments. */
+int hsort_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_bytes,
+               hsort_plan_t* out);
+
+/* ---------------------------------------------------------------------------------------------
+ * Device-resident entry points (current device, library-owned scratch; stream-ordered).
+ * ------------------------------------------------------------------------------------------- */
+
+/* GPUSort of one batch, device -> device:  d_out = totalOrder-sorted d_in.
+ * d_in == d_out allowed.  Runs K1 (digit histograms) + K2 (bin scan / pass plan) + up to 8
+ * K3 onesweep passes; trivial digits are skipped on the device.  Requires hsort_init(). */
+int hsort_sort_device(const double* d_in, double* d_out, uint64_t n, void* stream);
+
+/* Same, keys already uint64 (ascending unsigned); in_f64/out_f64 select whether the input is
+ * float64 bits (key transform fused into the first pass) and whether the output is stored as
+ * float64 bits (inverse transform fused into the last pass). */
+int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, int in_f64,
+                           int out_f64, void* stream);
+
+/* K1 alone: d_hist[8*256] (uint64, device) = per-digit histograms of the keys (digit d =
+ * bits [8d, 8d+8) of key(x) if in_f64 else of the raw uint64).  Synchronous. */
+int hsort_device_histograms(const uint64_t* d_keys, uint64_t n, int in_f64, uint64_t* d_hist,
+                            void* stream);
+
+/* K3 alone: one stable LSD counting-sort pass by digit `digit` (0..7) of raw uint64 keys,
+ * d_src -> d_dst (must not overlap).  Synchronous. */
+int hsort_device_radix_pass(const uint64_t* d_src, uint64_t* d_dst, uint64_t n, int digit,
+                            void* stream);
+
+/* K4 alone: exact co-ranks (merge path) of output positions o_b = min(b*step, total)
+ * for b = 0..n_bounds-1 over k sorted uint64 runs d_keys[h_off[j] .. h_off[j+1]).  d_ranks is
+ * (n_bounds x k) uint64 row-major on the device; h_off is k+1 HOST offsets.  Ties are taken in
+ * run order.  Synchronous. */
+int hsort_device_corank(const uint64_t* d_keys, const uint64_t* h_off, int k, uint64_t step,
+                        uint64_t n_bounds, uint64_t* d_ranks, void* stream);
+
+/* K4+K5: multiway merge of k sorted uint64 runs (layout as above) into d_out
+ * (total = h_off[k]-h_off[0] elements); out_f64 = 1 stores inverse-transformed float64 bits.
+ * Synchronous. */
+int hsort_device_merge(const uint64_t* d_keys, const uint64_t* h_off, int k, uint64_t* d_out,
+                       int out_f64, void* stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * Host-native components (no GPU needed)
+ * ------------------------------------------------------------------------------------------- */
+
+/* Parallel host memcpy (PARMEMCPY) with `threads` workers (0 = option default). */
+int hsort_par_memcpy(void* dst, const void* src, uint64_t bytes, int threads);
+
+/* CPU multiway merge (H2): k sorted uint64 key runs keys[off[j]..off[j+1]) (host)
+ * -> out (host, total elements); out_f64 = 1 stores inverse-transformed float64 bits.
+ * Output ranges are split by exact co-ranks and merged by `threads` loser trees. */
+int hsort_host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out,
+                     int out_f64, int threads);
+
+/* Exact co-ranks of output position o over the k host runs (same definition as K4). */
+int hsort_host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o,
+                      uint64_t* ranks);
+
+/* The PIPEMERGE heuristic (reading A-9): number of pair-wise merges overlapped with
+ * GPU sorting.  Pure arithmetic. */
+uint64_t hsort_pipemerge_count(uint64_t n_b, int n_gpus);
+
+/* Number of GPUs visible to the library (0 when none; never an error). */
+int hsort_device_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HSORT_H_ */

@@ -1,0 +1,1077 @@
+// api.cpp — the C ABI (include/hsort.h), planner (A1), staging ring (A2/A8), stream pipeline
+// (A3/A7/A9) and the three sort modes, for the B200-native heterogeneous sort.
+//
+// Paper workflows (§III-D):
+//   BLINE       A -> HtoD -> GPUSort -> DtoH -> B
+//   BLINEMULTI  A -> HtoD -> GPUSort -> DtoH -> W -> Merge -> B, blocking
+//   PIPEDATA    A -> Stage -> HtoD -> GPUSort -> DtoH -> Stage -> W -> Merge -> B on n_s streams
+//               with pinned buffers of p_s elements
+//   PARMEMCPY   the Stage MCpy done by several host threads
+// B200 design: per GPU an uploader thread (Stage+HtoD, then the sort is enqueued on
+// the compute stream) and a downloader thread (DtoH+Stage into W), so HtoD, GPUSort and DtoH of
+// consecutive batches overlap on three streams; pinned inputs/outputs skip the staging copy; when
+// all runs fit in HBM they stay resident and are merged by the GPU (merge.cu) with the merged
+// chunks' DtoH overlapped with the merge.
+#include <cuda_runtime.h>
+#include <sys/mman.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <map>
+#include <mutex>
+#include <stdexcept>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/hsort.h"
+#include "internal.h"
+#include "pool.h"
+
+namespace hsort {
+void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, uint64_t* ranks);
+void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, bool out_f64,
+                int threads);
+}  // namespace hsort
+
+using namespace hsort;
+
+namespace {
+
+using Clock = std::chrono::steady_clock;
+inline double secs_since(Clock::time_point t0) {
+  return std::chrono::duration<double>(Clock::now() - t0).count();
+}
+
+thread_local std::string g_err = "";
+
+struct HsortError : std::runtime_error {
+  int code;
+  HsortError(int c, const std::string& m) : std::runtime_error(m), code(c) {}
+};
+
+#define CK(expr)                                                                              \
+  do {                                                                                        \
+    cudaError_t _e = (expr);                                                                  \
+    if (_e != cudaSuccess) {                                                                  \
+      throw HsortError(_e == cudaErrorMemoryAllocation ? HSORT_ERR_DEVICE_OOM : HSORT_ERR_CUDA, \
+                       std::string(#expr) + ": " + cudaGetErrorString(_e));                  \
+    }                                                                                         \
+  } while (0)
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  void reserve(size_t bytes) {
+    if (bytes <= cap) return;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    if (bytes == 0) return;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+      throw HsortError(HSORT_ERR_DEVICE_OOM, "cudaMalloc(" + std::to_string(bytes) + ") failed: " +
+                                                 cudaGetErrorString(e));
+    }
+    cap = bytes;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+  uint64_t* u64() const { return (uint64_t*)p; }
+};
+
+struct Options {
+  std::map<std::string, int64_t> v = {
+      {"n_s", 3},                    // device batch slots per GPU (default 3, see DESIGN)
+      {"p_s", 64ll << 20},           // pinned staging chunk bytes (reading A-6)
+      {"n_ring", 3},                 // pinned chunks per direction per GPU
+      {"memcpy_threads", 0},         // PARMEMCPY threads (0 = all host threads; 1 = serial MCpy)
+      {"merge_threads", 0},          // CPU merge threads (0 = all)
+      {"resident", -1},              // -1 auto, 0 force STREAM, 1 force RESIDENT
+      {"merge_gpu_permille", -1},    // A12 share f (per mille) of merge output on GPUs; -1 auto
+      {"pipeline", 1},               // 1 PIPEDATA overlap, 0 blocking BLINEMULTI ablation
+      {"merge_chunk", 1ll << 26},    // GPU merge output chunk (keys)
+      {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
+      {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
+  };
+  int64_t get(const char* k) const { return v.at(k); }
+};
+
+struct GpuCtx {
+  int dev = -1;
+  cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
+  RadixScratch rs;
+  DevBuf runs, alt, mout, ranks, off;
+  std::vector<char*> ring_in, ring_out;
+  uint64_t ring_bytes = 0;
+  std::vector<cudaEvent_t> ev_in, ev_out;
+  uint64_t in_next = 0;
+};
+
+struct State {
+  std::mutex m;
+  bool inited = false;
+  bool poisoned = false;
+  std::atomic<bool> busy{false};
+  std::vector<GpuCtx> gpus;
+  Options opt;
+  hsort_stats last{};
+  double t_init = 0;
+};
+State& S() {
+  static State s;
+  return s;
+}
+
+struct BusyGuard {
+  bool ok;
+  BusyGuard() { ok = !S().busy.exchange(true); }
+  ~BusyGuard() {
+    if (ok) S().busy.store(false);
+  }
+};
+
+template <class F>
+int guarded(F f) {
+  try {
+    return f();
+  } catch (const HsortError& e) {
+    g_err = e.what();
+    if (e.code == HSORT_ERR_CUDA) S().poisoned = true;
+    return e.code;
+  } catch (const std::bad_alloc&) {
+    g_err = "host allocation failed";
+    return HSORT_ERR_HOST_OOM;
+  } catch (const std::exception& e) {
+    g_err = e.what();
+    return HSORT_ERR_INTERNAL;
+  } catch (...) {
+    g_err = "unknown exception";
+    return HSORT_ERR_INTERNAL;
+  }
+}
+
+bool is_pinned(const void* p, uint64_t bytes) {
+  if (!p || bytes == 0) return false;
+  auto one = [](const void* q) {
+    cudaPointerAttributes a;
+    cudaError_t e = cudaPointerGetAttributes(&a, q);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    return a.type == cudaMemoryTypeHost;
+  };
+  return one(p) && one((const char*)p + bytes - 1);
+}
+
+// ---- staging ring (A2/A3, A7/A8) -------------------------------------------------------------
+struct Acc {  // per-thread stage accumulators
+  double t_stage = 0;
+  uint64_t h2d = 0, d2h = 0;
+};
+
+// Host -> device, through the pinned ring (PIPEDATA Stage + PARMEMCPY) unless direct.
+void upload(GpuCtx& g, void* d_dst, const void* h_src, uint64_t bytes, cudaStream_t st, bool direct,
+            int threads, Acc& acc) {
+  acc.h2d += bytes;
+  if (bytes == 0) return;
+  if (direct) {
+    CK(cudaMemcpyAsync(d_dst, h_src, bytes, cudaMemcpyHostToDevice, st));
+    return;
+  }
+  const uint64_t R = g.ring_in.size(), C = g.ring_bytes;
+  for (uint64_t o = 0; o < bytes; o += C) {
+    uint64_t len = std::min(C, bytes - o);
+    uint64_t s = g.in_next++ % R;
+    CK(cudaEventSynchronize(g.ev_in[s]));
+    auto t0 = Clock::now();
+    par_memcpy(g.ring_in[s], (const char*)h_src + o, len, threads);
+    acc.t_stage += secs_since(t0);
+    CK(cudaMemcpyAsync((char*)d_dst + o, g.ring_in[s], len, cudaMemcpyHostToDevice, st));
+    CK(cudaEventRecord(g.ev_in[s], st));
+  }
+}
+
+// Device -> host.  Direct: enqueued only (caller synchronises st).  Staged: returns when every
+// byte is in h_dst (DMA of chunk c overlaps the host copy-out of chunk c-1).
+void download(GpuCtx& g, void* h_dst, const void* d_src, uint64_t bytes, cudaStream_t st,
+              bool direct, int threads, Acc& acc) {
+  acc.d2h += bytes;
+  if (bytes == 0) return;
+  if (direct) {
+    CK(cudaMemcpyAsync(h_dst, d_src, bytes, cudaMemcpyDeviceToHost, st));
+    return;
+  }
+  const uint64_t R = g.ring_out.size(), C = g.ring_bytes;
+  const uint64_t nch = (bytes + C - 1) / C;
+  auto drain = [&](uint64_t c) {
+    uint64_t s = c % R, o = c * C, len = std::min(C, bytes - o);
+    CK(cudaEventSynchronize(g.ev_out[s]));
+    auto t0 = Clock::now();
+    par_memcpy((char*)h_dst + o, g.ring_out[s], len, threads);
+    acc.t_stage += secs_since(t0);
+  };
+  for (uint64_t c = 0; c < nch; ++c) {
+    if (c >= R) drain(c - R);
+    uint64_t s = c % R, o = c * C, len = std::min(C, bytes - o);
+    CK(cudaMemcpyAsync(g.ring_out[s], (const char*)d_src + o, len, cudaMemcpyDeviceToHost, st));
+    CK(cudaEventRecord(g.ev_out[s], st));
+  }
+  for (uint64_t c = (nch > R ? nch - R : 0); c < nch; ++c) drain(c);
+}
+
+struct EvPair {
+  cudaEvent_t a = nullptr, b = nullptr;
+  void make() {
+    CK(cudaEventCreate(&a));
+    CK(cudaEventCreate(&b));
+  }
+  void destroy() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+    a = b = nullptr;
+  }
+  double ms() const {
+    float t = 0;
+    if (cudaEventElapsedTime(&t, a, b) != cudaSuccess) {
+      cudaGetLastError();
+      return 0;
+    }
+    return t;
+  }
+};
+
+// ---- planner (A1) --------------------------------------------------------------------------
+constexpr double kLookbackBytesPerKey = 256.0 * 8.0 / kRadixTile;  // 0.5 B/key
+
+hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_bytes,
+                       const Options& opt) {
+  hsort_plan_t p{};
+  p.n = n;
+  p.n_gpus = n_gpus;
+  int n_s = (int)std::max<int64_t>(1, opt.get("n_s"));
+  uint64_t reserve = (uint64_t)std::max<int64_t>(0, opt.get("device_reserve_mb")) << 20;
+  uint64_t merge_buf = 2ull * (uint64_t)opt.get("merge_chunk") * 8;
+  uint64_t budget = device_bytes > reserve ? device_bytes - reserve : 0;
+  // single batch footprint: keys + alt + look-back
+  auto bline_bytes = [&](uint64_t b) { return (uint64_t)(b * (16.0 + kLookbackBytesPerKey)); };
+  uint64_t b_s;
+  if (batch_elems == 0) {
+    if (bline_bytes(n) <= budget) {
+      b_s = n;
+    } else {
+      // n_s resident slots + one shared alt buffer (b_s chosen to fill global memory)
+      double per = 8.0 * (n_s + 1) + kLookbackBytesPerKey;
+      b_s = (uint64_t)((double)budget / per);
+      b_s -= b_s % kRadixTile;
+      if (b_s == 0) b_s = kRadixTile;
+    }
+  } else {
+    b_s = std::min<uint64_t>(batch_elems, n ? n : 1);
+  }
+  if (b_s == 0) b_s = 1;
+  p.b_s = b_s;
+  p.n_b = n ? (n + b_s - 1) / b_s : 0;
+  p.last_batch = n ? n - (p.n_b - 1) * b_s : 0;
+  p.n_s = p.n_b <= 1 ? 1 : (int)std::min<uint64_t>((uint64_t)n_s, p.n_b);
+  int64_t res = opt.get("resident");
+  uint64_t resident_bytes = n * 8 + (uint64_t)(b_s * (8.0 + kLookbackBytesPerKey)) + merge_buf +
+                            ((n / kMergeTile + 2) * std::min<uint64_t>(p.n_b, kMaxMergeRuns) * 8);
+  if (p.n_b <= 1) {
+    p.mode = HSORT_MODE_BLINE;
+    p.device_bytes_per_gpu = bline_bytes(n);
+    p.n_gpus = std::min(n_gpus, 1);
+    if (n_gpus >= 1) p.n_gpus = 1;
+  } else if (n_gpus == 1 && p.n_b <= (uint64_t)kMaxMergeRuns &&
+             (res == 1 || (res == -1 && resident_bytes <= budget))) {
+    p.mode = HSORT_MODE_RESIDENT;
+    p.device_bytes_per_gpu = resident_bytes;
+  } else {
+    p.mode = HSORT_MODE_STREAM;
+    p.device_bytes_per_gpu = (uint64_t)(b_s * (8.0 * (p.n_s + 1) + kLookbackBytesPerKey));
+  }
+  p.host_bytes = (p.mode == HSORT_MODE_STREAM ? n * 8 : 0) +
+                 2ull * (uint64_t)opt.get("n_ring") * (uint64_t)opt.get("p_s") * (uint64_t)std::max(1, p.n_gpus);
+  p.batches_per_stream = p.n_b ? (double)p.n_b / ((double)p.n_s * std::max(1, p.n_gpus)) : 0.0;
+  return p;
+}
+
+// ---- mode drivers --------------------------------------------------------------------------
+struct CallCtx {
+  const void* A;
+  void* B;
+  uint64_t n;
+  bool f64;  // keys are float64 bits (transform on the GPU) vs raw uint64
+  hsort_plan_t plan;
+  bool direct_in, direct_out;
+  int mc_threads, merge_threads;
+  hsort_stats* st;
+};
+
+void sort_bline(GpuCtx& g, CallCtx& c) {
+  CK(cudaSetDevice(g.dev));
+  const uint64_t n = c.n;
+  g.runs.reserve(n * 8);
+  g.alt.reserve(n * 8);
+  Acc acc;
+  EvPair eh, es, ed;
+  eh.make();
+  es.make();
+  ed.make();
+  auto t0 = Clock::now();
+  CK(cudaEventRecord(eh.a, g.s_h2d));
+  upload(g, g.runs.p, c.A, n * 8, g.s_h2d, c.direct_in, c.mc_threads, acc);
+  CK(cudaEventRecord(eh.b, g.s_h2d));
+  CK(cudaStreamWaitEvent(g.s_comp, eh.b, 0));
+  CK(cudaEventRecord(es.a, g.s_comp));
+  CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), n, c.f64, c.f64, g.s_comp));
+  CK(cudaEventRecord(es.b, g.s_comp));
+  CK(cudaStreamWaitEvent(g.s_d2h, es.b, 0));
+  CK(cudaEventRecord(ed.a, g.s_d2h));
+  download(g, c.B, g.runs.p, n * 8, g.s_d2h, c.direct_out, c.mc_threads, acc);
+  CK(cudaEventRecord(ed.b, g.s_d2h));
+  CK(cudaStreamSynchronize(g.s_d2h));
+  c.st->t_sort_phase = secs_since(t0);
+  c.st->t_h2d = eh.ms() / 1e3;
+  c.st->t_gpu_sort = es.ms() / 1e3;
+  c.st->t_d2h = ed.ms() / 1e3;
+  c.st->t_stage = acc.t_stage;
+  c.st->bytes_h2d = acc.h2d;
+  c.st->bytes_d2h = acc.d2h;
+  c.st->passes_run = g.rs.h_plan->num_active;
+  c.st->passes_skipped = 8 - g.rs.h_plan->num_active;
+  eh.destroy();
+  es.destroy();
+  ed.destroy();
+}
+
+void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std::vector<uint64_t>& h_off,
+                       Acc& acc, double* t_merge_gpu) {
+  const int k = (int)h_off.size() - 1;
+  const uint64_t total = h_off[k] - h_off[0];
+  g.off.reserve((k + 1) * 8);
+  CK(cudaMemcpyAsync(g.off.p, h_off.data(), (k + 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
+  const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
+  g.ranks.reserve((tiles + 1) * (uint64_t)k * 8);
+  EvPair em;
+  em.make();
+  CK(cudaEventRecord(em.a, g.s_comp));
+  CK(merge_corank(d_runs, g.off.u64(), k, total, kMergeTile, tiles + 1, g.ranks.u64(), g.s_comp));
+  uint64_t ctiles = std::max<uint64_t>(1, (uint64_t)c.plan.n ? (uint64_t)S().opt.get("merge_chunk") / kMergeTile : 1);
+  const uint64_t chunk = ctiles * kMergeTile;
+  const uint64_t nch = (total + chunk - 1) / chunk;
+  const uint64_t slots = nch > 1 ? 2 : 1;
+  g.mout.reserve(slots * chunk * 8);
+  std::vector<cudaEvent_t> ev_done(slots), ev_free(slots);
+  for (uint64_t s = 0; s < slots; ++s) {
+    CK(cudaEventCreateWithFlags(&ev_done[s], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ev_free[s], cudaEventDisableTiming));
+    CK(cudaEventRecord(ev_free[s], g.s_d2h));
+  }
+  char* B = (char*)c.B;
+  auto enqueue_merge = [&](uint64_t ch) {
+    uint64_t s = ch % slots;
+    uint64_t tb = ch * ctiles, tc = std::min(ctiles, tiles - tb);
+    CK(cudaStreamWaitEvent(g.s_comp, ev_free[s], 0));
+    CK(merge_tiles(d_runs, g.off.u64(), k, total, g.ranks.u64(), tb, tc,
+                   g.mout.u64() + s * chunk, ch * chunk, c.f64, g.s_comp));
+    CK(cudaEventRecord(ev_done[s], g.s_comp));
+  };
+  enqueue_merge(0);
+  for (uint64_t ch = 0; ch < nch; ++ch) {
+    if (ch + 1 < nch) enqueue_merge(ch + 1);
+    if (ch + 1 == nch) CK(cudaEventRecord(em.b, g.s_comp));
+    uint64_t s = ch % slots;
+    uint64_t o = ch * chunk, len = std::min(chunk, total - o);
+    CK(cudaStreamWaitEvent(g.s_d2h, ev_done[s], 0));
+    download(g, B + o * 8, g.mout.u64() + s * chunk, len * 8, g.s_d2h, c.direct_out, c.mc_threads, acc);
+    CK(cudaEventRecord(ev_free[s], g.s_d2h));
+  }
+  CK(cudaStreamSynchronize(g.s_d2h));
+  CK(cudaStreamSynchronize(g.s_comp));
+  *t_merge_gpu += em.ms() / 1e3;
+  em.destroy();
+  for (uint64_t s = 0; s < slots; ++s) {
+    cudaEventDestroy(ev_done[s]);
+    cudaEventDestroy(ev_free[s]);
+  }
+}
+
+void sort_resident(GpuCtx& g, CallCtx& c) {
+  CK(cudaSetDevice(g.dev));
+  const uint64_t n = c.n, b_s = c.plan.b_s, n_b = c.plan.n_b;
+  g.runs.reserve(n * 8);
+  g.alt.reserve(b_s * 8);
+  Acc acc;
+  std::vector<EvPair> eh(n_b), es(n_b);
+  for (auto& e : eh) e.make();
+  for (auto& e : es) e.make();
+  auto t0 = Clock::now();
+  int passes = 0;
+  for (uint64_t i = 0; i < n_b; ++i) {
+    uint64_t o = i * b_s, len = std::min(b_s, n - o);
+    CK(cudaEventRecord(eh[i].a, g.s_h2d));
+    upload(g, g.runs.u64() + o, (const char*)c.A + o * 8, len * 8, g.s_h2d, c.direct_in, c.mc_threads, acc);
+    CK(cudaEventRecord(eh[i].b, g.s_h2d));
+    CK(cudaStreamWaitEvent(g.s_comp, eh[i].b, 0));
+    CK(cudaEventRecord(es[i].a, g.s_comp));
+    CK(radix_sort(g.rs, g.runs.u64() + o, g.runs.u64() + o, g.alt.u64(), len, c.f64, false, g.s_comp));
+    CK(cudaEventRecord(es[i].b, g.s_comp));
+  }
+  CK(cudaStreamSynchronize(g.s_comp));
+  passes = g.rs.h_plan->num_active;  // plan of the last batch
+  c.st->t_sort_phase = secs_since(t0);
+  auto t1 = Clock::now();
+  std::vector<uint64_t> h_off(n_b + 1);
+  for (uint64_t i = 0; i <= n_b; ++i) h_off[i] = std::min(i * b_s, n);
+  double tmg = 0;
+  gpu_merge_to_host(g, c, g.runs.u64(), h_off, acc, &tmg);
+  c.st->t_merge_phase = secs_since(t1);
+  c.st->t_merge_gpu = tmg;
+  c.st->merge_gpu_fraction = 1.0;
+  for (uint64_t i = 0; i < n_b; ++i) {
+    c.st->t_h2d += eh[i].ms() / 1e3;
+    c.st->t_gpu_sort += es[i].ms() / 1e3;
+  }
+  c.st->t_stage = acc.t_stage;
+  c.st->bytes_h2d = acc.h2d;
+  c.st->bytes_d2h = acc.d2h;
+  c.st->passes_run = passes;
+  c.st->passes_skipped = 8 - passes;
+  for (auto& e : eh) e.destroy();
+  for (auto& e : es) e.destroy();
+}
+
+// STREAM mode: batches -> W (host) through per-GPU uploader/downloader threads, then the CPU
+// multiway merge W -> B.
+void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
+  const uint64_t n = c.n, b_s = c.plan.b_s, n_b = c.plan.n_b;
+  const int n_s = std::max(1, c.plan.n_s);
+  const bool pipelined = S().opt.get("pipeline") != 0;
+  // W: working memory for the sorted sublists; transformed uint64 keys
+  uint64_t* W = nullptr;
+  {
+    size_t bytes = n * 8;
+    void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+    if (p == MAP_FAILED) throw HsortError(HSORT_ERR_HOST_OOM, "mmap W failed");
+    madvise(p, bytes, MADV_HUGEPAGE);
+    W = (uint64_t*)p;
+  }
+  struct WFree {
+    void* p;
+    size_t b;
+    ~WFree() { munmap(p, b); }
+  } wfree{W, n * 8};
+
+  std::atomic<uint64_t> next_batch{0};
+  std::mutex err_m;
+  std::string err_msg;
+  int err_code = 0;
+  std::atomic<bool> failed{false};
+  auto fail = [&](int code, const std::string& m) {
+    std::lock_guard<std::mutex> gd(err_m);
+    if (!err_code) {
+      err_code = code;
+      err_msg = m;
+    }
+    failed = true;
+  };
+  struct PerGpu {
+    Acc up, down;
+    double t_h2d = 0, t_sort = 0, t_d2h = 0;
+    int passes = 0;
+  };
+  std::vector<PerGpu> pg(gs.size());
+  auto t0 = Clock::now();
+
+  auto gpu_main = [&](size_t gi) {
+    GpuCtx& g = *gs[gi];
+    PerGpu& P = pg[gi];
+    try {
+      CK(cudaSetDevice(g.dev));
+      g.runs.reserve((uint64_t)n_s * b_s * 8);
+      g.alt.reserve(b_s * 8);
+      std::vector<cudaEvent_t> ev_up(n_s), ev_sorted(n_s);
+      for (int s = 0; s < n_s; ++s) {
+        CK(cudaEventCreateWithFlags(&ev_up[s], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&ev_sorted[s], cudaEventDisableTiming));
+      }
+      struct Item {
+        uint64_t batch;
+        int slot;
+        EvPair eh, es, ed;
+      };
+      std::deque<Item*> fifo;
+      std::vector<Item*> all;
+      std::mutex m;
+      std::condition_variable cv;
+      bool up_done = false;
+      std::vector<int> slot_busy(n_s, 0);
+      if (!pipelined) {
+        // BLINEMULTI: blocking, one stream, no overlap
+        while (!failed) {
+          uint64_t i = next_batch.fetch_add(1);
+          if (i >= n_b) break;
+          uint64_t o = i * b_s, len = std::min(b_s, n - o);
+          Item* it = new Item{i, 0, {}, {}, {}};
+          all.push_back(it);
+          it->eh.make();
+          it->es.make();
+          it->ed.make();
+          CK(cudaEventRecord(it->eh.a, g.s_comp));
+          upload(g, g.runs.p, (const char*)c.A + o * 8, len * 8, g.s_comp, c.direct_in, c.mc_threads, P.up);
+          CK(cudaEventRecord(it->eh.b, g.s_comp));
+          CK(cudaEventRecord(it->es.a, g.s_comp));
+          CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), len, c.f64, false, g.s_comp));
+          CK(cudaEventRecord(it->es.b, g.s_comp));
+          CK(cudaEventRecord(it->ed.a, g.s_comp));
+          download(g, W + o, g.runs.p, len * 8, g.s_comp, false, c.mc_threads, P.down);
+          CK(cudaEventRecord(it->ed.b, g.s_comp));
+          CK(cudaStreamSynchronize(g.s_comp));
+          P.passes += g.rs.h_plan->num_active;
+        }
+      } else {
+        std::thread downloader([&] {
+          try {
+            CK(cudaSetDevice(g.dev));
+            while (true) {
+              Item* it;
+              {
+                std::unique_lock<std::mutex> lk(m);
+                cv.wait(lk, [&] { return !fifo.empty() || up_done || failed; });
+                if (fifo.empty()) break;
+                it = fifo.front();
+                fifo.pop_front();
+              }
+              uint64_t o = it->batch * b_s, len = std::min(b_s, n - o);
+              CK(cudaStreamWaitEvent(g.s_d2h, ev_sorted[it->slot], 0));
+              CK(cudaEventRecord(it->ed.a, g.s_d2h));
+              download(g, W + o, g.runs.u64() + (uint64_t)it->slot * b_s, len * 8, g.s_d2h, false,
+                       c.mc_threads, P.down);
+              CK(cudaEventRecord(it->ed.b, g.s_d2h));
+              CK(cudaEventSynchronize(it->ed.b));
+              {
+                std::lock_guard<std::mutex> gd(m);
+                slot_busy[it->slot] = 0;
+              }
+              cv.notify_all();
+            }
+          } catch (const HsortError& e) {
+            fail(e.code, e.what());
+            cv.notify_all();
+          }
+        });
+        uint64_t local = 0;
+        try {
+          while (!failed) {
+            uint64_t i = next_batch.fetch_add(1);
+            if (i >= n_b) break;
+            int s = (int)(local++ % n_s);
+            {
+              std::unique_lock<std::mutex> lk(m);
+              cv.wait(lk, [&] { return !slot_busy[s] || failed; });
+              if (failed) break;
+              slot_busy[s] = 1;
+            }
+            uint64_t o = i * b_s, len = std::min(b_s, n - o);
+            Item* it = new Item{i, s, {}, {}, {}};
+            all.push_back(it);
+            it->eh.make();
+            it->es.make();
+            it->ed.make();
+            uint64_t* dslot = g.runs.u64() + (uint64_t)s * b_s;
+            CK(cudaEventRecord(it->eh.a, g.s_h2d));
+            upload(g, dslot, (const char*)c.A + o * 8, len * 8, g.s_h2d, c.direct_in, c.mc_threads, P.up);
+            CK(cudaEventRecord(it->eh.b, g.s_h2d));
+            CK(cudaStreamWaitEvent(g.s_comp, it->eh.b, 0));
+            CK(cudaEventRecord(it->es.a, g.s_comp));
+            CK(radix_sort(g.rs, dslot, dslot, g.alt.u64(), len, c.f64, false, g.s_comp));
+            CK(cudaEventRecord(it->es.b, g.s_comp));
+            CK(cudaEventRecord(ev_sorted[s], g.s_comp));
+            {
+              std::lock_guard<std::mutex> gd(m);
+              fifo.push_back(it);
+            }
+            cv.notify_all();
+          }
+        } catch (const HsortError& e) {
+          fail(e.code, e.what());
+        }
+        {
+          std::lock_guard<std::mutex> gd(m);
+          up_done = true;
+        }
+        cv.notify_all();
+        downloader.join();
+        CK(cudaStreamSynchronize(g.s_comp));
+        P.passes += g.rs.h_plan->num_active;
+      }
+      CK(cudaDeviceSynchronize());
+      for (Item* it : all) {
+        P.t_h2d += it->eh.ms() / 1e3;
+        P.t_sort += it->es.ms() / 1e3;
+        P.t_d2h += it->ed.ms() / 1e3;
+        it->eh.destroy();
+        it->es.destroy();
+        it->ed.destroy();
+        delete it;
+      }
+      for (int s = 0; s < n_s; ++s) {
+        cudaEventDestroy(ev_up[s]);
+        cudaEventDestroy(ev_sorted[s]);
+      }
+    } catch (const HsortError& e) {
+      fail(e.code, e.what());
+    }
+  };
+  if (gs.size() == 1) {
+    gpu_main(0);
+  } else {
+    std::vector<std::thread> th;
+    for (size_t gi = 0; gi < gs.size(); ++gi) th.emplace_back(gpu_main, gi);
+    for (auto& t : th) t.join();
+  }
+  if (failed) throw HsortError(err_code ? err_code : HSORT_ERR_INTERNAL, err_msg);
+  c.st->t_sort_phase = secs_since(t0);
+  for (auto& P : pg) {
+    c.st->t_h2d += P.t_h2d;
+    c.st->t_gpu_sort += P.t_sort;
+    c.st->t_d2h += P.t_d2h;
+    c.st->t_stage += P.up.t_stage + P.down.t_stage;
+    c.st->bytes_h2d += P.up.h2d;
+    c.st->bytes_d2h += P.down.d2h;
+    c.st->passes_run += P.passes;
+  }
+  // Merge: CPU multiway merge of the n_b runs in W into B.
+  auto t1 = Clock::now();
+  std::vector<uint64_t> off(n_b + 1);
+  for (uint64_t i = 0; i <= n_b; ++i) off[i] = std::min(i * b_s, n);
+  host_merge(W, off.data(), (int)n_b, (uint64_t*)c.B, c.f64, c.merge_threads);
+  c.st->t_merge_cpu = secs_since(t1);
+  c.st->t_merge_phase = c.st->t_merge_cpu;
+  c.st->merge_gpu_fraction = 0.0;
+}
+
+void ctx_create(GpuCtx& g, int dev, const Options& opt) {
+  g.dev = dev;
+  CK(cudaSetDevice(dev));
+  CK(cudaStreamCreateWithFlags(&g.s_h2d, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&g.s_comp, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&g.s_d2h, cudaStreamNonBlocking));
+  int R = (int)std::max<int64_t>(2, opt.get("n_ring"));
+  g.ring_bytes = (uint64_t)std::max<int64_t>(1 << 20, opt.get("p_s"));
+  g.ring_bytes = (g.ring_bytes + 4095) & ~4095ull;
+  for (int i = 0; i < R; ++i) {
+    void* p = nullptr;
+    CK(cudaHostAlloc(&p, g.ring_bytes, cudaHostAllocDefault));
+    g.ring_in.push_back((char*)p);
+    CK(cudaHostAlloc(&p, g.ring_bytes, cudaHostAllocDefault));
+    g.ring_out.push_back((char*)p);
+    cudaEvent_t e;
+    CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    g.ev_in.push_back(e);
+    CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    g.ev_out.push_back(e);
+  }
+  CK(radix_scratch_reserve(g.rs, kRadixTile));
+}
+
+void ctx_destroy(GpuCtx& g) {
+  if (g.dev < 0) return;
+  cudaSetDevice(g.dev);
+  cudaDeviceSynchronize();
+  for (auto p : g.ring_in) cudaFreeHost(p);
+  for (auto p : g.ring_out) cudaFreeHost(p);
+  for (auto e : g.ev_in) cudaEventDestroy(e);
+  for (auto e : g.ev_out) cudaEventDestroy(e);
+  g.runs.release();
+  g.alt.release();
+  g.mout.release();
+  g.ranks.release();
+  g.off.release();
+  radix_scratch_release(g.rs);
+  if (g.s_h2d) cudaStreamDestroy(g.s_h2d);
+  if (g.s_comp) cudaStreamDestroy(g.s_comp);
+  if (g.s_d2h) cudaStreamDestroy(g.s_d2h);
+  g = GpuCtx();
+}
+
+GpuCtx& current_ctx() {
+  int dev = 0;
+  CK(cudaGetDevice(&dev));
+  for (auto& g : S().gpus)
+    if (g.dev == dev) return g;
+  throw HsortError(HSORT_ERR_INVALID, "current device not managed by hsort_init");
+}
+
+int check_ready() {
+  if (!S().inited) {
+    g_err = "hsort_init() has not been called";
+    return HSORT_ERR_NOT_INITIALIZED;
+  }
+  if (S().poisoned) {
+    g_err = "library poisoned by an earlier CUDA error; call hsort_finalize()";
+    return HSORT_ERR_CUDA;
+  }
+  return HSORT_OK;
+}
+
+int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus, bool f64) {
+  int rc = check_ready();
+  if (rc) return rc;
+  BusyGuard busy;
+  if (!busy.ok) {
+    g_err = "hsort_sort already running";
+    return HSORT_ERR_BUSY;
+  }
+  if (n == 0) {
+    S().last = hsort_stats{};
+    return HSORT_OK;
+  }
+  if (!A || !B) {
+    g_err = "null A or B with n > 0";
+    return HSORT_ERR_INVALID;
+  }
+  if (((uintptr_t)A & 7) || ((uintptr_t)B & 7)) {
+    g_err = "A and B must be 8-byte aligned";
+    return HSORT_ERR_INVALID;
+  }
+  const uintptr_t a0 = (uintptr_t)A, b0 = (uintptr_t)B, bytes = n * 8;
+  if (A != B && a0 < b0 + bytes && b0 < a0 + bytes) {
+    g_err = "A and B partially overlap";
+    return HSORT_ERR_INVALID;
+  }
+  const int vis = (int)S().gpus.size();
+  if (n_gpus < 0 || n_gpus > vis) {
+    g_err = "n_gpus must be in [0, " + std::to_string(vis) + "]";
+    return HSORT_ERR_INVALID;
+  }
+  if (n_gpus == 0) n_gpus = vis;
+  return guarded([&]() -> int {
+    auto t0 = Clock::now();
+    GpuCtx& g0 = S().gpus[0];
+    CK(cudaSetDevice(g0.dev));
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    // budget: free memory plus what this library already holds on the device
+    uint64_t held = g0.runs.cap + g0.alt.cap + g0.mout.cap + g0.ranks.cap;
+    hsort_plan_t plan = make_plan(n, batch_elems, n_gpus, fr + held, S().opt);
+    hsort_stats st{};
+    st.n = n;
+    st.b_s = plan.b_s;
+    st.n_b = plan.n_b;
+    st.n_gpus = plan.n_gpus;
+    st.n_s = plan.n_s;
+    st.mode = plan.mode;
+    st.merge_k = (int)plan.n_b;
+    st.t_init = S().t_init;
+    CallCtx c;
+    c.A = A;
+    c.B = B;
+    c.n = n;
+    c.f64 = f64;
+    c.plan = plan;
+    c.direct_in = is_pinned(A, bytes);
+    c.direct_out = is_pinned(B, bytes);
+    c.mc_threads = (int)S().opt.get("memcpy_threads");
+    c.merge_threads = (int)S().opt.get("merge_threads");
+    c.st = &st;
+    st.direct_in = c.direct_in;
+    st.direct_out = c.direct_out;
+    if (plan.mode == HSORT_MODE_BLINE) {
+      sort_bline(g0, c);
+    } else if (plan.mode == HSORT_MODE_RESIDENT) {
+      sort_resident(g0, c);
+    } else {
+      // in-place (B == A) is safe: W holds the runs, B is written only by the merge
+      std::vector<GpuCtx*> gs;
+      for (int i = 0; i < plan.n_gpus; ++i) gs.push_back(&S().gpus[i]);
+      sort_stream(gs, c);
+    }
+    st.t_total = secs_since(t0);
+    S().last = st;
+    return HSORT_OK;
+  });
+}
+
+}  // namespace
+
+// =============================================================================================
+extern "C" {
+
+const char* hsort_last_error(void) { return g_err.c_str(); }
+const char* hsort_version(void) { return "hsort-b200 0.1 (sm_100a)"; }
+
+int hsort_device_count(void) {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
+}
+
+int hsort_init(void) {
+  std::lock_guard<std::mutex> lk(S().m);
+  if (S().inited) {
+    g_err = "hsort_init called twice";
+    return HSORT_ERR_BUSY;
+  }
+  return guarded([&]() -> int {
+    auto t0 = Clock::now();
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0) {
+      cudaGetLastError();
+      throw HsortError(HSORT_ERR_CUDA, std::string("no CUDA device: ") + cudaGetErrorString(e));
+    }
+    S().gpus.resize(n);
+    try {
+      for (int d = 0; d < n; ++d) ctx_create(S().gpus[d], d, S().opt);
+    } catch (...) {
+      for (auto& g : S().gpus) ctx_destroy(g);
+      S().gpus.clear();
+      throw;
+    }
+    host_pool();
+    if (S().opt.get("kernel_timing"))
+      for (auto& g : S().gpus) {
+        CK(cudaSetDevice(g.dev));
+        CK(radix_set_timing(g.rs, true));
+      }
+    S().inited = true;
+    S().poisoned = false;
+    S().t_init = secs_since(t0);
+    return HSORT_OK;
+  });
+}
+
+int hsort_finalize(void) {
+  std::lock_guard<std::mutex> lk(S().m);
+  for (auto& g : S().gpus) ctx_destroy(g);
+  S().gpus.clear();
+  S().inited = false;
+  S().poisoned = false;
+  return HSORT_OK;
+}
+
+int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_elems, int n_gpus) {
+  return do_sort(A_host, B_host, n, batch_elems, n_gpus, true);
+}
+
+int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_t batch_elems,
+                   int n_gpus) {
+  return do_sort(A_host, B_host, n, batch_elems, n_gpus, false);
+}
+
+int hsort_set_option(const char* key, int64_t value) {
+  if (!key || !S().opt.v.count(key)) {
+    g_err = std::string("unknown option ") + (key ? key : "(null)");
+    return HSORT_ERR_INVALID;
+  }
+  std::string k = key;
+  if ((k == "n_s" || k == "n_ring") && value < 1) return g_err = k + " must be >= 1", HSORT_ERR_INVALID;
+  if (k == "p_s" && value < (1 << 20)) return g_err = "p_s must be >= 1 MiB", HSORT_ERR_INVALID;
+  if (k == "merge_chunk" && value < kMergeTile) return g_err = "merge_chunk too small", HSORT_ERR_INVALID;
+  if (k == "merge_gpu_permille" && (value < -1 || value > 1000)) return g_err = "bad permille", HSORT_ERR_INVALID;
+  if (k == "resident" && (value < -1 || value > 1)) return g_err = "resident in {-1,0,1}", HSORT_ERR_INVALID;
+  if (S().inited && (k == "p_s" || k == "n_ring")) {
+    g_err = k + " must be set before hsort_init";
+    return HSORT_ERR_BUSY;
+  }
+  S().opt.v[k] = value;
+  if (k == "kernel_timing") {
+    return guarded([&]() -> int {
+      for (auto& g : S().gpus) {
+        CK(cudaSetDevice(g.dev));
+        CK(radix_set_timing(g.rs, value != 0));
+      }
+      return HSORT_OK;
+    });
+  }
+  return HSORT_OK;
+}
+
+int hsort_get_kernel_times(float* ms, int max_entries, int* num_active_passes) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (!ms || max_entries < 0) return g_err = "bad arguments", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    if (num_active_passes) *num_active_passes = g.rs.h_plan ? g.rs.h_plan->num_active : 0;
+    return radix_kernel_times(g.rs, ms, max_entries);
+  });
+}
+
+int hsort_get_option(const char* key, int64_t* value) {
+  if (!key || !value || !S().opt.v.count(key)) {
+    g_err = "unknown option";
+    return HSORT_ERR_INVALID;
+  }
+  *value = S().opt.v[key];
+  return HSORT_OK;
+}
+
+int hsort_get_stats(hsort_stats* out) {
+  if (!out) return HSORT_ERR_INVALID;
+  *out = S().last;
+  return HSORT_OK;
+}
+
+int hsort_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_bytes,
+               hsort_plan_t* out) {
+  if (!out || n_gpus < 0) {
+    g_err = "bad arguments";
+    return HSORT_ERR_INVALID;
+  }
+  return guarded([&]() -> int {
+    uint64_t db = device_bytes;
+    int ng = n_gpus;
+    if (db == 0 || ng == 0) {
+      int cnt = hsort_device_count();
+      if (cnt == 0) throw HsortError(HSORT_ERR_CUDA, "no CUDA device to query");
+      if (ng == 0) ng = cnt;
+      if (db == 0) {
+        size_t fr = 0, tot = 0;
+        CK(cudaMemGetInfo(&fr, &tot));
+        db = fr;
+      }
+    }
+    *out = make_plan(n, batch_elems, ng, db, S().opt);
+    return HSORT_OK;
+  });
+}
+
+int hsort_sort_device(const double* d_in, double* d_out, uint64_t n, void* stream) {
+  return hsort_sort_device_keys((const uint64_t*)d_in, (uint64_t*)d_out, n, 1, 1, stream);
+}
+
+int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, int in_f64,
+                           int out_f64, void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (n && (!d_in || !d_out)) return g_err = "null device pointer", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    g.alt.reserve(n * 8);
+    CK(radix_sort(g.rs, d_in, d_out, g.alt.u64(), n, in_f64 != 0, out_f64 != 0,
+                  (cudaStream_t)stream));
+    return HSORT_OK;
+  });
+}
+
+int hsort_device_histograms(const uint64_t* d_keys, uint64_t n, int in_f64, uint64_t* d_hist,
+                            void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    CK(radix_histograms(g.rs, d_keys, n, in_f64 != 0, d_hist, (cudaStream_t)stream));
+    CK(cudaStreamSynchronize((cudaStream_t)stream));
+    return HSORT_OK;
+  });
+}
+
+int hsort_device_radix_pass(const uint64_t* d_src, uint64_t* d_dst, uint64_t n, int digit,
+                            void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (digit < 0 || digit > 7) return g_err = "digit must be 0..7", HSORT_ERR_INVALID;
+  if (d_src == d_dst && n) return g_err = "src and dst must differ", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    CK(radix_one_pass(g.rs, d_src, d_dst, n, digit, (cudaStream_t)stream));
+    CK(cudaStreamSynchronize((cudaStream_t)stream));
+    return HSORT_OK;
+  });
+}
+
+int hsort_device_corank(const uint64_t* d_keys, const uint64_t* h_off, int k, uint64_t step,
+                        uint64_t n_bounds, uint64_t* d_ranks, void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (k < 1 || k > kMaxMergeRuns || !h_off) return g_err = "k must be 1..1024", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    g.off.reserve((k + 1) * 8);
+    cudaStream_t st = (cudaStream_t)stream;
+    CK(cudaMemcpyAsync(g.off.p, h_off, (k + 1) * 8, cudaMemcpyHostToDevice, st));
+    CK(merge_corank(d_keys, g.off.u64(), k, h_off[k] - h_off[0], step, n_bounds, d_ranks, st));
+    CK(cudaStreamSynchronize(st));
+    return HSORT_OK;
+  });
+}
+
+int hsort_device_merge(const uint64_t* d_keys, const uint64_t* h_off, int k, uint64_t* d_out,
+                       int out_f64, void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (k < 1 || k > kMaxMergeRuns || !h_off) return g_err = "k must be 1..1024", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    cudaStream_t st = (cudaStream_t)stream;
+    const uint64_t total = h_off[k] - h_off[0];
+    if (total == 0) return HSORT_OK;
+    g.off.reserve((k + 1) * 8);
+    CK(cudaMemcpyAsync(g.off.p, h_off, (k + 1) * 8, cudaMemcpyHostToDevice, st));
+    const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
+    g.ranks.reserve((tiles + 1) * (uint64_t)k * 8);
+    CK(merge_corank(d_keys, g.off.u64(), k, total, kMergeTile, tiles + 1, g.ranks.u64(), st));
+    CK(merge_tiles(d_keys, g.off.u64(), k, total, g.ranks.u64(), 0, tiles, d_out, 0, out_f64 != 0, st));
+    CK(cudaStreamSynchronize(st));
+    return HSORT_OK;
+  });
+}
+
+int hsort_par_memcpy(void* dst, const void* src, uint64_t bytes, int threads) {
+  if (bytes && (!dst || !src)) return g_err = "null pointer", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    par_memcpy(dst, src, bytes, threads > 0 ? threads : (int)S().opt.get("memcpy_threads"));
+    return HSORT_OK;
+  });
+}
+
+int hsort_host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, int out_f64,
+                     int threads) {
+  if (k < 1 || !off || (off[k] > off[0] && (!keys || !out)))
+    return g_err = "bad arguments", HSORT_ERR_INVALID;
+  for (int j = 0; j < k; ++j)
+    if (off[j + 1] < off[j]) return g_err = "offsets must be non-decreasing", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    host_merge(keys, off, k, out, out_f64 != 0, threads > 0 ? threads : (int)S().opt.get("merge_threads"));
+    return HSORT_OK;
+  });
+}
+
+int hsort_host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o,
+                      uint64_t* ranks) {
+  if (k < 1 || !off || !ranks) return g_err = "bad arguments", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    std::vector<uint64_t> o2(k + 1);
+    for (int j = 0; j <= k; ++j) o2[j] = off[j] - off[0];
+    host_corank(keys + off[0], o2.data(), k, o, ranks);
+    return HSORT_OK;
+  });
+}
+
+uint64_t hsort_pipemerge_count(uint64_t n_b, int n_gpus) {
+  // P:430-454 (reading A-9): one GPU -> floor((n_b-1)/2); two or more -> floor(n_b/(2 n_GPU))
+  if (n_b == 0) return 0;
+  if (n_gpus <= 1) return (n_b - 1) / 2;
+  return n_b / (2 * (uint64_t)n_gpus);
+}
+
+}  // extern "C"

@@ -1,0 +1,80 @@
+// internal.h — declarations shared by the library's own translation units (never by oracle/).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace hsort {
+
+// ---- radix sort (radix.cu) -----------------------------------------------------------------
+// Device pass plan written by K2 (k_scan_plan) and read by every K3 launch, so the whole sort is
+// stream-ordered with no host round trip (trivial digits are skipped on the device).
+// Buffer ids: 0 = in, 1 = out, 2 = tmp.
+struct RadixPlan {
+  int32_t num_active;   // P_eff: number of non-trivial digits
+  int32_t digit[8];     // active digits, ascending (LSD order)
+  int32_t src[8];       // buffer id read by pass p
+  int32_t dst[8];       // buffer id written by pass p
+  int32_t copy_src;     // -1: no final copy; else buffer id copied to out (with conversion)
+  int32_t copy_in_f64;  // conversion of the final copy: source is float64 bits
+  int32_t copy_out_f64; // conversion of the final copy: destination is float64 bits
+  int32_t pad;
+};
+
+struct RadixScratch {
+  // small block (one allocation, zeroed per sort): hist[8*256] | bin_base[8*256] | plan |
+  // tile counters[8]
+  void* small = nullptr;
+  uint64_t* hist = nullptr;
+  uint64_t* bin_base = nullptr;
+  RadixPlan* plan = nullptr;
+  uint32_t* tile_ctr = nullptr;
+  size_t small_zero_bytes = 0;  // bytes of `small` zeroed per sort (hist + plan + counters)
+  // decoupled look-back status words, [max_tiles][256] uint64 (flag | epoch | count)
+  uint64_t* lookback = nullptr;
+  uint64_t max_tiles = 0;
+  uint32_t epoch = 0;
+  int device = -1;
+  // host-pinned mirror of the plan, read back for statistics
+  RadixPlan* h_plan = nullptr;
+  // optional per-kernel CUDA events (hsort_set_option("kernel_timing", 1)):
+  // ev[0] before K1, ev[1] after K1, ev[2] after K2, ev[3+p] after pass p, ev[11] after copy
+  bool timing = false;
+  cudaEvent_t ev[12] = {};
+};
+constexpr int kNumKernelEvents = 12;
+
+constexpr int kRadixTile = 4096;  // keys per onesweep tile (THREADS x ITEMS), see radix.cu
+
+cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n);
+cudaError_t radix_set_timing(RadixScratch& s, bool on);
+// durations (ms) of [K1, K2, pass0..pass7, final copy] of the last timed sort; returns count
+int radix_kernel_times(RadixScratch& s, float* ms, int max);
+void radix_scratch_release(RadixScratch& s);
+
+// GPUSort of n keys: out = sorted(in).  tmp: n-element scratch (must differ from in and out).
+// in == out allowed.  in_f64: input holds float64 bits (key transform fused into the first
+// pass).  out_f64: store float64 bits (inverse transform fused into the last pass).
+cudaError_t radix_sort(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,
+                       uint64_t n, bool in_f64, bool out_f64, cudaStream_t st);
+// K1 only (hist zeroed first); d_hist receives 8*256 counts.
+cudaError_t radix_histograms(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
+                             uint64_t* d_hist, cudaStream_t st);
+// K1 + K2 + one K3 pass by `digit` over raw uint64 keys, src -> dst.
+cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, uint64_t n,
+                           int digit, cudaStream_t st);
+
+// ---- GPU merge (merge.cu) ------------------------------------------------------------------
+constexpr int kMergeTile = 4096;  // output keys per merge CTA
+constexpr int kMaxMergeRuns = 1024;
+
+// K4: ranks[(b)*k + j] for b in [0, n_bounds): co-ranks of o_b = min(b*step, total).
+cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
+                         uint64_t step, uint64_t n_bounds, uint64_t* ranks, cudaStream_t st);
+// K5: merge tiles [tile_begin, tile_begin + tile_count) (tile t = output [t*kMergeTile, ...)),
+// given ranks for boundaries of step kMergeTile; writes out[o - out_origin].
+cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
+                        const uint64_t* ranks, uint64_t tile_begin, uint64_t tile_count,
+                        uint64_t* out, uint64_t out_origin, bool out_f64, cudaStream_t st);
+
+}  // namespace hsort

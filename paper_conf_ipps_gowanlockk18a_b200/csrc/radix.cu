@@ -1,0 +1,558 @@
+// radix.cu — GPUSort (§III-B) re-designed for sm_100a.
+//
+// The paper sorts each batch with Thrust (a CUB radix sort, out-of-place, 2x memory).
+// Here the same step is a hand-written LSD onesweep radix sort over 64-bit keys:
+//
+//   K1 k_hist      one streaming read of the batch -> all 8 digit histograms (8 x 256), with the
+//                  float64 -> order-preserving uint64 key transform applied in registers.
+//   K2 k_scan_plan exclusive scans -> bin bases; digits with one non-empty bin are "trivial" and
+//                  skipped; writes the device pass plan (src/dst ping-pong) so no host sync.
+//   K3 k_onesweep  one 8-bit LSD digit pass per launch: tile load (warp-striped, coalesced) ->
+//                  warp match.any ranking -> decoupled look-back prefix over tiles (per digit) ->
+//                  shared-memory-staged scatter so global stores are runs of consecutive keys.
+//                  The key transform is fused into the first pass's load and the inverse into
+//                  the last pass's store.
+//
+// All arithmetic is integer; no tensor cores (not a contraction).  HBM bytes per key:
+// K1 8, each K3 pass 16.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "internal.h"
+
+namespace hsort {
+namespace {
+
+constexpr int kDigits = 8;
+constexpr int kRadix = 256;
+constexpr uint64_t kFlagA = 1ull << 62;  // aggregate (tile count) available
+constexpr uint64_t kFlagP = 2ull << 62;  // inclusive prefix available
+constexpr uint64_t kCountMask = (1ull << 40) - 1;
+constexpr uint32_t kEpochMask = (1u << 22) - 1;
+
+// float64 bits -> key: negative -> ~u, non-negative -> u | 2^63 (IEEE totalOrder as unsigned).
+__device__ __forceinline__ uint64_t to_key(uint64_t u) {
+  return u ^ ((uint64_t)((int64_t)u >> 63) | 0x8000000000000000ull);
+}
+// key -> float64 bits (inverse of to_key).
+__device__ __forceinline__ uint64_t from_key(uint64_t k) {
+  return k ^ ((uint64_t)((int64_t)(~k) >> 63) | 0x8000000000000000ull);
+}
+
+__device__ __forceinline__ uint64_t ld_stream(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void ld_stream2(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.global.nc.L1::no_allocate.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p));
+}
+__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// ------------------------------------------------------------------------------------------
+// K1: digit histograms.  Per-CTA shared histograms [8][256]; each thread keeps, per digit, the
+// last digit value and a run count in registers and only issues a shared atomic when the value
+// changes — constant high digits (e.g. the exponent byte of U[0,1)) cost one atomic per run
+// instead of a 32-way conflict per key.
+constexpr int kHistThreads = 512;
+
+template <bool IN_F64>
+__device__ __forceinline__ void hist_key(uint64_t k, uint32_t (*sh)[kRadix], uint32_t* cd,
+                                         uint32_t* cc) {
+  if (IN_F64) k = to_key(k);
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p) {
+    uint32_t d = (uint32_t)(k >> (8 * p)) & 255u;
+    if (d == cd[p]) {
+      ++cc[p];
+    } else {
+      if (cc[p]) atomicAdd(&sh[p][cd[p]], cc[p]);
+      cd[p] = d;
+      cc[p] = 1;
+    }
+  }
+}
+
+template <bool IN_F64>
+__global__ void __launch_bounds__(kHistThreads) k_hist(const uint64_t* __restrict__ src, uint64_t n,
+                                                      uint64_t* __restrict__ hist) {
+  __shared__ uint32_t sh[kDigits][kRadix];
+  for (int i = threadIdx.x; i < kDigits * kRadix; i += kHistThreads) (&sh[0][0])[i] = 0;
+  __syncthreads();
+  uint32_t cd[kDigits], cc[kDigits];
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p) { cd[p] = 0; cc[p] = 0; }
+
+  // head element if src is not 16-byte aligned
+  uint64_t head = ((uintptr_t)src & 15) ? 1 : 0;
+  if (head > n) head = n;
+  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist_key<IN_F64>(src[0], sh, cd, cc);
+  const uint64_t* base = src + head;
+  const uint64_t m = n - head;
+  const uint64_t pairs = m / 2;
+  const uint64_t stride = (uint64_t)gridDim.x * kHistThreads;
+  uint64_t i = (uint64_t)blockIdx.x * kHistThreads + threadIdx.x;
+  // 4 independent 16-byte loads in flight per thread
+  for (; i + 3 * stride < pairs; i += 4 * stride) {
+    uint64_t a[8];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) ld_stream2(base + 2 * (i + u * stride), a[2 * u], a[2 * u + 1]);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) hist_key<IN_F64>(a[u], sh, cd, cc);
+  }
+  for (; i < pairs; i += stride) {
+    uint64_t a0, a1;
+    ld_stream2(base + 2 * i, a0, a1);
+    hist_key<IN_F64>(a0, sh, cd, cc);
+    hist_key<IN_F64>(a1, sh, cd, cc);
+  }
+  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == kHistThreads - 1)
+    hist_key<IN_F64>(base[m - 1], sh, cd, cc);
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p)
+    if (cc[p]) atomicAdd(&sh[p][cd[p]], cc[p]);
+  __syncthreads();
+  for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
+    uint32_t c = (&sh[0][0])[j];
+    if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
+  }
+}
+
+// ------------------------------------------------------------------------------------------
+// Block-wide exclusive scan of one uint64 per thread over the first 256 threads (8 warps).
+__device__ __forceinline__ uint64_t scan256_excl(uint64_t v, uint64_t* s_warp /*[8]*/,
+                                                 uint64_t* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (threadIdx.x < 256 && lane == 31) s_warp[warp] = x;
+  __syncthreads();
+  uint64_t wpre = 0, tot = 0;
+#pragma unroll
+  for (int w = 0; w < 8; ++w) {
+    uint64_t s = s_warp[w];
+    if (w < warp) wpre += s;
+    tot += s;
+  }
+  __syncthreads();
+  if (total) *total = tot;
+  return wpre + x - v;
+}
+
+// K2: bin bases + pass plan.  One CTA of 256 threads.
+__global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ hist,
+                                                   uint64_t* __restrict__ bin_base,
+                                                   RadixPlan* __restrict__ plan, uint64_t n,
+                                                   int in_eq_out, int in_f64, int out_f64) {
+  __shared__ uint64_t s_warp[8];
+  __shared__ int s_nz[kDigits];
+  const int t = threadIdx.x;
+  for (int p = 0; p < kDigits; ++p) {
+    uint64_t v = hist[p * kRadix + t];
+    uint64_t e = scan256_excl(v, s_warp, nullptr);
+    bin_base[p * kRadix + t] = e;
+    int nz = __syncthreads_count(v != 0);
+    if (t == 0) s_nz[p] = nz;
+  }
+  __syncthreads();
+  if (t == 0) {
+    RadixPlan P;
+    int na = 0;
+    for (int p = 0; p < kDigits; ++p)
+      if (s_nz[p] > 1) P.digit[na++] = p;
+    for (int p = na; p < kDigits; ++p) P.digit[p] = -1;
+    P.num_active = na;
+    P.copy_src = -1;
+    P.copy_in_f64 = 0;
+    P.copy_out_f64 = 0;
+    P.pad = 0;
+    // ping-pong assignment: buffers 0 = in, 1 = out, 2 = tmp; the last pass must land in out
+    int cur = 0;
+    if (!in_eq_out) {
+      int nxt = (na & 1) ? 1 : 2;
+      for (int p = 0; p < na; ++p) {
+        P.src[p] = cur;
+        P.dst[p] = nxt;
+        cur = nxt;
+        nxt = (nxt == 1) ? 2 : 1;
+      }
+    } else {
+      int nxt = 2;
+      for (int p = 0; p < na; ++p) {
+        P.src[p] = cur;
+        P.dst[p] = nxt;
+        cur = nxt;
+        nxt = (nxt == 2) ? 0 : 2;
+      }
+      if (na & 1) P.copy_src = 2;  // result sits in tmp: raw copy tmp -> out
+    }
+    for (int p = na; p < kDigits; ++p) { P.src[p] = -1; P.dst[p] = -1; }
+    if (na == 0 && n > 0) {
+      // every digit trivial: all keys identical (or n == 1): out = converted in
+      if (!in_eq_out || in_f64 != out_f64) {
+        P.copy_src = 0;
+        P.copy_in_f64 = in_f64;
+        P.copy_out_f64 = out_f64;
+      }
+    }
+    *plan = P;
+  }
+}
+
+// Single-pass plan (tests / hsort_device_radix_pass): in -> out by `digit`.
+__global__ void k_force_plan(RadixPlan* plan, int digit) {
+  RadixPlan P;
+  P.num_active = 1;
+  for (int p = 0; p < kDigits; ++p) { P.digit[p] = -1; P.src[p] = -1; P.dst[p] = -1; }
+  P.digit[0] = digit;
+  P.src[0] = 0;
+  P.dst[0] = 1;
+  P.copy_src = -1;
+  P.copy_in_f64 = P.copy_out_f64 = P.pad = 0;
+  *plan = P;
+}
+
+__device__ __forceinline__ uint64_t* pick(int id, uint64_t* in, uint64_t* out, uint64_t* tmp) {
+  return id == 0 ? in : (id == 1 ? out : tmp);
+}
+
+// ------------------------------------------------------------------------------------------
+// K3: one onesweep LSD pass.  Tile = THREADS x ITEMS keys; tile ids are taken from an atomic
+// counter in launch order so every tile this CTA waits on is already resident (forward progress
+// of the look-back).
+template <int THREADS, int ITEMS, bool IN_F64>
+__global__ void __launch_bounds__(THREADS) k_onesweep(uint64_t* in, uint64_t* out, uint64_t* tmp,
+                                                       uint64_t n, const RadixPlan* __restrict__ plan,
+                                                       const uint64_t* __restrict__ bin_base,
+                                                       uint64_t* __restrict__ lookback,
+                                                       uint32_t* __restrict__ tile_ctr,
+                                                       uint32_t epoch, int p, int out_f64) {
+  constexpr int WARPS = THREADS / 32;
+  constexpr int TILE = THREADS * ITEMS;
+  static_assert(THREADS >= 256, "one thread per digit");
+  __shared__ uint64_t s_keys[TILE];
+  __shared__ uint32_t s_whist[WARPS][kRadix + 1];
+  __shared__ uint32_t s_tstart[kRadix];
+  __shared__ uint64_t s_gofs[kRadix];
+  __shared__ uint64_t s_warp[8];
+  __shared__ uint32_t s_tile;
+
+  const int na = plan->num_active;
+  if (p >= na) return;
+  const int digit = plan->digit[p];
+  const int shift = 8 * digit;
+  const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
+  uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const bool inv = out_f64 && (p == na - 1);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+
+  if (tid == 0) s_tile = atomicAdd(&tile_ctr[p], 1u);
+  for (int i = tid; i < WARPS * (kRadix + 1); i += THREADS) (&s_whist[0][0])[i] = 0;
+  __syncthreads();
+  const uint64_t tile = s_tile;
+  const uint64_t tbase = tile * TILE;
+  const uint64_t wbase = tbase + (uint64_t)warp * 32 * ITEMS;
+
+  // ---- load (warp-striped: item i of lane l is key wbase + i*32 + l; coalesced 256 B/warp)
+  uint64_t k[ITEMS];
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    uint64_t idx = wbase + (uint64_t)i * 32 + lane;
+    k[i] = idx < n ? ld_stream(src + idx) : 0;
+  }
+  // ---- rank: stable within the warp (item-major, then lane), per-warp digit counters
+  uint32_t r[ITEMS];
+  const uint32_t lt = lanemask_lt();
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    uint64_t idx = wbase + (uint64_t)i * 32 + lane;
+    if (IN_F64) k[i] = to_key(k[i]);
+    uint32_t d = idx < n ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+    uint32_t peers = __match_any_sync(0xffffffffu, d);
+    int leader = __ffs(peers) - 1;
+    uint32_t old = 0;
+    if (lane == leader) {
+      old = s_whist[warp][d];
+      s_whist[warp][d] = old + __popc(peers);
+    }
+    old = __shfl_sync(0xffffffffu, old, leader);
+    r[i] = old + __popc(peers & lt);
+    __syncwarp();
+  }
+  __syncthreads();
+
+  // ---- per digit: warp-exclusive offsets, tile count, early aggregate publish
+  uint64_t cnt = 0;
+  if (tid < kRadix) {
+    uint32_t run = 0;
+#pragma unroll
+    for (int w = 0; w < WARPS; ++w) {
+      uint32_t c = s_whist[w][tid];
+      s_whist[w][tid] = run;
+      run += c;
+    }
+    cnt = run;
+    uint64_t word = (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)(epoch & kEpochMask) << 40) | cnt;
+    st_relaxed(&lookback[tile * kRadix + tid], word);
+  }
+  uint64_t tstart = scan256_excl(cnt, s_warp, nullptr);
+  if (tid < kRadix) s_tstart[tid] = (uint32_t)tstart;
+  __syncthreads();
+
+  // ---- stage the tile in shared memory in digit order
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    uint64_t idx = wbase + (uint64_t)i * 32 + lane;
+    if (idx < n) {
+      uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+      s_keys[s_tstart[d] + s_whist[warp][d] + r[i]] = k[i];
+    }
+  }
+
+  // ---- decoupled look-back (thread = digit)
+  if (tid < kRadix) {
+    uint64_t excl = 0;
+    if (tile > 0) {
+      int64_t j = (int64_t)tile - 1;
+      const uint32_t ep = epoch & kEpochMask;
+      while (j >= 0) {
+        uint64_t w = ld_relaxed(&lookback[(uint64_t)j * kRadix + tid]);
+        uint64_t flag = w & (3ull << 62);
+        if (flag == 0 || (uint32_t)((w >> 40) & kEpochMask) != ep) continue;  // not yet published
+        excl += w & kCountMask;
+        if (flag == kFlagP) break;
+        --j;
+      }
+      st_relaxed(&lookback[tile * kRadix + tid],
+                 kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
+    }
+    s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)s_tstart[tid];
+  }
+  __syncthreads();
+
+  // ---- coalesced scatter: consecutive smem slots are runs of one digit -> consecutive HBM
+  const uint64_t rem = n - tbase;
+  const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+  if (inv) {
+#pragma unroll 4
+    for (int j = tid; j < tile_n; j += THREADS) {
+      uint64_t v = s_keys[j];
+      dst[s_gofs[(uint32_t)(v >> shift) & 255u] + j] = from_key(v);
+    }
+  } else {
+#pragma unroll 4
+    for (int j = tid; j < tile_n; j += THREADS) {
+      uint64_t v = s_keys[j];
+      dst[s_gofs[(uint32_t)(v >> shift) & 255u] + j] = v;
+    }
+  }
+}
+
+constexpr int kPassThreads = 256;
+constexpr int kPassItems = kRadixTile / kPassThreads;
+static_assert(kPassThreads * kPassItems == kRadixTile, "tile");
+
+// Final conversion/copy (P_eff == 0, or odd P_eff with in == out).
+__global__ void k_final_copy(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
+                             const RadixPlan* __restrict__ plan) {
+  const int cs = plan->copy_src;
+  if (cs < 0) return;
+  const uint64_t* s = pick(cs, in, out, tmp);
+  const bool fin = plan->copy_in_f64, fout = plan->copy_out_f64;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t v = s[i];
+    if (fin != fout) v = fin ? to_key(v) : from_key(v);
+    out[i] = v;
+  }
+}
+
+int num_sms(int dev) {
+  static int cached[64] = {0};
+  if (dev < 0 || dev >= 64) return 148;
+  if (!cached[dev]) {
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    cached[dev] = v > 0 ? v : 148;
+  }
+  return cached[dev];
+}
+
+cudaError_t next_epoch(RadixScratch& s, cudaStream_t st, uint32_t* ep) {
+  if (s.epoch >= kEpochMask) {
+    cudaError_t e = cudaMemsetAsync(s.lookback, 0, s.max_tiles * kRadix * sizeof(uint64_t), st);
+    if (e != cudaSuccess) return e;
+    s.epoch = 0;
+  }
+  *ep = ++s.epoch;
+  return cudaSuccess;
+}
+
+cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
+                        uint64_t* hist, cudaStream_t st) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  uint64_t want = (n / 2 + kHistThreads * 8 - 1) / (kHistThreads * 8);
+  uint64_t cap = (uint64_t)num_sms(dev) * 4;
+  int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
+  if (in_f64)
+    k_hist<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+  else
+    k_hist<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
+                        int p, bool first_in_f64, bool out_f64, cudaStream_t st) {
+  uint32_t ep = 0;
+  cudaError_t e = next_epoch(s, st, &ep);
+  if (e != cudaSuccess) return e;
+  uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
+  if (first_in_f64)
+    k_onesweep<kPassThreads, kPassItems, true><<<(unsigned)tiles, kPassThreads, 0, st>>>(
+        in, out, tmp, n, s.plan, s.bin_base, s.lookback, s.tile_ctr, ep, p, out_f64 ? 1 : 0);
+  else
+    k_onesweep<kPassThreads, kPassItems, false><<<(unsigned)tiles, kPassThreads, 0, st>>>(
+        in, out, tmp, n, s.plan, s.bin_base, s.lookback, s.tile_ctr, ep, p, out_f64 ? 1 : 0);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------
+cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
+  cudaError_t e;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (s.small && s.device != dev) return cudaErrorInvalidDevice;
+  s.device = dev;
+  if (!s.small) {
+    size_t bytes = 2 * kDigits * kRadix * sizeof(uint64_t) + sizeof(RadixPlan) + 64;
+    if ((e = cudaMalloc(&s.small, bytes)) != cudaSuccess) return e;
+    char* b = (char*)s.small;
+    s.hist = (uint64_t*)b;
+    s.plan = (RadixPlan*)(b + kDigits * kRadix * sizeof(uint64_t));
+    s.tile_ctr = (uint32_t*)((char*)s.plan + sizeof(RadixPlan));
+    s.bin_base = (uint64_t*)((char*)s.tile_ctr + 64);
+    s.small_zero_bytes = (char*)s.bin_base - b;
+    if ((e = cudaMemset(s.small, 0, bytes)) != cudaSuccess) return e;
+    if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)
+      return e;
+  }
+  uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
+  if (tiles < 1) tiles = 1;
+  if (tiles > s.max_tiles) {
+    if (s.lookback) cudaFree(s.lookback);
+    s.lookback = nullptr;
+    s.max_tiles = 0;
+    uint64_t t2 = tiles + tiles / 8;  // headroom for slightly larger later calls
+    if ((e = cudaMalloc(&s.lookback, t2 * kRadix * sizeof(uint64_t))) != cudaSuccess) return e;
+    if ((e = cudaMemset(s.lookback, 0, t2 * kRadix * sizeof(uint64_t))) != cudaSuccess) return e;
+    s.max_tiles = t2;
+    s.epoch = 0;
+  }
+  return cudaSuccess;
+}
+
+cudaError_t radix_set_timing(RadixScratch& s, bool on) {
+  if (on && !s.ev[0])
+    for (int i = 0; i < kNumKernelEvents; ++i) {
+      cudaError_t e = cudaEventCreate(&s.ev[i]);
+      if (e != cudaSuccess) return e;
+    }
+  s.timing = on;
+  return cudaSuccess;
+}
+
+int radix_kernel_times(RadixScratch& s, float* ms, int max) {
+  if (!s.ev[0]) return 0;
+  int m = 0;
+  for (int i = 1; i < kNumKernelEvents && m < max; ++i) {
+    float t = 0;
+    if (cudaEventElapsedTime(&t, s.ev[i - 1], s.ev[i]) != cudaSuccess) {
+      cudaGetLastError();
+      t = -1;
+    }
+    ms[m++] = t;
+  }
+  return m;
+}
+
+void radix_scratch_release(RadixScratch& s) {
+  for (int i = 0; i < kNumKernelEvents; ++i)
+    if (s.ev[i]) cudaEventDestroy(s.ev[i]);
+  if (s.lookback) cudaFree(s.lookback);
+  if (s.small) cudaFree(s.small);
+  if (s.h_plan) cudaFreeHost(s.h_plan);
+  s = RadixScratch();
+}
+
+cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
+                       uint64_t n, bool in_f64, bool out_f64, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  cudaError_t e = radix_scratch_reserve(s, n);
+  if (e != cudaSuccess) return e;
+  uint64_t* in = const_cast<uint64_t*>(in_c);
+  auto mark = [&](int i) -> cudaError_t {
+    return s.timing ? cudaEventRecord(s.ev[i], st) : cudaSuccess;
+  };
+  if ((e = cudaMemsetAsync(s.small, 0, s.small_zero_bytes, st)) != cudaSuccess) return e;
+  if ((e = mark(0)) != cudaSuccess) return e;
+  if ((e = launch_hist(s, in, n, in_f64, s.hist, st)) != cudaSuccess) return e;
+  if ((e = mark(1)) != cudaSuccess) return e;
+  k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
+                                 out_f64 ? 1 : 0);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = mark(2)) != cudaSuccess) return e;
+  for (int p = 0; p < kDigits; ++p) {
+    if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st)) != cudaSuccess)
+      return e;
+    if ((e = mark(3 + p)) != cudaSuccess) return e;
+  }
+  int dev = 0;
+  cudaGetDevice(&dev);
+  k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = mark(11)) != cudaSuccess) return e;
+  return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);
+}
+
+cudaError_t radix_histograms(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
+                             uint64_t* d_hist, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(d_hist, 0, kDigits * kRadix * sizeof(uint64_t), st);
+  if (e != cudaSuccess || n == 0) return e;
+  return launch_hist(s, in, n, in_f64, d_hist, st);
+}
+
+cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, uint64_t n,
+                           int digit, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  cudaError_t e = radix_scratch_reserve(s, n);
+  if (e != cudaSuccess) return e;
+  uint64_t* in = const_cast<uint64_t*>(src);
+  if ((e = cudaMemsetAsync(s.small, 0, s.small_zero_bytes, st)) != cudaSuccess) return e;
+  if ((e = launch_hist(s, in, n, false, s.hist, st)) != cudaSuccess) return e;
+  k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, 0, 0, 0);
+  k_force_plan<<<1, 1, 0, st>>>(s.plan, digit);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  return launch_pass(s, in, dst, nullptr, n, 0, false, false, st);
+}
+
+}  // namespace hsort

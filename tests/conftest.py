@@ -30,3 +30,22 @@ def inputs_mod():
     import hsort_inputs
     hsort_inputs.build()
     return hsort_inputs
+
+
+@pytest.fixture(scope="session")
+def hs():
+    """The product binding (libhsort.so must already be built: __graft_entry__.build())."""
+    import paper_conf_ipps_gowanlockk18a_b200 as hs_mod
+    hs_mod.lib()
+    return hs_mod
+
+
+@pytest.fixture(scope="session")
+def hs_gpu(hs):
+    """Initialised library on a real GPU (gpu-marked tests only)."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    hs.hsort_init()
+    yield hs
+    hs.hsort_finalize()

@@ -1,0 +1,150 @@
+"""GPU parity: K4 co-ranks, K5 merge, and the host->host hsort_sort in every mode vs the oracle."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+
+def _bits(a):
+    return np.ascontiguousarray(a).view(np.uint64)
+
+
+def _runs(rng, k, maxlen, hi=2**64):
+    runs = [np.sort(rng.integers(0, hi, size=int(rng.integers(0, maxlen + 1)), dtype=np.uint64))
+            for _ in range(k)]
+    off = np.zeros(k + 1, dtype=np.uint64)
+    for j, r in enumerate(runs):
+        off[j + 1] = off[j] + r.size
+    return runs, np.concatenate(runs), off
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 8, 33, 100, 300])
+@pytest.mark.parametrize("hi", [2**64, 50])
+def test_corank_matches_oracle(hs_gpu, oracle_mod, k, hi):
+    import torch
+    rng = np.random.default_rng(k + hi % 1000)
+    runs, keys, off = _runs(rng, k, 3000 if k < 50 else 400, hi)
+    total = int(off[-1])
+    step = max(1, total // 37)
+    nb = total // step + 2
+    d_keys = torch.from_numpy(keys).cuda()
+    d_r = torch.zeros(nb * k, dtype=torch.uint64, device="cuda")
+    hs_gpu.hsort_device_corank(d_keys, off, step, nb, d_r)
+    got = d_r.cpu().numpy().reshape(nb, k)
+    for b in range(nb):
+        o = min(b * step, total)
+        assert np.array_equal(got[b], oracle_mod.corank(runs, o)), (b, o)
+
+
+@pytest.mark.parametrize("k", [1, 2, 5, 16, 120, 1024])
+@pytest.mark.parametrize("hi", [2**64, 7])
+def test_device_merge_matches_oracle(hs_gpu, oracle_mod, k, hi):
+    import torch
+    rng = np.random.default_rng(3 * k + hi % 100)
+    runs, keys, off = _runs(rng, k, 20000 if k <= 16 else 300, hi)
+    d_keys = torch.from_numpy(keys).cuda()
+    d_out = torch.empty_like(d_keys)
+    hs_gpu.hsort_device_merge(d_keys, off, d_out, False)
+    assert np.array_equal(d_out.cpu().numpy(), oracle_mod.merge_runs(runs))
+
+
+def test_device_merge_inverse_transform(hs_gpu, oracle_mod, inputs_mod):
+    import torch
+    A = inputs_mod.generate("special", 200_000, seed=12)
+    K = oracle_mod.keys_from_f64(A)
+    parts = [oracle_mod.sort_u64(p) for p in np.array_split(K, 9)]
+    off = np.cumsum([0] + [p.size for p in parts]).astype(np.uint64)
+    d_keys = torch.from_numpy(np.concatenate(parts)).cuda()
+    d_out = torch.empty_like(d_keys)
+    hs_gpu.hsort_device_merge(d_keys, off, d_out, True)
+    assert np.array_equal(d_out.cpu().numpy(), _bits(oracle_mod.sort_f64(A)))
+
+
+# ---- host -> host ------------------------------------------------------------------------------
+def _pinned(a):
+    import torch
+    t = torch.from_numpy(a).pin_memory()
+    return t
+
+
+CASES = [
+    # (n, batch_elems, resident option, pipeline option, expected mode)
+    (1 << 20, 0, -1, 1, "BLINE"),
+    (1_000_003, 150_000, -1, 1, "RESIDENT"),
+    (1_000_003, 150_000, 0, 1, "STREAM"),
+    (1_000_003, 150_000, 0, 0, "STREAM"),
+    (777_777, 4096, -1, 1, "RESIDENT"),
+    (300_001, 1, 0, 1, None),  # b_s = 1 -> n_b > 1024: STREAM with huge k on the CPU merge
+]
+
+
+@pytest.mark.parametrize("n,b,res,pipe,mode", CASES)
+@pytest.mark.parametrize("pinned", [False, True])
+def test_hsort_sort_modes(hs_gpu, oracle_mod, inputs_mod, n, b, res, pipe, mode, pinned):
+    if b == 1 and n > 5000:
+        n, b = 5000, 1
+    A = inputs_mod.generate("salted", n, seed=n + b)
+    want = _bits(oracle_mod.sort_f64(A))
+    hs_gpu.hsort_set_option("resident", res)
+    hs_gpu.hsort_set_option("pipeline", pipe)
+    try:
+        if pinned:
+            At, Bt = _pinned(A.copy()), _pinned(np.zeros_like(A))
+            hs_gpu.hsort_sort(At, Bt, batch_elems=b, n_gpus=1)
+            B = Bt.numpy()
+        else:
+            B = hs_gpu.hsort_sort(A, batch_elems=b, n_gpus=1)
+        st = hs_gpu.hsort_get_stats()
+    finally:
+        hs_gpu.hsort_set_option("resident", -1)
+        hs_gpu.hsort_set_option("pipeline", 1)
+    assert np.array_equal(_bits(B), want)
+    if mode:
+        assert st["mode_name"] == mode
+    assert st["direct_in"] == int(pinned) and st["direct_out"] == int(pinned)
+    assert st["n"] == n and st["n_b"] == -(-n // (b or n))
+
+
+@pytest.mark.parametrize("dist", ["uniform", "normal", "zipf_dup", "special", "all_equal",
+                                  "closed_form", "reverse"])
+def test_hsort_sort_distributions(hs_gpu, oracle_mod, inputs_mod, dist):
+    A = inputs_mod.generate(dist, 2_000_003, seed=77)
+    want = _bits(oracle_mod.sort_f64(A))
+    for b in (0, 300_000):
+        assert np.array_equal(_bits(hs_gpu.hsort_sort(A, batch_elems=b)), want), (dist, b)
+
+
+def test_hsort_sort_in_place_and_u64(hs_gpu, oracle_mod, inputs_mod):
+    A = inputs_mod.generate("special", 500_001, seed=4)
+    want = _bits(oracle_mod.sort_f64(A))
+    for b in (0, 100_000):
+        X = A.copy()
+        hs_gpu.hsort_sort(X, X, batch_elems=b)
+        assert np.array_equal(_bits(X), want)
+    K = np.random.default_rng(3).integers(0, 2**64, size=400_000, dtype=np.uint64)
+    for b in (0, 64_000):
+        assert np.array_equal(hs_gpu.hsort_sort_u64(K, batch_elems=b), oracle_mod.sort_u64(K))
+
+
+def test_hsort_sort_edge_cases(hs_gpu, oracle_mod):
+    hs_gpu.hsort_sort(np.zeros(0))
+    for n in (1, 2, 3):
+        A = np.array([np.nan, -0.0, 0.0][:n])
+        assert np.array_equal(_bits(hs_gpu.hsort_sort(A)), _bits(oracle_mod.sort_f64(A)))
+    with pytest.raises(hs_gpu.HsortError) as e:
+        hs_gpu.hsort_sort(np.zeros(10), n_gpus=99)
+    assert e.value.code == -1
+    buf = np.zeros(20)
+    with pytest.raises(hs_gpu.HsortError):
+        hs_gpu.lib().hsort_sort(buf.ctypes.data, buf.ctypes.data + 40, 10, 0, 1)  # partial overlap
+    with pytest.raises(hs_gpu.HsortError):
+        hs_gpu.hsort_init()  # second init -> BUSY
+
+
+def test_stats_fields(hs_gpu, inputs_mod):
+    A = inputs_mod.generate("uniform", 1 << 22, seed=1)
+    hs_gpu.hsort_sort(A, batch_elems=1 << 20)
+    st = hs_gpu.hsort_get_stats()
+    assert st["n_b"] == 4 and st["passes_run"] >= 1
+    assert st["bytes_h2d"] == A.nbytes and st["bytes_d2h"] == A.nbytes
+    assert st["t_total"] > 0 and st["t_gpu_sort"] > 0 and st["t_h2d"] > 0

@@ -1,0 +1,144 @@
+"""Host-native components of the product library against the oracle (CPU, no GPU needed).
+
+H2 CPU multiway merge + co-rank (§III-A), PARMEMCPY, the planner
+(Table I) and the PIPEMERGE count (Fig. 3).
+"""
+import os
+
+import numpy as np
+import pytest
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _runs(rng, k, maxlen, hi=2**64, allow_empty=True):
+    runs = []
+    for _ in range(k):
+        m = int(rng.integers(0 if allow_empty else 1, maxlen + 1))
+        runs.append(np.sort(rng.integers(0, hi, size=m, dtype=np.uint64)))
+    return runs
+
+
+def _pack(runs):
+    off = np.zeros(len(runs) + 1, dtype=np.uint64)
+    for j, r in enumerate(runs):
+        off[j + 1] = off[j] + r.size
+    keys = np.concatenate(runs) if runs else np.zeros(0, np.uint64)
+    return np.ascontiguousarray(keys, dtype=np.uint64), off
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 5, 16, 64, 130])
+@pytest.mark.parametrize("hi", [2**64, 1000, 3])
+def test_host_merge_equals_oracle(hs, oracle_mod, k, hi):
+    rng = np.random.default_rng(k * 7 + (hi % 97))
+    runs = _runs(rng, k, 40000 if k < 20 else 3000, hi)
+    keys, off = _pack(runs)
+    got = hs.hsort_host_merge(keys, off, out_f64=False, threads=8)
+    assert np.array_equal(got, oracle_mod.merge_runs(runs))
+
+
+def test_host_merge_inverse_transform_on_store(hs, oracle_mod, inputs_mod):
+    A = inputs_mod.generate("special", 300_000, seed=3)
+    K = oracle_mod.keys_from_f64(A)
+    parts = np.array_split(K, 7)
+    runs = [oracle_mod.sort_u64(p) for p in parts]
+    keys, off = _pack(runs)
+    got = hs.hsort_host_merge(keys, off, out_f64=True, threads=8)
+    want = oracle_mod.sort_f64(A)
+    assert np.array_equal(got.view(np.uint64), want.view(np.uint64))
+
+
+def test_host_merge_offset_base_and_single_thread(hs, oracle_mod):
+    rng = np.random.default_rng(1)
+    runs = _runs(rng, 9, 5000, 50)
+    keys, off = _pack(runs)
+    pad = np.concatenate([np.full(13, 7, np.uint64), keys])
+    off2 = off + np.uint64(13)
+    got = hs.hsort_host_merge(pad, off2, threads=1)
+    assert np.array_equal(got, oracle_mod.merge_runs(runs))
+
+
+@pytest.mark.parametrize("k", [1, 2, 7, 40])
+def test_host_corank_equals_oracle(hs, oracle_mod, k):
+    rng = np.random.default_rng(100 + k)
+    for hi in (2**64, 20):
+        runs = _runs(rng, k, 200, hi)
+        keys, off = _pack(runs)
+        n = int(off[-1])
+        for o in sorted({0, 1, n // 3, n // 2, max(n - 1, 0), n}):
+            assert np.array_equal(hs.hsort_host_corank(keys, off, o), oracle_mod.corank(runs, o))
+
+
+def test_par_memcpy(hs):
+    rng = np.random.default_rng(0)
+    src = rng.integers(0, 255, size=(64 << 20) + 77, dtype=np.uint8)
+    for t in (1, 3, 8):
+        dst = np.zeros_like(src)
+        hs.hsort_par_memcpy(dst, src, threads=t)
+        assert np.array_equal(dst, src)
+
+
+def test_pipemerge_count_matches_fig3_golden(hs):
+    rows = [l.split() for l in open(os.path.join(GOLDEN, "fig3_pipemerge.txt"))
+            if l.strip() and not l.startswith("#")]
+    for n_b, n_gpu, merges, final_lists in rows:
+        assert hs.hsort_pipemerge_count(int(n_b), int(n_gpu)) == int(merges)
+    for n_b in range(0, 50):
+        for g in (1, 2, 4, 8):
+            assert hs.hsort_pipemerge_count(n_b, g) <= max(0, (n_b - 1) // 2) if n_b else True
+
+
+def test_planner_table1_identities(hs):
+    rows = [l.split() for l in open(os.path.join(GOLDEN, "table1_identities.txt"))
+            if l.strip() and not l.startswith("#")]
+    old = hs.hsort_get_option("n_s")
+    try:
+        for n, b_s, n_s, n_gpu, n_b, per_stream, gpu_bytes in rows:
+            hs.hsort_set_option("n_s", int(n_s))
+            # a GPU exactly as large as the paper's (16 GiB / 12 GiB)
+            dev = 16 << 30 if int(b_s) == 500000000 else 12 << 30
+            p = hs.hsort_plan(int(n), int(b_s), int(n_gpu), dev)
+            assert p["b_s"] == int(b_s)
+            assert p["n_b"] == int(n_b) == -(-int(n) // int(b_s))
+            assert abs(p["batches_per_stream"] - float(per_stream)) < 1e-9
+            if p["mode_name"] == "STREAM":
+                # B200 design shares one alt buffer: (n_s + 1) b_s keys <= paper's 2 b_s n_s
+                assert p["device_bytes_per_gpu"] <= int(gpu_bytes) + int(b_s)
+    finally:
+        hs.hsort_set_option("n_s", old)
+
+
+def test_planner_modes_and_ragged_batches(hs):
+    G = 180 << 30
+    p = hs.hsort_plan(1 << 30, 0, 1, G)
+    assert p["mode_name"] == "BLINE" and p["n_b"] == 1 and p["b_s"] == 1 << 30
+    p = hs.hsort_plan(10**9 + 7, 250_000_000, 1, G)
+    assert p["n_b"] == 5 and p["last_batch"] == 7 and p["mode_name"] == "RESIDENT"
+    p = hs.hsort_plan(3 * 10**10, 250_000_000, 1, G)  # 240 GB: runs cannot stay in HBM
+    assert p["n_b"] == 120 and p["mode_name"] == "STREAM"
+    p = hs.hsort_plan(3 * 10**10, 0, 1, G)  # auto b_s fills HBM with n_s + 1 buffers
+    assert p["mode_name"] == "STREAM" and p["b_s"] % 4096 == 0
+    assert p["device_bytes_per_gpu"] <= G
+    p = hs.hsort_plan(10**9, 10**8, 4, G)
+    assert p["mode_name"] == "STREAM" and p["n_gpus"] == 4
+    hs.hsort_set_option("resident", 0)
+    try:
+        assert hs.hsort_plan(10**9, 10**8, 1, G)["mode_name"] == "STREAM"
+    finally:
+        hs.hsort_set_option("resident", -1)
+
+
+def test_options_validation(hs):
+    with pytest.raises(hs.HsortError):
+        hs.hsort_set_option("no_such_option", 1)
+    with pytest.raises(hs.HsortError):
+        hs.hsort_set_option("resident", 5)
+    with pytest.raises(hs.HsortError):
+        hs.hsort_set_option("n_s", 0)
+
+
+def test_sort_without_init_fails_cleanly(hs):
+    A = np.zeros(10)
+    with pytest.raises(hs.HsortError) as e:
+        hs.hsort_sort(A)
+    assert e.value.code == -2

@@ -444,13 +444,16 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
   if (s.small && s.device != dev) return cudaErrorInvalidDevice;
   s.device = dev;
   if (!s.small) {
-    size_t bytes = 2 * kDigits * kRadix * sizeof(uint64_t) + sizeof(RadixPlan) + 64;
+    // layout (256-byte aligned pieces): hist | plan | tile counters | bin_base
+    const size_t hist_b = kDigits * kRadix * sizeof(uint64_t);
+    const size_t plan_b = (sizeof(RadixPlan) + 255) & ~(size_t)255;
+    const size_t bytes = hist_b + plan_b + 256 + hist_b;
     if ((e = cudaMalloc(&s.small, bytes)) != cudaSuccess) return e;
     char* b = (char*)s.small;
     s.hist = (uint64_t*)b;
-    s.plan = (RadixPlan*)(b + kDigits * kRadix * sizeof(uint64_t));
-    s.tile_ctr = (uint32_t*)((char*)s.plan + sizeof(RadixPlan));
-    s.bin_base = (uint64_t*)((char*)s.tile_ctr + 64);
+    s.plan = (RadixPlan*)(b + hist_b);
+    s.tile_ctr = (uint32_t*)(b + hist_b + plan_b);
+    s.bin_base = (uint64_t*)(b + hist_b + plan_b + 256);
     s.small_zero_bytes = (char*)s.bin_base - b;
     if ((e = cudaMemset(s.small, 0, bytes)) != cudaSuccess) return e;
     if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)

@@ -18,6 +18,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 #include "internal.h"
 
@@ -30,6 +31,9 @@ constexpr uint64_t kFlagA = 1ull << 62;  // aggregate (tile count) available
 constexpr uint64_t kFlagP = 2ull << 62;  // inclusive prefix available
 constexpr uint64_t kCountMask = (1ull << 40) - 1;
 constexpr uint32_t kEpochMask = (1u << 22) - 1;
+#ifdef HSORT_PHASE_TIMING
+__device__ unsigned long long g_phase_dbg[256];  // instrumented builds only
+#endif
 
 // float64 bits -> key: negative -> ~u, non-negative -> u | 2^63 (IEEE totalOrder as unsigned).
 __device__ __forceinline__ uint64_t to_key(uint64_t u) {
@@ -369,6 +373,684 @@ constexpr int kPassThreads = 256;
 constexpr int kPassItems = kRadixTile / kPassThreads;
 static_assert(kPassThreads * kPassItems == kRadixTile, "tile");
 
+// ------------------------------------------------------------------------------------------
+// K3 v2: persistent onesweep pass with TMA bulk tile prefetch.
+//
+// Each resident CTA loops over tiles taken from the pass's atomic counter.  While it ranks and
+// scatters tile i, one elected thread has already issued a cp.async.bulk (TMA, SASS UBLKCP) of
+// tile i+1 into the other half of a double-buffered shared-memory stage, completing on an
+// mbarrier; so the HBM read latency of the next tile overlaps the current tile's work.  The
+// stage buffer that held tile i is reused as the digit-ordered scatter buffer of tile i.
+// Forward progress of the look-back: a CTA holds at most one claimed-but-unstarted tile, which
+// was claimed after its current tile, so the smallest current tile never waits on it.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+// Windowed decoupled look-back for one digit: reads the status words of W predecessor tiles
+// per round trip (independent loads in flight) and accumulates aggregates back to the first
+// inclusive prefix.  A serial walk costs one L2 round trip per step and, with tiles claimed a
+// few tens of cycles apart, needs ~latency/interval steps; the window resolves them together.
+template <int W>
+__device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__ lookback,
+                                                    int64_t j, int d, uint32_t ep) {
+  uint64_t excl = 0;
+  while (true) {
+#ifdef HSORT_PHASE_TIMING
+    if (d == 0) atomicAdd(&g_phase_dbg[200], 1ull);
+#endif
+    uint64_t w[W];
+#pragma unroll
+    for (int q = 0; q < W; ++q)
+      w[q] = (j - q >= 0) ? ld_relaxed(&lookback[(uint64_t)(j - q) * kRadix + d])
+                          : (kFlagP | ((uint64_t)ep << 40));  // before tile 0: prefix 0
+    int q = 0;
+    bool done = false;
+#pragma unroll
+    for (int u = 0; u < W; ++u) {
+      if (done || q != u) continue;
+      const uint64_t flag = w[u] & (3ull << 62);
+      if (flag == 0 || (uint32_t)((w[u] >> 40) & kEpochMask) != ep) continue;  // not yet: re-read
+      excl += w[u] & kCountMask;
+      if (flag == kFlagP) done = true;
+      else ++q;
+    }
+    if (done) return excl;
+    j -= q;  // all consumed aggregates; re-read from the first unavailable tile
+  }
+}
+
+// Same, with the first window already loaded (issued before the tile's scan/scatter so the L2
+// round trip overlaps them).
+template <int W>
+__device__ __forceinline__ uint64_t lookback_window_pre(const uint64_t* __restrict__ lookback,
+                                                        int64_t j, int d, uint32_t ep,
+                                                        const uint64_t* pre) {
+  uint64_t excl = 0;
+  int q = 0;
+#pragma unroll
+  for (int u = 0; u < W; ++u) {
+    if (q != u) continue;
+    const uint64_t flag = pre[u] & (3ull << 62);
+    if (flag == 0 || (uint32_t)((pre[u] >> 40) & kEpochMask) != ep) continue;
+    excl += pre[u] & kCountMask;
+    if (flag == kFlagP) return excl;
+    ++q;
+  }
+  return excl + lookback_window<W>(lookback, j - q, d, ep);
+}
+
+#ifdef HSORT_PHASE_TIMING
+#define HSORT_PHASE(i)                         \
+  if (tid == 0) {                              \
+    const long long _now = clock64();          \
+    ph_acc[i] += (unsigned long long)(_now - ph_last); \
+    ph_last = _now;                            \
+  }
+#else
+#define HSORT_PHASE(i)
+#endif
+
+template <int THREADS, int ITEMS>
+struct TmaPassSmem {
+  static constexpr int WARPS = THREADS / 32;
+  static constexpr int TILE = THREADS * ITEMS;
+  static constexpr size_t stage_off = 0;                                   // [2][TILE] u64
+  static constexpr size_t whist_off = stage_off + 2ull * TILE * 8;         // [WARPS][257] u32
+  static constexpr size_t tstart_off = whist_off + (size_t)WARPS * (kRadix + 1) * 4;
+  static constexpr size_t gofs_off = (tstart_off + kRadix * 4 + 15) & ~(size_t)15;  // [256] u64
+  static constexpr size_t bar_off = gofs_off + kRadix * 8;                 // [2] u64
+  static constexpr size_t swarp_off = bar_off + 16;                        // [8] u64
+  static constexpr size_t tile_off = swarp_off + 64;                       // [2] u32
+  static constexpr size_t thist_off = tile_off + 16;                       // [257] u32
+  static constexpr size_t bytes = thist_off + (kRadix + 1) * 4;
+};
+
+template <int THREADS, int ITEMS, bool IN_F64, int LBW>
+__global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THREADS * ITEMS <= 4096) ? 2 : 1)) k_onesweep_tma(uint64_t* in, uint64_t* out, uint64_t* tmp,
+                                                           uint64_t n,
+                                                           const RadixPlan* __restrict__ plan,
+                                                           const uint64_t* __restrict__ bin_base,
+                                                           uint64_t* __restrict__ lookback,
+                                                           uint32_t* __restrict__ tile_ctr,
+                                                           uint32_t epoch, int p, int out_f64) {
+  using L = TmaPassSmem<THREADS, ITEMS>;
+  constexpr int WARPS = L::WARPS;
+  constexpr int TILE = L::TILE;
+  static_assert(THREADS >= 256 && THREADS % 32 == 0, "one thread per digit");
+  extern __shared__ __align__(128) unsigned char smem[];
+  uint64_t* stage = (uint64_t*)(smem + L::stage_off);
+  uint32_t* whist = (uint32_t*)(smem + L::whist_off);
+  uint32_t* s_tstart = (uint32_t*)(smem + L::tstart_off);
+  uint64_t* s_gofs = (uint64_t*)(smem + L::gofs_off);
+  uint64_t* bars = (uint64_t*)(smem + L::bar_off);
+  uint64_t* s_warp = (uint64_t*)(smem + L::swarp_off);
+  uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
+  uint32_t* s_thist = (uint32_t*)(smem + L::thist_off);
+
+  const int na = plan->num_active;
+  if (p >= na) return;
+  const int digit = plan->digit[p];
+  const int shift = 8 * digit;
+  const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
+  uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const bool inv = out_f64 && (p == na - 1);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t num_tiles = (n + TILE - 1) / TILE;
+  const uint32_t ep = epoch & kEpochMask;
+
+  auto issue = [&](uint64_t t, int b) {  // one thread: claim stage b for tile t
+    const uint64_t base = t * (uint64_t)TILE;
+    const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
+    const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
+    // WAR on the buffer (generic reads/writes of the previous tile) is ordered by the
+    // __syncthreads that precedes every issue; no proxy fence is needed for a TMA load.
+    mbar_arrive_expect_tx(&bars[b], bytes);
+    if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bars[b]);
+  };
+
+  uint32_t claim_next = 0;  // thread 0: tile id claimed one iteration ahead (atomic off the path)
+  if (tid == 0) {
+    mbar_init(&bars[0], 1);
+    mbar_init(&bars[1], 1);
+    mbar_fence_init();
+    uint32_t t = atomicAdd(&tile_ctr[p], 1u);
+    s_tile[0] = t;
+    if (t < num_tiles) issue(t, 0);
+    claim_next = atomicAdd(&tile_ctr[p], 1u);
+  }
+  __syncthreads();
+  uint32_t phase = 0;  // bit b = parity to wait for on bars[b]
+  int cb = 0;
+  const uint32_t lt = lanemask_lt();
+#ifdef HSORT_PHASE_TIMING
+  unsigned long long ph_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+  long long ph_last = clock64();
+  unsigned long long ph_tiles = 0;
+#endif
+  while (true) {
+    const uint64_t tile = s_tile[cb];
+    if (tile >= num_tiles) break;
+    if (tid == 0) {
+      const uint32_t t = claim_next;
+      s_tile[cb ^ 1] = t;
+      if (t < num_tiles) {
+        issue(t, cb ^ 1);
+        claim_next = atomicAdd(&tile_ctr[p], 1u);
+      }
+    }
+    for (int i = tid; i < WARPS * (kRadix + 1); i += THREADS) whist[i] = 0;
+    mbar_wait(&bars[cb], (phase >> cb) & 1u);
+    phase ^= 1u << cb;
+    __syncthreads();
+    HSORT_PHASE(0);
+
+    const uint64_t tbase = tile * (uint64_t)TILE;
+    const uint64_t rem = n - tbase;
+    const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+    const bool full = tile_n == TILE;
+    const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
+    uint64_t* sb = stage + (size_t)cb * TILE;
+    const int wofs = warp * 32 * ITEMS + lane;
+    uint32_t* wh = whist + warp * (kRadix + 1);
+
+    // ---- keys: shared stage -> registers (warp-striped: conflict-free 8-byte reads)
+    uint64_t k[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      const int j = wofs + i * 32;
+      uint64_t v;
+      if (full) v = sb[j];
+      else v = j < bulk_n ? sb[j] : (j < tile_n ? src[tbase + j] : 0);
+      k[i] = IN_F64 ? to_key(v) : v;
+    }
+    // ---- rank: per-warp digit counters; the highest peer lane adds the group's count.
+    // Three unrolled phases so the match.any latencies and the leaders' shared atomics of all
+    // ITEMS items are in flight together (same-digit atomics still serialise in hardware order).
+    uint32_t r[ITEMS];
+    {
+      uint32_t dd[ITEMS], peers[ITEMS];
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const bool valid = full || (wofs + i * 32 < tile_n);
+        dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+      }
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const int leader = 31 - __clz(peers[i]);
+        r[i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+      }
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const int leader = 31 - __clz(peers[i]);
+        r[i] = __shfl_sync(0xffffffffu, r[i], leader) + __popc(peers[i] & lt);
+      }
+    }
+    __syncthreads();
+    HSORT_PHASE(2);
+
+    // ---- per digit: warp-exclusive offsets, tile count, aggregate publish, tile-local starts
+    uint64_t cnt = 0;
+    if (tid < kRadix) {
+      uint32_t run = 0;
+#pragma unroll
+      for (int w = 0; w < WARPS; ++w) {
+        const uint32_t c = whist[w * (kRadix + 1) + tid];
+        whist[w * (kRadix + 1) + tid] = run;
+        run += c;
+      }
+      cnt = run;
+      st_relaxed(&lookback[tile * kRadix + tid],
+                 (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+    }
+    const uint32_t tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
+    if (tid < kRadix) {
+      s_tstart[tid] = tstart;
+#pragma unroll
+      for (int w = 0; w < WARPS; ++w) whist[w * (kRadix + 1) + tid] += tstart;
+    }
+    __syncthreads();
+    HSORT_PHASE(3);
+
+    // ---- scatter into the (already consumed) stage buffer in digit order
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      if (full || wofs + i * 32 < tile_n) {
+        const uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+        sb[wh[d] + r[i]] = k[i];
+      }
+    }
+    // ---- decoupled look-back (thread = digit), LBW predecessors read per round trip
+    if (tid < kRadix) {
+      uint64_t excl = 0;
+      if (tile > 0) {
+        excl = lookback_window<LBW>(lookback, (int64_t)tile - 1, tid, ep);
+        st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
+      }
+      s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)s_tstart[tid];
+    }
+    __syncthreads();
+    HSORT_PHASE(4);
+
+    // ---- write out: consecutive slots are runs of one digit -> coalesced HBM stores
+    if (full) {
+      uint64_t v[ITEMS], g[ITEMS];
+#pragma unroll
+      for (int q = 0; q < ITEMS; ++q) v[q] = sb[tid + q * THREADS];
+#pragma unroll
+      for (int q = 0; q < ITEMS; ++q) g[q] = s_gofs[(uint32_t)(v[q] >> shift) & 255u];
+      if (inv) {
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = from_key(v[q]);
+      } else {
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = v[q];
+      }
+    } else if (inv) {
+#pragma unroll 4
+      for (int j = tid; j < tile_n; j += THREADS) {
+        const uint64_t v = sb[j];
+        dst[s_gofs[(uint32_t)(v >> shift) & 255u] + j] = from_key(v);
+      }
+    } else {
+#pragma unroll 4
+      for (int j = tid; j < tile_n; j += THREADS) {
+        const uint64_t v = sb[j];
+        dst[s_gofs[(uint32_t)(v >> shift) & 255u] + j] = v;
+      }
+    }
+    __syncthreads();
+    HSORT_PHASE(5);
+#ifdef HSORT_PHASE_TIMING
+    ++ph_tiles;
+#endif
+    cb ^= 1;
+  }
+#ifdef HSORT_PHASE_TIMING
+  if (tid == 0) {
+    for (int i = 0; i < 10; ++i) atomicAdd(&g_phase_dbg[p * 16 + (i < 8 ? i : i + 1)], ph_acc[i]);
+    atomicAdd(&g_phase_dbg[p * 16 + 8], ph_tiles);
+  }
+#endif
+}
+
+// ------------------------------------------------------------------------------------------
+// K3 v3: software-pipelined persistent onesweep pass.
+//
+// Three shared-memory tile buffers rotate through the roles  load (TMA bulk, in flight) ->
+// rank + in-place digit-order scatter -> write-out.  Iteration i ranks tile i while the
+// look-back of tile i-1 (whose aggregate was published one iteration earlier) is in flight: its
+// status loads are issued at the start of the iteration and consumed after the ranking, so the
+// predecessors' inclusive prefixes are already published and the L2 round trip is hidden.  Tile
+// i-1 is then written out while tile i is scattered.  Tile ids are claimed one iteration ahead.
+// Forward progress: every tile publishes its aggregate before its CTA waits on any look-back,
+// so a look-back can always walk aggregates down to an inclusive prefix (tile 0 publishes one).
+template <int THREADS, int ITEMS>
+struct PipeSmem {
+  static constexpr int WARPS = THREADS / 32;
+  static constexpr int TILE = THREADS * ITEMS;
+  static constexpr size_t buf_off = 0;                                     // [3][TILE] u64
+  static constexpr size_t whist_off = buf_off + 3ull * TILE * 8;          // [WARPS][257] u32
+  static constexpr size_t thist_off = whist_off + (size_t)WARPS * (kRadix + 1) * 4;  // [257]
+  static constexpr size_t gofs_off = (thist_off + (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [256] u64
+  static constexpr size_t bar_off = gofs_off + kRadix * 8;                 // [3] u64
+  static constexpr size_t swarp_off = bar_off + 32;                        // [8] u64
+  static constexpr size_t tile_off = swarp_off + 64;                       // [3] u32
+  static constexpr size_t bytes = tile_off + 16;
+};
+
+template <int THREADS, int ITEMS, bool IN_F64, int LBW, bool EARLY>
+__global__ void __launch_bounds__(THREADS, 2) k_onesweep_pipe(uint64_t* in, uint64_t* out,
+                                                              uint64_t* tmp, uint64_t n,
+                                                              const RadixPlan* __restrict__ plan,
+                                                              const uint64_t* __restrict__ bin_base,
+                                                              uint64_t* __restrict__ lookback,
+                                                              uint32_t* __restrict__ tile_ctr,
+                                                              uint32_t epoch, int p, int out_f64) {
+  using L = PipeSmem<THREADS, ITEMS>;
+  constexpr int WARPS = L::WARPS;
+  constexpr int TILE = L::TILE;
+  static_assert(THREADS == 256, "one thread per digit, 8 warps");
+  extern __shared__ __align__(128) unsigned char smem[];
+  uint64_t* bufs = (uint64_t*)(smem + L::buf_off);
+  uint32_t* whist = (uint32_t*)(smem + L::whist_off);
+  uint32_t* s_thist = (uint32_t*)(smem + L::thist_off);
+  uint64_t* s_gofs = (uint64_t*)(smem + L::gofs_off);
+  uint64_t* bars = (uint64_t*)(smem + L::bar_off);
+  uint64_t* s_warp = (uint64_t*)(smem + L::swarp_off);
+  uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
+
+  const int na = plan->num_active;
+  if (p >= na) return;
+  const int digit = plan->digit[p];
+  const int shift = 8 * digit;
+  const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
+  uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const bool inv = out_f64 && (p == na - 1);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t num_tiles = (n + TILE - 1) / TILE;
+  const uint32_t ep = epoch & kEpochMask;
+  const uint64_t* __restrict__ bb = bin_base + digit * kRadix;
+
+  auto issue = [&](uint64_t t, int b) {  // thread 0: load tile t into buffer b
+    const uint64_t base = t * (uint64_t)TILE;
+    const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
+    const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
+    // WAR on the buffer (generic reads/writes of the previous tile) is ordered by the
+    // __syncthreads that precedes every issue; no proxy fence is needed for a TMA load.
+    mbar_arrive_expect_tx(&bars[b], bytes);
+    if (bytes) bulk_g2s(bufs + (size_t)b * TILE, src + base, bytes, &bars[b]);
+  };
+
+  uint32_t claim_next = 0;
+  if (tid == 0) {
+    for (int b = 0; b < 3; ++b) mbar_init(&bars[b], 1);
+    mbar_fence_init();
+    const uint32_t t0 = atomicAdd(&tile_ctr[p], 1u);
+    const uint32_t t1 = atomicAdd(&tile_ctr[p], 1u);
+    s_tile[0] = t0;
+    s_tile[1] = t1;
+    if (t0 < num_tiles) issue(t0, 0);
+    if (t1 < num_tiles) issue(t1, 1);
+    claim_next = atomicAdd(&tile_ctr[p], 1u);
+  }
+  __syncthreads();
+
+  const uint32_t lt = lanemask_lt();
+  uint32_t phase = 0;
+  int cur = 0;
+  bool prev_valid = false;
+  uint64_t prev_tile = 0;
+  uint32_t prev_cnt = 0, prev_tstart = 0;
+  uint32_t* wh = whist + warp * (kRadix + 1);
+  const int wofs = warp * 32 * ITEMS + lane;
+
+  while (true) {
+    const uint64_t tile = s_tile[cur];
+    const bool has_cur = tile < num_tiles;
+    if (!has_cur && !prev_valid) break;
+    const int prv = (cur + 2) % 3;
+
+    // (a) look-back loads for the previous tile, in flight during this tile's ranking
+    uint64_t lbw[LBW];
+    if (prev_valid && tid < kRadix) {
+#pragma unroll
+      for (int q = 0; q < LBW; ++q)
+        lbw[q] = ((int64_t)prev_tile - 1 - q >= 0)
+                     ? ld_relaxed(&lookback[(prev_tile - 1 - q) * kRadix + tid])
+                     : (kFlagP | ((uint64_t)ep << 40));
+    }
+
+    // (b) rank the current tile
+    uint64_t k[ITEMS];
+    uint32_t r[ITEMS];
+    uint32_t cnt = 0, tstart = 0;
+    int tile_n = 0;
+    bool full = false;
+    uint64_t* sb = bufs + (size_t)cur * TILE;
+    if (has_cur) {
+      for (int i = tid; i < WARPS * (kRadix + 1); i += THREADS) whist[i] = 0;
+      for (int i = tid; i < kRadix + 1; i += THREADS) s_thist[i] = 0;
+      mbar_wait(&bars[cur], (phase >> cur) & 1u);
+      phase ^= 1u << cur;
+      __syncthreads();
+      const uint64_t tbase = tile * (uint64_t)TILE;
+      const uint64_t rem = n - tbase;
+      tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+      full = tile_n == TILE;
+      const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const int j = wofs + i * 32;
+        uint64_t v;
+        if (full) v = sb[j];
+        else v = j < bulk_n ? sb[j] : (j < tile_n ? src[tbase + j] : 0);
+        k[i] = IN_F64 ? to_key(v) : v;
+      }
+      if (EARLY) {
+        // early counts -> aggregate published before the ranking
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+          const bool valid = full || (wofs + i * 32 < tile_n);
+          atomicAdd(&s_thist[valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix], 1u);
+        }
+        __syncthreads();
+        if (tid < kRadix) {
+          cnt = s_thist[tid];
+          st_relaxed(&lookback[tile * kRadix + tid],
+                     (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+        }
+        tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
+      }
+      {
+        uint32_t dd[ITEMS], peers[ITEMS];
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+          const bool valid = full || (wofs + i * 32 < tile_n);
+          dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+        }
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+          const int leader = 31 - __clz(peers[i]);
+          r[i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+          const int leader = 31 - __clz(peers[i]);
+          r[i] = __shfl_sync(0xffffffffu, r[i], leader) + __popc(peers[i] & lt);
+        }
+      }
+      __syncthreads();
+      if (!EARLY) {
+        // counts from the per-warp ranking counters; aggregate published now (its look-back
+        // successors read it one iteration later)
+        if (tid < kRadix) {
+#pragma unroll
+          for (int w = 0; w < WARPS; ++w) cnt += whist[w * (kRadix + 1) + tid];
+          st_relaxed(&lookback[tile * kRadix + tid],
+                     (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+        }
+        tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
+      }
+      if (tid < kRadix) {
+        uint32_t run = tstart;
+#pragma unroll
+        for (int w = 0; w < WARPS; ++w) {
+          const uint32_t c = whist[w * (kRadix + 1) + tid];
+          whist[w * (kRadix + 1) + tid] = run;
+          run += c;
+        }
+      }
+    }
+    // (c) finish the previous tile's look-back
+    if (prev_valid && tid < kRadix) {
+      uint64_t excl = 0;
+      if (prev_tile > 0) {
+        excl = lookback_window_pre<LBW>(lookback, (int64_t)prev_tile - 1, tid, ep, lbw);
+        st_relaxed(&lookback[prev_tile * kRadix + tid],
+                   kFlagP | ((uint64_t)ep << 40) | (excl + prev_cnt));
+      }
+      s_gofs[tid] = bb[tid] + excl - (uint64_t)prev_tstart;
+    }
+    __syncthreads();
+
+    // (d) write out the previous tile; (e) scatter the current tile in place
+    if (prev_valid) {
+      const uint64_t* pb = bufs + (size_t)prv * TILE;
+      const uint64_t prem = n - prev_tile * (uint64_t)TILE;
+      const int pn = prem < (uint64_t)TILE ? (int)prem : TILE;
+      if (pn == TILE) {
+        uint64_t v[ITEMS], g[ITEMS];
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q) v[q] = pb[tid + q * THREADS];
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q) g[q] = s_gofs[(uint32_t)(v[q] >> shift) & 255u];
+        if (inv) {
+#pragma unroll
+          for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = from_key(v[q]);
+        } else {
+#pragma unroll
+          for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = v[q];
+        }
+      } else {
+        for (int j = tid; j < pn; j += THREADS) {
+          const uint64_t v = pb[j];
+          const uint64_t o = s_gofs[(uint32_t)(v >> shift) & 255u] + j;
+          dst[o] = inv ? from_key(v) : v;
+        }
+      }
+    }
+    if (has_cur) {
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        if (full || wofs + i * 32 < tile_n) {
+          const uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+          sb[wh[d] + r[i]] = k[i];
+        }
+      }
+    }
+    __syncthreads();
+
+    // (f) buffer prv is free: load the tile claimed last iteration into it, claim the next one
+    if (tid == 0) {
+      s_tile[prv] = claim_next;
+      if (claim_next < num_tiles) {
+        issue(claim_next, prv);
+        claim_next = atomicAdd(&tile_ctr[p], 1u);
+      }
+    }
+    prev_valid = has_cur;
+    prev_tile = tile;
+    prev_cnt = cnt;
+    prev_tstart = tstart;
+    cur = (cur + 1) % 3;
+    __syncthreads();
+  }
+}
+
+// K1 v2: per-warp entropy probe picks, for each digit, either direct shared atomics (spread
+// digits) or the register run-length cache (low-entropy digits, e.g. the exponent byte).
+template <bool IN_F64, uint32_t MASK>
+__device__ __forceinline__ void hist2_key(uint64_t k, uint32_t* sh, uint32_t* cd, uint32_t* cc,
+                                          uint32_t mask) {
+  if (IN_F64) k = to_key(k);
+  const uint32_t lo = (uint32_t)k, hi = (uint32_t)(k >> 32);
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p) {
+    const uint32_t d = ((p < 4 ? lo : hi) >> (8 * (p & 3))) & 255u;
+    const bool low = (MASK == 0xFFFFFFFFu) ? ((mask >> p) & 1u) : ((MASK >> p) & 1u);
+    if (low) {
+      if (d == cd[p]) {
+        ++cc[p];
+      } else {
+        if (cc[p]) atomicAdd(&sh[p * kRadix + cd[p]], cc[p]);
+        cd[p] = d;
+        cc[p] = 1;
+      }
+    } else {
+      atomicAdd(&sh[p * kRadix + d], 1u);
+    }
+  }
+}
+
+template <bool IN_F64, uint32_t MASK>
+__device__ __forceinline__ void hist2_loop(const uint64_t* base, uint64_t pairs, uint64_t i,
+                                           uint64_t stride, uint32_t* sh, uint32_t* cd,
+                                           uint32_t* cc, uint32_t mask) {
+  for (; i + 3 * stride < pairs; i += 4 * stride) {
+    uint64_t a[8];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) ld_stream2(base + 2 * (i + u * stride), a[2 * u], a[2 * u + 1]);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) hist2_key<IN_F64, MASK>(a[u], sh, cd, cc, mask);
+  }
+  for (; i < pairs; i += stride) {
+    uint64_t a0, a1;
+    ld_stream2(base + 2 * i, a0, a1);
+    hist2_key<IN_F64, MASK>(a0, sh, cd, cc, mask);
+    hist2_key<IN_F64, MASK>(a1, sh, cd, cc, mask);
+  }
+}
+
+template <bool IN_F64>
+__global__ void __launch_bounds__(kHistThreads) k_hist2(const uint64_t* __restrict__ src, uint64_t n,
+                                                       uint64_t* __restrict__ hist) {
+  __shared__ uint32_t sh[kDigits * kRadix];
+  for (int i = threadIdx.x; i < kDigits * kRadix; i += kHistThreads) sh[i] = 0;
+  __syncthreads();
+  uint32_t cd[kDigits], cc[kDigits];
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p) { cd[p] = 0; cc[p] = 0; }
+  const uint64_t head = (((uintptr_t)src & 15) && n) ? 1 : 0;
+  const uint64_t* base = src + head;
+  const uint64_t m = n - head;
+  const uint64_t pairs = m / 2;
+  const uint64_t stride = (uint64_t)gridDim.x * kHistThreads;
+  const uint64_t i0 = (uint64_t)blockIdx.x * kHistThreads + threadIdx.x;
+  // entropy probe on this warp's first keys: <= 4 distinct values among 32 lanes -> run cache
+  uint32_t mask = 0;
+  {
+    uint64_t k = i0 < pairs ? base[2 * i0] : (m ? base[0] : 0);
+    if (IN_F64) k = to_key(k);
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int p = 0; p < kDigits; ++p) {
+      const uint32_t d = (uint32_t)(k >> (8 * p)) & 255u;
+      const uint32_t peers = __match_any_sync(0xffffffffu, d);
+      const uint32_t leaders = __ballot_sync(0xffffffffu, lane == 31 - __clz(peers));
+      if (__popc(leaders) <= 4) mask |= 1u << p;
+    }
+  }
+  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist2_key<IN_F64, 0xFFFFFFFFu>(src[0], sh, cd, cc, 0xFF);
+  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else if (mask == 0u) hist2_loop<IN_F64, 0u>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else hist2_loop<IN_F64, 0xFFFFFFFFu>(base, pairs, i0, stride, sh, cd, cc, mask);
+  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == kHistThreads - 1)
+    hist2_key<IN_F64, 0xFFFFFFFFu>(base[m - 1], sh, cd, cc, 0xFF);
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p)
+    if (cc[p]) atomicAdd(&sh[p * kRadix + cd[p]], cc[p]);
+  __syncthreads();
+  for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
+    uint32_t c = sh[j];
+    if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
+  }
+}
+
 // Final conversion/copy (P_eff == 0, or odd P_eff with in == out).
 __global__ void k_final_copy(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
                              const RadixPlan* __restrict__ plan) {
@@ -405,17 +1087,111 @@ cudaError_t next_epoch(RadixScratch& s, cudaStream_t st, uint32_t* ep) {
   return cudaSuccess;
 }
 
+// Kernel variant selection (tuning knob; HSORT_PASS_VARIANT / HSORT_HIST_VARIANT env vars).
+//   pass 0: v1 register-load, one CTA per tile (256 x 16)
+//   pass 1: TMA persistent 256 x 16    2: TMA 512 x 8    3: TMA 384 x 16    4: TMA 512 x 16
+int env_int(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return v ? atoi(v) : dflt;
+}
+int pass_variant() {
+  static int v = env_int("HSORT_PASS_VARIANT", 1);
+  return v;
+}
+int hist_variant() {
+  static int v = env_int("HSORT_HIST_VARIANT", 1);
+  return v;
+}
+
+// keys per tile of the selected pass variant (sizes the look-back array)
+int variant_tile(int v) {
+  switch (v) {
+    case 11: return 256 * 8;
+    case 12: return 256 * 12;
+    case 3: return 384 * 16;
+    case 4: case 7: return 512 * 16;
+    default: return 4096;
+  }
+}
+
 cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
                         uint64_t* hist, cudaStream_t st) {
   int dev = 0;
   cudaGetDevice(&dev);
   uint64_t want = (n / 2 + kHistThreads * 8 - 1) / (kHistThreads * 8);
-  uint64_t cap = (uint64_t)num_sms(dev) * 4;
+  uint64_t cap = (uint64_t)num_sms(dev) * 2;
   int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-  if (in_f64)
-    k_hist<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+  if (hist_variant() == 0) {
+    if (in_f64) k_hist<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+    else k_hist<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+  } else {
+    if (in_f64) k_hist2<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+    else k_hist2<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+  }
+  return cudaGetLastError();
+}
+
+template <int THREADS, int ITEMS, int LBW = 8>
+cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
+                            RadixScratch& s, uint32_t ep, int p, bool first_in_f64, bool out_f64,
+                            cudaStream_t st) {
+  using L = TmaPassSmem<THREADS, ITEMS>;
+  static int blocks_per_sm[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  auto kt = k_onesweep_tma<THREADS, ITEMS, true, LBW>;
+  auto kf = k_onesweep_tma<THREADS, ITEMS, false, LBW>;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  if (!blocks_per_sm[dev]) {
+    cudaError_t e;
+    if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
+    if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
+    int b = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, THREADS, L::bytes)) != cudaSuccess) return e;
+    blocks_per_sm[dev] = b > 0 ? b : 1;
+  }
+  const uint64_t tiles = (n + L::TILE - 1) / L::TILE;
+  if (tiles > s.max_tiles) return cudaErrorInvalidValue;  // look-back array too small
+  uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
+  if (grid > tiles) grid = tiles ? tiles : 1;
+  if (first_in_f64)
+    kt<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
+                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
   else
-    k_hist<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+    kf<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
+                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
+  return cudaGetLastError();
+}
+
+template <int THREADS, int ITEMS, int LBW, bool EARLY = true>
+cudaError_t launch_pipe_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
+                             RadixScratch& s, uint32_t ep, int p, bool first_in_f64, bool out_f64,
+                             cudaStream_t st) {
+  using L = PipeSmem<THREADS, ITEMS>;
+  static int blocks_per_sm[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  auto kt = k_onesweep_pipe<THREADS, ITEMS, true, LBW, EARLY>;
+  auto kf = k_onesweep_pipe<THREADS, ITEMS, false, LBW, EARLY>;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  if (!blocks_per_sm[dev]) {
+    cudaError_t e;
+    if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
+    if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
+    int b = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, THREADS, L::bytes)) != cudaSuccess) return e;
+    blocks_per_sm[dev] = b > 0 ? b : 1;
+  }
+  const uint64_t tiles = (n + L::TILE - 1) / L::TILE;
+  if (tiles > s.max_tiles) return cudaErrorInvalidValue;  // look-back array too small
+  uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
+  if (grid > tiles) grid = tiles ? tiles : 1;
+  if (first_in_f64)
+    kt<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
+                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
+  else
+    kf<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
+                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
   return cudaGetLastError();
 }
 
@@ -424,6 +1200,24 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   uint32_t ep = 0;
   cudaError_t e = next_epoch(s, st, &ep);
   if (e != cudaSuccess) return e;
+  // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
+  const bool aligned = !(((uintptr_t)in | (uintptr_t)out | (uintptr_t)(tmp ? tmp : out)) & 15);
+  const int v = aligned ? pass_variant() : 0;
+  switch (v) {
+    case 1: return launch_tma_pass<256, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 2: return launch_tma_pass<512, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 3: return launch_tma_pass<384, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 4: return launch_tma_pass<512, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 5: return launch_tma_pass<256, 16, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 6: return launch_tma_pass<256, 16, 32>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 7: return launch_tma_pass<512, 16, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 8: return launch_pipe_pass<256, 16, 4>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 9: return launch_pipe_pass<256, 16, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 10: return launch_pipe_pass<256, 16, 4, false>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 11: return launch_tma_pass<256, 8, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 12: return launch_tma_pass<256, 12, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    default: break;
+  }
   uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
   if (first_in_f64)
     k_onesweep<kPassThreads, kPassItems, true><<<(unsigned)tiles, kPassThreads, 0, st>>>(
@@ -435,6 +1229,18 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
 }
 
 }  // namespace
+
+#ifdef HSORT_PHASE_TIMING
+extern "C" int hsort_debug_phase_counters(unsigned long long* out, int max, int reset) {
+  if (max > 256) max = 256;
+  cudaMemcpyFromSymbol(out, g_phase_dbg, max * sizeof(unsigned long long));
+  if (reset) {
+    static unsigned long long z[256] = {0};
+    cudaMemcpyToSymbol(g_phase_dbg, z, sizeof(z));
+  }
+  return (int)cudaGetLastError();
+}
+#endif
 
 // ------------------------------------------------------------------------------------------
 cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
@@ -459,7 +1265,8 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
     if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)
       return e;
   }
-  uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
+  const int tile_keys = variant_tile(pass_variant()) < kRadixTile ? variant_tile(pass_variant()) : kRadixTile;
+  uint64_t tiles = (n + tile_keys - 1) / tile_keys;
   if (tiles < 1) tiles = 1;
   if (tiles > s.max_tiles) {
     if (s.lookback) cudaFree(s.lookback);

@@ -60,6 +60,12 @@ __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
 __device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void ld_relaxed2(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st_relaxed2(uint64_t* p, uint64_t a, uint64_t b) {
+  asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -486,17 +492,16 @@ struct TmaPassSmem {
   static constexpr int TILE = THREADS * ITEMS;
   static constexpr size_t stage_off = 0;                                   // [2][TILE] u64
   static constexpr size_t whist_off = stage_off + 2ull * TILE * 8;         // [WARPS][257] u32
-  static constexpr size_t tstart_off = whist_off + (size_t)WARPS * (kRadix + 1) * 4;
-  static constexpr size_t gofs_off = (tstart_off + kRadix * 4 + 15) & ~(size_t)15;  // [256] u64
+  static constexpr size_t gofs_off = (whist_off + (size_t)WARPS * (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [256] u64
   static constexpr size_t bar_off = gofs_off + kRadix * 8;                 // [2] u64
   static constexpr size_t swarp_off = bar_off + 16;                        // [8] u64
   static constexpr size_t tile_off = swarp_off + 64;                       // [2] u32
-  static constexpr size_t thist_off = tile_off + 16;                       // [257] u32
-  static constexpr size_t bytes = thist_off + (kRadix + 1) * 4;
+  static constexpr size_t ct_off = tile_off + 16;                          // [256] (count, start)
+  static constexpr size_t bytes = ct_off + kRadix * 8;
 };
 
-template <int THREADS, int ITEMS, bool IN_F64, int LBW>
-__global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THREADS * ITEMS <= 4096) ? 2 : 1)) k_onesweep_tma(uint64_t* in, uint64_t* out, uint64_t* tmp,
+template <int THREADS, int ITEMS, bool IN_F64, int LBW, int MINB>
+__global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, uint64_t* out, uint64_t* tmp,
                                                            uint64_t n,
                                                            const RadixPlan* __restrict__ plan,
                                                            const uint64_t* __restrict__ bin_base,
@@ -510,12 +515,11 @@ __global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THR
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* stage = (uint64_t*)(smem + L::stage_off);
   uint32_t* whist = (uint32_t*)(smem + L::whist_off);
-  uint32_t* s_tstart = (uint32_t*)(smem + L::tstart_off);
   uint64_t* s_gofs = (uint64_t*)(smem + L::gofs_off);
   uint64_t* bars = (uint64_t*)(smem + L::bar_off);
   uint64_t* s_warp = (uint64_t*)(smem + L::swarp_off);
   uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
-  uint32_t* s_thist = (uint32_t*)(smem + L::thist_off);
+  uint2* s_ct = (uint2*)(smem + L::ct_off);
 
   const int na = plan->num_active;
   if (p >= na) return;
@@ -537,6 +541,39 @@ __global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THR
     mbar_arrive_expect_tx(&bars[b], bytes);
     if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bars[b]);
   };
+
+  // LBW < 0: the first CTA to arrive becomes the prefix scanner: it turns every tile's
+  // aggregate into its exclusive prefix, in tile order, with PF status loads in flight per digit;
+  // the workers then wait on their own tile's word only (no look-back walk).
+  if (LBW < 0) {
+    if (tid == 0) s_tile[0] = atomicAdd(&tile_ctr[8 + p], 1u);
+    __syncthreads();
+    if (s_tile[0] == 0) {
+      if (tid < kRadix) {
+        constexpr int PF = 16;
+        uint64_t run = 0;
+        for (uint64_t t0 = 0; t0 < num_tiles; t0 += PF) {
+          uint64_t w[PF];
+#pragma unroll
+          for (int q = 0; q < PF; ++q)
+            w[q] = (t0 + q < num_tiles) ? ld_relaxed(&lookback[(t0 + q) * kRadix + tid]) : 0;
+#pragma unroll
+          for (int q = 0; q < PF; ++q) {
+            if (t0 + q >= num_tiles) break;
+            uint64_t* wp = &lookback[(t0 + q) * kRadix + tid];
+            while ((w[q] & (3ull << 62)) != kFlagA || (uint32_t)((w[q] >> 40) & kEpochMask) != ep) {
+              __nanosleep(20);
+              w[q] = ld_relaxed(wp);
+            }
+            st_relaxed(wp, kFlagP | ((uint64_t)ep << 40) | run);
+            run += w[q] & kCountMask;
+          }
+        }
+      }
+      return;
+    }
+    __syncthreads();
+  }
 
   uint32_t claim_next = 0;  // thread 0: tile id claimed one iteration ahead (atomic off the path)
   if (tid == 0) {
@@ -597,24 +634,26 @@ __global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THR
     // Three unrolled phases so the match.any latencies and the leaders' shared atomics of all
     // ITEMS items are in flight together (same-digit atomics still serialise in hardware order).
     uint32_t r[ITEMS];
-    {
-      uint32_t dd[ITEMS], peers[ITEMS];
+    constexpr int RC = (MINB >= 3 && ITEMS % 2 == 0) ? ITEMS / 2 : ITEMS;  // ranking chunk
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
-        const bool valid = full || (wofs + i * 32 < tile_n);
-        dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+    for (int c0 = 0; c0 < ITEMS; c0 += RC) {
+      uint32_t dd[RC], peers[RC];
+#pragma unroll
+      for (int i = 0; i < RC; ++i) {
+        const bool valid = full || (wofs + (c0 + i) * 32 < tile_n);
+        dd[i] = valid ? ((uint32_t)(k[c0 + i] >> shift) & 255u) : (uint32_t)kRadix;
       }
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+      for (int i = 0; i < RC; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
+      for (int i = 0; i < RC; ++i) {
         const int leader = 31 - __clz(peers[i]);
-        r[i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+        r[c0 + i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
       }
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
+      for (int i = 0; i < RC; ++i) {
         const int leader = 31 - __clz(peers[i]);
-        r[i] = __shfl_sync(0xffffffffu, r[i], leader) + __popc(peers[i] & lt);
+        r[c0 + i] = __shfl_sync(0xffffffffu, r[c0 + i], leader) + __popc(peers[i] & lt);
       }
     }
     __syncthreads();
@@ -632,17 +671,65 @@ __global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THR
       }
       cnt = run;
       st_relaxed(&lookback[tile * kRadix + tid],
-                 (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+                 ((tile == 0 && LBW >= 0) ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
     }
     const uint32_t tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
     if (tid < kRadix) {
-      s_tstart[tid] = tstart;
 #pragma unroll
       for (int w = 0; w < WARPS; ++w) whist[w * (kRadix + 1) + tid] += tstart;
+      if (LBW == 0) s_ct[tid] = make_uint2((uint32_t)cnt, tstart);
     }
     __syncthreads();
     HSORT_PHASE(3);
 
+    // ---- LBW == 0: warp-cooperative decoupled look-back by warp 0 (lane = 8 consecutive
+    // digits, one coalesced 2 KB status row per step, warp-uniform control flow), overlapped
+    // with the other warps' scatter
+    if (LBW == 0 && warp == 0) {
+      uint64_t ex[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) ex[q] = 0;
+      uint32_t todo = tile > 0 ? 0xFFu : 0u, cons = 0;
+      int64_t j = (int64_t)tile - 1;
+      while (__any_sync(0xffffffffu, todo != 0)) {
+        if (todo & ~cons) {
+          const uint64_t* row = lookback + (uint64_t)j * kRadix + lane * 8;
+          uint64_t w[8];
+#pragma unroll
+          for (int q = 0; q < 8; q += 2) ld_relaxed2(row + q, w[q], w[q + 1]);
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const uint32_t bit = 1u << q;
+            const uint64_t flag = w[q] & (3ull << 62);
+            const bool ok = flag != 0 && (uint32_t)((w[q] >> 40) & kEpochMask) == ep;
+            if ((todo & ~cons & bit) && ok) {
+              ex[q] += w[q] & kCountMask;
+              cons |= bit;
+              if (flag == kFlagP) todo &= ~bit;
+            }
+          }
+        }
+        if (__all_sync(0xffffffffu, (todo & ~cons) == 0)) {
+          --j;
+          cons = 0;
+        } else {
+          __nanosleep(32);
+        }
+      }
+      uint64_t g[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int d = lane * 8 + q;
+        const uint2 ct = s_ct[d];
+        g[q] = kFlagP | ((uint64_t)ep << 40) | (ex[q] + ct.x);
+        s_gofs[d] = bin_base[digit * kRadix + d] + ex[q] - (uint64_t)ct.y;
+      }
+      if (tile > 0) {
+        uint64_t* row = lookback + tile * kRadix + lane * 8;
+#pragma unroll
+        for (int q = 0; q < 8; q += 2) st_relaxed2(row + q, g[q], g[q + 1]);
+      }
+    }
     // ---- scatter into the (already consumed) stage buffer in digit order
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -651,31 +738,45 @@ __global__ void __launch_bounds__(THREADS, (THREADS * ITEMS <= 2048) ? 4 : ((THR
         sb[wh[d] + r[i]] = k[i];
       }
     }
+    // ---- scanner mode: wait for this tile's exclusive prefix
+    if (LBW < 0 && tid < kRadix) {
+      const uint64_t* wp = &lookback[tile * kRadix + tid];
+      uint64_t w = ld_relaxed(wp);
+      while ((w & (3ull << 62)) != kFlagP || (uint32_t)((w >> 40) & kEpochMask) != ep) {
+        __nanosleep(32);
+        w = ld_relaxed(wp);
+      }
+      s_gofs[tid] = bin_base[digit * kRadix + tid] + (w & kCountMask) - (uint64_t)tstart;
+    }
     // ---- decoupled look-back (thread = digit), LBW predecessors read per round trip
-    if (tid < kRadix) {
+    if (LBW > 0 && tid < kRadix) {
       uint64_t excl = 0;
       if (tile > 0) {
-        excl = lookback_window<LBW>(lookback, (int64_t)tile - 1, tid, ep);
+        excl = lookback_window<(LBW > 0 ? LBW : 1)>(lookback, (int64_t)tile - 1, tid, ep);
         st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
       }
-      s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)s_tstart[tid];
+      s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)tstart;
     }
     __syncthreads();
     HSORT_PHASE(4);
 
     // ---- write out: consecutive slots are runs of one digit -> coalesced HBM stores
     if (full) {
-      uint64_t v[ITEMS], g[ITEMS];
+      constexpr int WC = (MINB >= 3) ? ITEMS / 2 : ITEMS;  // write-out chunk
 #pragma unroll
-      for (int q = 0; q < ITEMS; ++q) v[q] = sb[tid + q * THREADS];
+      for (int c0 = 0; c0 < ITEMS; c0 += WC) {
+        uint64_t v[WC], g[WC];
 #pragma unroll
-      for (int q = 0; q < ITEMS; ++q) g[q] = s_gofs[(uint32_t)(v[q] >> shift) & 255u];
-      if (inv) {
+        for (int q = 0; q < WC; ++q) v[q] = sb[tid + (c0 + q) * THREADS];
 #pragma unroll
-        for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = from_key(v[q]);
-      } else {
+        for (int q = 0; q < WC; ++q) g[q] = s_gofs[(uint32_t)(v[q] >> shift) & 255u];
+        if (inv) {
 #pragma unroll
-        for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = v[q];
+          for (int q = 0; q < WC; ++q) dst[g[q] + tid + (c0 + q) * THREADS] = from_key(v[q]);
+        } else {
+#pragma unroll
+          for (int q = 0; q < WC; ++q) dst[g[q] + tid + (c0 + q) * THREADS] = v[q];
+        }
       }
     } else if (inv) {
 #pragma unroll 4
@@ -1131,7 +1232,7 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
   return cudaGetLastError();
 }
 
-template <int THREADS, int ITEMS, int LBW = 8>
+template <int THREADS, int ITEMS, int LBW = 8, int MINB = ((THREADS * ITEMS <= 2048) ? 4 : ((THREADS * ITEMS <= 4096) ? 2 : 1))>
 cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
                             RadixScratch& s, uint32_t ep, int p, bool first_in_f64, bool out_f64,
                             cudaStream_t st) {
@@ -1139,8 +1240,8 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
   static int blocks_per_sm[64] = {0};
   int dev = 0;
   cudaGetDevice(&dev);
-  auto kt = k_onesweep_tma<THREADS, ITEMS, true, LBW>;
-  auto kf = k_onesweep_tma<THREADS, ITEMS, false, LBW>;
+  auto kt = k_onesweep_tma<THREADS, ITEMS, true, LBW, MINB>;
+  auto kf = k_onesweep_tma<THREADS, ITEMS, false, LBW, MINB>;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   if (!blocks_per_sm[dev]) {
     cudaError_t e;
@@ -1153,7 +1254,8 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
   const uint64_t tiles = (n + L::TILE - 1) / L::TILE;
   if (tiles > s.max_tiles) return cudaErrorInvalidValue;  // look-back array too small
   uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
-  if (grid > tiles) grid = tiles ? tiles : 1;
+  const uint64_t need = tiles + (LBW < 0 ? 1 : 0);  // scanner mode: one CTA scans
+  if (grid > need) grid = need ? need : 1;
   if (first_in_f64)
     kt<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
                                                  s.tile_ctr, ep, p, out_f64 ? 1 : 0);
@@ -1216,6 +1318,11 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
     case 10: return launch_pipe_pass<256, 16, 4, false>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
     case 11: return launch_tma_pass<256, 8, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
     case 12: return launch_tma_pass<256, 12, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 13: return launch_tma_pass<256, 16, 8, 3>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 14: return launch_tma_pass<256, 16, 0>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 15: return launch_tma_pass<256, 16, 0, 3>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 16: return launch_tma_pass<256, 16, -1>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    case 17: return launch_tma_pass<256, 16, -1, 3>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
     default: break;
   }
   uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;

@@ -60,12 +60,6 @@ __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
 __device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
-__device__ __forceinline__ void ld_relaxed2(const uint64_t* p, uint64_t& a, uint64_t& b) {
-  asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
-}
-__device__ __forceinline__ void st_relaxed2(uint64_t* p, uint64_t a, uint64_t b) {
-  asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
-}
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -398,9 +392,6 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
 __device__ __forceinline__ void mbar_fence_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
-__device__ __forceinline__ void fence_proxy_async_smem() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
                "r"(bytes)
@@ -455,26 +446,6 @@ __device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__
   }
 }
 
-// Same, with the first window already loaded (issued before the tile's scan/scatter so the L2
-// round trip overlaps them).
-template <int W>
-__device__ __forceinline__ uint64_t lookback_window_pre(const uint64_t* __restrict__ lookback,
-                                                        int64_t j, int d, uint32_t ep,
-                                                        const uint64_t* pre) {
-  uint64_t excl = 0;
-  int q = 0;
-#pragma unroll
-  for (int u = 0; u < W; ++u) {
-    if (q != u) continue;
-    const uint64_t flag = pre[u] & (3ull << 62);
-    if (flag == 0 || (uint32_t)((pre[u] >> 40) & kEpochMask) != ep) continue;
-    excl += pre[u] & kCountMask;
-    if (flag == kFlagP) return excl;
-    ++q;
-  }
-  return excl + lookback_window<W>(lookback, j - q, d, ep);
-}
-
 #ifdef HSORT_PHASE_TIMING
 #define HSORT_PHASE(i)                         \
   if (tid == 0) {                              \
@@ -496,8 +467,7 @@ struct TmaPassSmem {
   static constexpr size_t bar_off = gofs_off + kRadix * 8;                 // [2] u64
   static constexpr size_t swarp_off = bar_off + 16;                        // [8] u64
   static constexpr size_t tile_off = swarp_off + 64;                       // [2] u32
-  static constexpr size_t ct_off = tile_off + 16;                          // [256] (count, start)
-  static constexpr size_t bytes = ct_off + kRadix * 8;
+  static constexpr size_t bytes = tile_off + 16;
 };
 
 template <int THREADS, int ITEMS, bool IN_F64, int LBW, int MINB>
@@ -519,7 +489,6 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
   uint64_t* bars = (uint64_t*)(smem + L::bar_off);
   uint64_t* s_warp = (uint64_t*)(smem + L::swarp_off);
   uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
-  uint2* s_ct = (uint2*)(smem + L::ct_off);
 
   const int na = plan->num_active;
   if (p >= na) return;
@@ -541,39 +510,6 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
     mbar_arrive_expect_tx(&bars[b], bytes);
     if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bars[b]);
   };
-
-  // LBW < 0: the first CTA to arrive becomes the prefix scanner: it turns every tile's
-  // aggregate into its exclusive prefix, in tile order, with PF status loads in flight per digit;
-  // the workers then wait on their own tile's word only (no look-back walk).
-  if (LBW < 0) {
-    if (tid == 0) s_tile[0] = atomicAdd(&tile_ctr[8 + p], 1u);
-    __syncthreads();
-    if (s_tile[0] == 0) {
-      if (tid < kRadix) {
-        constexpr int PF = 16;
-        uint64_t run = 0;
-        for (uint64_t t0 = 0; t0 < num_tiles; t0 += PF) {
-          uint64_t w[PF];
-#pragma unroll
-          for (int q = 0; q < PF; ++q)
-            w[q] = (t0 + q < num_tiles) ? ld_relaxed(&lookback[(t0 + q) * kRadix + tid]) : 0;
-#pragma unroll
-          for (int q = 0; q < PF; ++q) {
-            if (t0 + q >= num_tiles) break;
-            uint64_t* wp = &lookback[(t0 + q) * kRadix + tid];
-            while ((w[q] & (3ull << 62)) != kFlagA || (uint32_t)((w[q] >> 40) & kEpochMask) != ep) {
-              __nanosleep(20);
-              w[q] = ld_relaxed(wp);
-            }
-            st_relaxed(wp, kFlagP | ((uint64_t)ep << 40) | run);
-            run += w[q] & kCountMask;
-          }
-        }
-      }
-      return;
-    }
-    __syncthreads();
-  }
 
   uint32_t claim_next = 0;  // thread 0: tile id claimed one iteration ahead (atomic off the path)
   if (tid == 0) {
@@ -671,65 +607,16 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
       }
       cnt = run;
       st_relaxed(&lookback[tile * kRadix + tid],
-                 ((tile == 0 && LBW >= 0) ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+                 (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
     }
     const uint32_t tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
     if (tid < kRadix) {
 #pragma unroll
       for (int w = 0; w < WARPS; ++w) whist[w * (kRadix + 1) + tid] += tstart;
-      if (LBW == 0) s_ct[tid] = make_uint2((uint32_t)cnt, tstart);
     }
     __syncthreads();
     HSORT_PHASE(3);
 
-    // ---- LBW == 0: warp-cooperative decoupled look-back by warp 0 (lane = 8 consecutive
-    // digits, one coalesced 2 KB status row per step, warp-uniform control flow), overlapped
-    // with the other warps' scatter
-    if (LBW == 0 && warp == 0) {
-      uint64_t ex[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) ex[q] = 0;
-      uint32_t todo = tile > 0 ? 0xFFu : 0u, cons = 0;
-      int64_t j = (int64_t)tile - 1;
-      while (__any_sync(0xffffffffu, todo != 0)) {
-        if (todo & ~cons) {
-          const uint64_t* row = lookback + (uint64_t)j * kRadix + lane * 8;
-          uint64_t w[8];
-#pragma unroll
-          for (int q = 0; q < 8; q += 2) ld_relaxed2(row + q, w[q], w[q + 1]);
-#pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const uint32_t bit = 1u << q;
-            const uint64_t flag = w[q] & (3ull << 62);
-            const bool ok = flag != 0 && (uint32_t)((w[q] >> 40) & kEpochMask) == ep;
-            if ((todo & ~cons & bit) && ok) {
-              ex[q] += w[q] & kCountMask;
-              cons |= bit;
-              if (flag == kFlagP) todo &= ~bit;
-            }
-          }
-        }
-        if (__all_sync(0xffffffffu, (todo & ~cons) == 0)) {
-          --j;
-          cons = 0;
-        } else {
-          __nanosleep(32);
-        }
-      }
-      uint64_t g[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const int d = lane * 8 + q;
-        const uint2 ct = s_ct[d];
-        g[q] = kFlagP | ((uint64_t)ep << 40) | (ex[q] + ct.x);
-        s_gofs[d] = bin_base[digit * kRadix + d] + ex[q] - (uint64_t)ct.y;
-      }
-      if (tile > 0) {
-        uint64_t* row = lookback + tile * kRadix + lane * 8;
-#pragma unroll
-        for (int q = 0; q < 8; q += 2) st_relaxed2(row + q, g[q], g[q + 1]);
-      }
-    }
     // ---- scatter into the (already consumed) stage buffer in digit order
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -738,21 +625,11 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
         sb[wh[d] + r[i]] = k[i];
       }
     }
-    // ---- scanner mode: wait for this tile's exclusive prefix
-    if (LBW < 0 && tid < kRadix) {
-      const uint64_t* wp = &lookback[tile * kRadix + tid];
-      uint64_t w = ld_relaxed(wp);
-      while ((w & (3ull << 62)) != kFlagP || (uint32_t)((w >> 40) & kEpochMask) != ep) {
-        __nanosleep(32);
-        w = ld_relaxed(wp);
-      }
-      s_gofs[tid] = bin_base[digit * kRadix + tid] + (w & kCountMask) - (uint64_t)tstart;
-    }
     // ---- decoupled look-back (thread = digit), LBW predecessors read per round trip
-    if (LBW > 0 && tid < kRadix) {
+    if (tid < kRadix) {
       uint64_t excl = 0;
       if (tile > 0) {
-        excl = lookback_window<(LBW > 0 ? LBW : 1)>(lookback, (int64_t)tile - 1, tid, ep);
+        excl = lookback_window<LBW>(lookback, (int64_t)tile - 1, tid, ep);
         st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
       }
       s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)tstart;
@@ -804,262 +681,6 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
     atomicAdd(&g_phase_dbg[p * 16 + 8], ph_tiles);
   }
 #endif
-}
-
-// ------------------------------------------------------------------------------------------
-// K3 v3: software-pipelined persistent onesweep pass.
-//
-// Three shared-memory tile buffers rotate through the roles  load (TMA bulk, in flight) ->
-// rank + in-place digit-order scatter -> write-out.  Iteration i ranks tile i while the
-// look-back of tile i-1 (whose aggregate was published one iteration earlier) is in flight: its
-// status loads are issued at the start of the iteration and consumed after the ranking, so the
-// predecessors' inclusive prefixes are already published and the L2 round trip is hidden.  Tile
-// i-1 is then written out while tile i is scattered.  Tile ids are claimed one iteration ahead.
-// Forward progress: every tile publishes its aggregate before its CTA waits on any look-back,
-// so a look-back can always walk aggregates down to an inclusive prefix (tile 0 publishes one).
-template <int THREADS, int ITEMS>
-struct PipeSmem {
-  static constexpr int WARPS = THREADS / 32;
-  static constexpr int TILE = THREADS * ITEMS;
-  static constexpr size_t buf_off = 0;                                     // [3][TILE] u64
-  static constexpr size_t whist_off = buf_off + 3ull * TILE * 8;          // [WARPS][257] u32
-  static constexpr size_t thist_off = whist_off + (size_t)WARPS * (kRadix + 1) * 4;  // [257]
-  static constexpr size_t gofs_off = (thist_off + (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [256] u64
-  static constexpr size_t bar_off = gofs_off + kRadix * 8;                 // [3] u64
-  static constexpr size_t swarp_off = bar_off + 32;                        // [8] u64
-  static constexpr size_t tile_off = swarp_off + 64;                       // [3] u32
-  static constexpr size_t bytes = tile_off + 16;
-};
-
-template <int THREADS, int ITEMS, bool IN_F64, int LBW, bool EARLY>
-__global__ void __launch_bounds__(THREADS, 2) k_onesweep_pipe(uint64_t* in, uint64_t* out,
-                                                              uint64_t* tmp, uint64_t n,
-                                                              const RadixPlan* __restrict__ plan,
-                                                              const uint64_t* __restrict__ bin_base,
-                                                              uint64_t* __restrict__ lookback,
-                                                              uint32_t* __restrict__ tile_ctr,
-                                                              uint32_t epoch, int p, int out_f64) {
-  using L = PipeSmem<THREADS, ITEMS>;
-  constexpr int WARPS = L::WARPS;
-  constexpr int TILE = L::TILE;
-  static_assert(THREADS == 256, "one thread per digit, 8 warps");
-  extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* bufs = (uint64_t*)(smem + L::buf_off);
-  uint32_t* whist = (uint32_t*)(smem + L::whist_off);
-  uint32_t* s_thist = (uint32_t*)(smem + L::thist_off);
-  uint64_t* s_gofs = (uint64_t*)(smem + L::gofs_off);
-  uint64_t* bars = (uint64_t*)(smem + L::bar_off);
-  uint64_t* s_warp = (uint64_t*)(smem + L::swarp_off);
-  uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
-
-  const int na = plan->num_active;
-  if (p >= na) return;
-  const int digit = plan->digit[p];
-  const int shift = 8 * digit;
-  const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
-  uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
-  const bool inv = out_f64 && (p == na - 1);
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint64_t num_tiles = (n + TILE - 1) / TILE;
-  const uint32_t ep = epoch & kEpochMask;
-  const uint64_t* __restrict__ bb = bin_base + digit * kRadix;
-
-  auto issue = [&](uint64_t t, int b) {  // thread 0: load tile t into buffer b
-    const uint64_t base = t * (uint64_t)TILE;
-    const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
-    const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
-    // WAR on the buffer (generic reads/writes of the previous tile) is ordered by the
-    // __syncthreads that precedes every issue; no proxy fence is needed for a TMA load.
-    mbar_arrive_expect_tx(&bars[b], bytes);
-    if (bytes) bulk_g2s(bufs + (size_t)b * TILE, src + base, bytes, &bars[b]);
-  };
-
-  uint32_t claim_next = 0;
-  if (tid == 0) {
-    for (int b = 0; b < 3; ++b) mbar_init(&bars[b], 1);
-    mbar_fence_init();
-    const uint32_t t0 = atomicAdd(&tile_ctr[p], 1u);
-    const uint32_t t1 = atomicAdd(&tile_ctr[p], 1u);
-    s_tile[0] = t0;
-    s_tile[1] = t1;
-    if (t0 < num_tiles) issue(t0, 0);
-    if (t1 < num_tiles) issue(t1, 1);
-    claim_next = atomicAdd(&tile_ctr[p], 1u);
-  }
-  __syncthreads();
-
-  const uint32_t lt = lanemask_lt();
-  uint32_t phase = 0;
-  int cur = 0;
-  bool prev_valid = false;
-  uint64_t prev_tile = 0;
-  uint32_t prev_cnt = 0, prev_tstart = 0;
-  uint32_t* wh = whist + warp * (kRadix + 1);
-  const int wofs = warp * 32 * ITEMS + lane;
-
-  while (true) {
-    const uint64_t tile = s_tile[cur];
-    const bool has_cur = tile < num_tiles;
-    if (!has_cur && !prev_valid) break;
-    const int prv = (cur + 2) % 3;
-
-    // (a) look-back loads for the previous tile, in flight during this tile's ranking
-    uint64_t lbw[LBW];
-    if (prev_valid && tid < kRadix) {
-#pragma unroll
-      for (int q = 0; q < LBW; ++q)
-        lbw[q] = ((int64_t)prev_tile - 1 - q >= 0)
-                     ? ld_relaxed(&lookback[(prev_tile - 1 - q) * kRadix + tid])
-                     : (kFlagP | ((uint64_t)ep << 40));
-    }
-
-    // (b) rank the current tile
-    uint64_t k[ITEMS];
-    uint32_t r[ITEMS];
-    uint32_t cnt = 0, tstart = 0;
-    int tile_n = 0;
-    bool full = false;
-    uint64_t* sb = bufs + (size_t)cur * TILE;
-    if (has_cur) {
-      for (int i = tid; i < WARPS * (kRadix + 1); i += THREADS) whist[i] = 0;
-      for (int i = tid; i < kRadix + 1; i += THREADS) s_thist[i] = 0;
-      mbar_wait(&bars[cur], (phase >> cur) & 1u);
-      phase ^= 1u << cur;
-      __syncthreads();
-      const uint64_t tbase = tile * (uint64_t)TILE;
-      const uint64_t rem = n - tbase;
-      tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
-      full = tile_n == TILE;
-      const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
-#pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
-        const int j = wofs + i * 32;
-        uint64_t v;
-        if (full) v = sb[j];
-        else v = j < bulk_n ? sb[j] : (j < tile_n ? src[tbase + j] : 0);
-        k[i] = IN_F64 ? to_key(v) : v;
-      }
-      if (EARLY) {
-        // early counts -> aggregate published before the ranking
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) {
-          const bool valid = full || (wofs + i * 32 < tile_n);
-          atomicAdd(&s_thist[valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix], 1u);
-        }
-        __syncthreads();
-        if (tid < kRadix) {
-          cnt = s_thist[tid];
-          st_relaxed(&lookback[tile * kRadix + tid],
-                     (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
-        }
-        tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
-      }
-      {
-        uint32_t dd[ITEMS], peers[ITEMS];
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) {
-          const bool valid = full || (wofs + i * 32 < tile_n);
-          dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
-        }
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) {
-          const int leader = 31 - __clz(peers[i]);
-          r[i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
-        }
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) {
-          const int leader = 31 - __clz(peers[i]);
-          r[i] = __shfl_sync(0xffffffffu, r[i], leader) + __popc(peers[i] & lt);
-        }
-      }
-      __syncthreads();
-      if (!EARLY) {
-        // counts from the per-warp ranking counters; aggregate published now (its look-back
-        // successors read it one iteration later)
-        if (tid < kRadix) {
-#pragma unroll
-          for (int w = 0; w < WARPS; ++w) cnt += whist[w * (kRadix + 1) + tid];
-          st_relaxed(&lookback[tile * kRadix + tid],
-                     (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
-        }
-        tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
-      }
-      if (tid < kRadix) {
-        uint32_t run = tstart;
-#pragma unroll
-        for (int w = 0; w < WARPS; ++w) {
-          const uint32_t c = whist[w * (kRadix + 1) + tid];
-          whist[w * (kRadix + 1) + tid] = run;
-          run += c;
-        }
-      }
-    }
-    // (c) finish the previous tile's look-back
-    if (prev_valid && tid < kRadix) {
-      uint64_t excl = 0;
-      if (prev_tile > 0) {
-        excl = lookback_window_pre<LBW>(lookback, (int64_t)prev_tile - 1, tid, ep, lbw);
-        st_relaxed(&lookback[prev_tile * kRadix + tid],
-                   kFlagP | ((uint64_t)ep << 40) | (excl + prev_cnt));
-      }
-      s_gofs[tid] = bb[tid] + excl - (uint64_t)prev_tstart;
-    }
-    __syncthreads();
-
-    // (d) write out the previous tile; (e) scatter the current tile in place
-    if (prev_valid) {
-      const uint64_t* pb = bufs + (size_t)prv * TILE;
-      const uint64_t prem = n - prev_tile * (uint64_t)TILE;
-      const int pn = prem < (uint64_t)TILE ? (int)prem : TILE;
-      if (pn == TILE) {
-        uint64_t v[ITEMS], g[ITEMS];
-#pragma unroll
-        for (int q = 0; q < ITEMS; ++q) v[q] = pb[tid + q * THREADS];
-#pragma unroll
-        for (int q = 0; q < ITEMS; ++q) g[q] = s_gofs[(uint32_t)(v[q] >> shift) & 255u];
-        if (inv) {
-#pragma unroll
-          for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = from_key(v[q]);
-        } else {
-#pragma unroll
-          for (int q = 0; q < ITEMS; ++q) dst[g[q] + tid + q * THREADS] = v[q];
-        }
-      } else {
-        for (int j = tid; j < pn; j += THREADS) {
-          const uint64_t v = pb[j];
-          const uint64_t o = s_gofs[(uint32_t)(v >> shift) & 255u] + j;
-          dst[o] = inv ? from_key(v) : v;
-        }
-      }
-    }
-    if (has_cur) {
-#pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
-        if (full || wofs + i * 32 < tile_n) {
-          const uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
-          sb[wh[d] + r[i]] = k[i];
-        }
-      }
-    }
-    __syncthreads();
-
-    // (f) buffer prv is free: load the tile claimed last iteration into it, claim the next one
-    if (tid == 0) {
-      s_tile[prv] = claim_next;
-      if (claim_next < num_tiles) {
-        issue(claim_next, prv);
-        claim_next = atomicAdd(&tile_ctr[p], 1u);
-      }
-    }
-    prev_valid = has_cur;
-    prev_tile = tile;
-    prev_cnt = cnt;
-    prev_tstart = tstart;
-    cur = (cur + 1) % 3;
-    __syncthreads();
-  }
 }
 
 // K1 v2: per-warp entropy probe picks, for each digit, either direct shared atomics (spread
@@ -1188,9 +809,9 @@ cudaError_t next_epoch(RadixScratch& s, cudaStream_t st, uint32_t* ep) {
   return cudaSuccess;
 }
 
-// Kernel variant selection (tuning knob; HSORT_PASS_VARIANT / HSORT_HIST_VARIANT env vars).
-//   pass 0: v1 register-load, one CTA per tile (256 x 16)
-//   pass 1: TMA persistent 256 x 16    2: TMA 512 x 8    3: TMA 384 x 16    4: TMA 512 x 16
+// Kernel selection: the TMA persistent pass (1, default) needs 16-byte aligned buffers; the
+// register-load pass (0) is the fallback.  HSORT_PASS_VARIANT / HSORT_HIST_VARIANT override
+// (experiments; DESIGN.md §6 lists the variants measured and removed).
 int env_int(const char* name, int dflt) {
   const char* v = getenv(name);
   return v ? atoi(v) : dflt;
@@ -1202,17 +823,6 @@ int pass_variant() {
 int hist_variant() {
   static int v = env_int("HSORT_HIST_VARIANT", 1);
   return v;
-}
-
-// keys per tile of the selected pass variant (sizes the look-back array)
-int variant_tile(int v) {
-  switch (v) {
-    case 11: return 256 * 8;
-    case 12: return 256 * 12;
-    case 3: return 384 * 16;
-    case 4: case 7: return 512 * 16;
-    default: return 4096;
-  }
 }
 
 cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
@@ -1254,39 +864,6 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
   const uint64_t tiles = (n + L::TILE - 1) / L::TILE;
   if (tiles > s.max_tiles) return cudaErrorInvalidValue;  // look-back array too small
   uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
-  const uint64_t need = tiles + (LBW < 0 ? 1 : 0);  // scanner mode: one CTA scans
-  if (grid > need) grid = need ? need : 1;
-  if (first_in_f64)
-    kt<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
-                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
-  else
-    kf<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
-                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
-  return cudaGetLastError();
-}
-
-template <int THREADS, int ITEMS, int LBW, bool EARLY = true>
-cudaError_t launch_pipe_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
-                             RadixScratch& s, uint32_t ep, int p, bool first_in_f64, bool out_f64,
-                             cudaStream_t st) {
-  using L = PipeSmem<THREADS, ITEMS>;
-  static int blocks_per_sm[64] = {0};
-  int dev = 0;
-  cudaGetDevice(&dev);
-  auto kt = k_onesweep_pipe<THREADS, ITEMS, true, LBW, EARLY>;
-  auto kf = k_onesweep_pipe<THREADS, ITEMS, false, LBW, EARLY>;
-  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
-  if (!blocks_per_sm[dev]) {
-    cudaError_t e;
-    if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
-    if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
-    int b = 0;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, THREADS, L::bytes)) != cudaSuccess) return e;
-    blocks_per_sm[dev] = b > 0 ? b : 1;
-  }
-  const uint64_t tiles = (n + L::TILE - 1) / L::TILE;
-  if (tiles > s.max_tiles) return cudaErrorInvalidValue;  // look-back array too small
-  uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
   if (grid > tiles) grid = tiles ? tiles : 1;
   if (first_in_f64)
     kt<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
@@ -1305,26 +882,7 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const bool aligned = !(((uintptr_t)in | (uintptr_t)out | (uintptr_t)(tmp ? tmp : out)) & 15);
   const int v = aligned ? pass_variant() : 0;
-  switch (v) {
-    case 1: return launch_tma_pass<256, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 2: return launch_tma_pass<512, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 3: return launch_tma_pass<384, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 4: return launch_tma_pass<512, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 5: return launch_tma_pass<256, 16, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 6: return launch_tma_pass<256, 16, 32>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 7: return launch_tma_pass<512, 16, 16>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 8: return launch_pipe_pass<256, 16, 4>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 9: return launch_pipe_pass<256, 16, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 10: return launch_pipe_pass<256, 16, 4, false>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 11: return launch_tma_pass<256, 8, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 12: return launch_tma_pass<256, 12, 8>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 13: return launch_tma_pass<256, 16, 8, 3>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 14: return launch_tma_pass<256, 16, 0>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 15: return launch_tma_pass<256, 16, 0, 3>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 16: return launch_tma_pass<256, 16, -1>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    case 17: return launch_tma_pass<256, 16, -1, 3>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
-    default: break;
-  }
+  if (v == 1) return launch_tma_pass<256, 16, 8, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
   uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
   if (first_in_f64)
     k_onesweep<kPassThreads, kPassItems, true><<<(unsigned)tiles, kPassThreads, 0, st>>>(
@@ -1372,8 +930,7 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
     if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)
       return e;
   }
-  const int tile_keys = variant_tile(pass_variant()) < kRadixTile ? variant_tile(pass_variant()) : kRadixTile;
-  uint64_t tiles = (n + tile_keys - 1) / tile_keys;
+  uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
   if (tiles < 1) tiles = 1;
   if (tiles > s.max_tiles) {
     if (s.lookback) cudaFree(s.lookback);

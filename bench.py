@@ -266,6 +266,19 @@ def main():
     share = sum(pass_ms) / sum(step_ms) if step_ms else None
 
     # ---- end-to-end arm (e2e): public API, pinned host buffers, HtoD + sort + DtoH ------------
+    # link floor: the first output key depends on the last input key, so HtoD and DtoH of the
+    # whole array serialise: T_floor = n*8/BW_h2d + n*8/BW_d2h (measured here, pinned copies)
+    bw = {}
+    for name, dst_t, src_t in (("h2d", d_out, A_h), ("d2h", B_h, d_in)):
+        dst_t.copy_(src_t, non_blocking=True)
+        torch.cuda.synchronize()
+        e_a, e_b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e_a.record()
+        dst_t.copy_(src_t, non_blocking=True)
+        e_b.record()
+        e_b.synchronize()
+        bw[name] = n * 8 / (e_a.elapsed_time(e_b) / 1e3)
+    link_floor_s = n * 8 / bw["h2d"] + n * 8 / bw["d2h"]
     e2e_steps = args.e2e_steps or max(3, min(args.steps, 5))
     hs.hsort_sort(A_h, B_h, batch_elems=0, n_gpus=1)  # warm (buffers cached)
     barrier()
@@ -322,10 +335,14 @@ def main():
             "unit": "keys/s",
             "h2d_bytes_per_step": n * 8,
             "d2h_bytes_per_step": n * 8,
-            "api": "hsort_sort(A pinned, B pinned, n, batch_elems=0 -> BLINE, n_gpus=1)",
+            "api": "hsort_sort(A pinned, B pinned, n, batch_elems=0 (auto plan), n_gpus=1)",
             "ms_per_step": 1e3 * e2e_total / e2e_steps,
+            "mode": st["mode_name"], "n_b": st["n_b"], "b_s": st["b_s"],
             "t_h2d_s": st["t_h2d"], "t_gpu_sort_s": st["t_gpu_sort"], "t_d2h_s": st["t_d2h"],
-            "mode": st["mode_name"],
+            "t_merge_gpu_s": st["t_merge_gpu"],
+            "link_gbs": {"h2d": bw["h2d"] / 1e9, "d2h": bw["d2h"] / 1e9},
+            "link_floor_ms": 1e3 * link_floor_s,
+            "link_frac": link_floor_s / (e2e_total / e2e_steps),
         },
         "gpu_launches": args.steps * 11,
         "clocks": sampler.summary(),

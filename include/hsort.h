@@ -93,6 +93,9 @@ typedef struct hsort_plan_t {
   uint64_t device_bytes_per_gpu;  /* predicted device footprint */
   uint64_t host_bytes;            /* predicted host working memory (W + staging) */
   double batches_per_stream;      /* n_b / (n_s * n_GPU) */
+  int32_t schedule;               /* 0: uniform b_s batches; 1: b_s batches + halving tail
+                                     (auto RESIDENT plan: the last batch's sort is the only one
+                                     not hidden behind an HtoD) */
 } hsort_plan_t;
 
 /* ---------------------------------------------------------------------------------------------
@@ -114,8 +117,10 @@ int hsort_finalize(void);
  *   B_host       n float64 writable host memory; B == A allowed (in place); partial overlap of
  *                A and B -> HSORT_ERR_INVALID.
  *   n            number of keys; 0 -> HSORT_OK, no-op.
- *   batch_elems  b_s; 0 -> auto (the largest batch with 2*b_s*n_s*8 bytes fitting in HBM,
- *                P:864-870); > n -> clamped to n.  n_b = ceil(n / b_s).
+ *   batch_elems  b_s; > n -> clamped to n; n_b = ceil(n / b_s).  0 -> auto: if n >= option
+ *                "auto_pipeline_min" (2^24) and the runs fit in HBM, a pipelined RESIDENT
+ *                schedule (b_s = min(2^27, n/8) batches + halving tail); else one batch if it
+ *                fits (BLINE), else the largest b_s filling HBM.
  *   n_gpus       1..visible devices; 0 -> all visible; > visible -> HSORT_ERR_INVALID.
  * ------------------------------------------------------------------------------------------- */
 int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_elems, int n_gpus);
@@ -132,7 +137,8 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
  *         STREAM, 1 force RESIDENT), "merge_gpu_permille" (A12 share f in 1/1000; -1 auto),
  *         "pipeline" (1 = overlapped streams PIPEDATA, 0 = blocking BLINEMULTI ablation),
  *         "merge_chunk" (GPU merge output chunk elements), "device_reserve_mb" (HBM left free),
- *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times).
+ *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times),
+ *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never).
  * ------------------------------------------------------------------------------------------- */
 int hsort_set_option(const char* key, int64_t value);
 int hsort_get_option(const char* key, int64_t* value);

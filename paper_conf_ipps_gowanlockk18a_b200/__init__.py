@@ -64,7 +64,7 @@ class hsort_plan_t(ctypes.Structure):
         ("n", _U64), ("b_s", _U64), ("n_b", _U64),
         ("n_gpus", ctypes.c_int32), ("n_s", ctypes.c_int32), ("mode", ctypes.c_int32),
         ("last_batch", _U64), ("device_bytes_per_gpu", _U64), ("host_bytes", _U64),
-        ("batches_per_stream", ctypes.c_double),
+        ("batches_per_stream", ctypes.c_double), ("schedule", ctypes.c_int32),
     ]
 
 

@@ -105,6 +105,7 @@ struct Options {
       {"merge_chunk", 1ll << 26},    // GPU merge output chunk (keys)
       {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
+      {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
   };
   int64_t get(const char* k) const { return v.at(k); }
 };
@@ -257,6 +258,30 @@ struct EvPair {
 // ---- planner (A1) --------------------------------------------------------------------------
 constexpr double kLookbackBytesPerKey = 256.0 * 8.0 / kRadixTile;  // 0.5 B/key
 
+// Batch boundaries (A1).  schedule 0: uniform b_s with a ragged last batch (A-12).
+// schedule 1 (auto RESIDENT): b_s-sized batches, then a halving tail, so the last batch — whose
+// sort is the only one no HtoD can hide — is small (~n/256).
+std::vector<uint64_t> batch_offsets(uint64_t n, uint64_t b_s, int schedule) {
+  std::vector<uint64_t> offs{0};
+  if (n == 0) return offs;
+  if (schedule == 0) {
+    for (uint64_t o = b_s; o < n; o += b_s) offs.push_back(o);
+    offs.push_back(n);
+    return offs;
+  }
+  const uint64_t min_b = std::max<uint64_t>(kRadixTile, (n / 256) & ~(uint64_t)(kRadixTile - 1));
+  uint64_t rem = n;
+  while (rem > 0) {
+    uint64_t sz;
+    if (rem > 2 * b_s) sz = b_s;
+    else if (rem > 2 * min_b) sz = ((rem / 2) + kRadixTile - 1) & ~(uint64_t)(kRadixTile - 1);
+    else sz = rem;
+    offs.push_back(offs.back() + sz);
+    rem -= sz;
+  }
+  return offs;
+}
+
 hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_bytes,
                        const Options& opt) {
   hsort_plan_t p{};
@@ -269,6 +294,30 @@ hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t de
   // single batch footprint: keys + alt + look-back
   auto bline_bytes = [&](uint64_t b) { return (uint64_t)(b * (16.0 + kLookbackBytesPerKey)); };
   uint64_t b_s;
+  int64_t res = opt.get("resident");
+  // auto plan for an array that fits in HBM: a pipelined RESIDENT schedule (HtoD of batch i+1
+  // overlaps the sort of batch i; the merge overlaps the DtoH) beats BLINE's serial
+  // HtoD -> sort -> DtoH once n is large enough for the overlap to matter.
+  const uint64_t auto_min = (uint64_t)std::max<int64_t>(0, opt.get("auto_pipeline_min"));
+  if (batch_elems == 0 && auto_min && n >= auto_min && n_gpus == 1 && res != 0) {
+    uint64_t b0 = std::min<uint64_t>(1ull << 27, std::max<uint64_t>(n / 8, kRadixTile));
+    b0 -= b0 % kRadixTile;
+    const uint64_t rb = n * 8 + (uint64_t)(b0 * (8.0 + kLookbackBytesPerKey)) + merge_buf +
+                        4 * ((uint64_t)opt.get("merge_chunk") / kMergeTile + 1) * 64 * 8;
+    if (rb <= budget) {
+      p.b_s = b0;
+      p.schedule = 1;
+      std::vector<uint64_t> offs = batch_offsets(n, b0, 1);
+      p.n_b = offs.size() - 1;
+      p.last_batch = offs[p.n_b] - offs[p.n_b - 1];
+      p.n_s = 1;
+      p.mode = HSORT_MODE_RESIDENT;
+      p.device_bytes_per_gpu = rb;
+      p.host_bytes = 2ull * (uint64_t)opt.get("n_ring") * (uint64_t)opt.get("p_s");
+      p.batches_per_stream = (double)p.n_b;
+      return p;
+    }
+  }
   if (batch_elems == 0) {
     if (bline_bytes(n) <= budget) {
       b_s = n;
@@ -287,7 +336,6 @@ hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t de
   p.n_b = n ? (n + b_s - 1) / b_s : 0;
   p.last_batch = n ? n - (p.n_b - 1) * b_s : 0;
   p.n_s = p.n_b <= 1 ? 1 : (int)std::min<uint64_t>((uint64_t)n_s, p.n_b);
-  int64_t res = opt.get("resident");
   uint64_t resident_bytes = n * 8 + (uint64_t)(b_s * (8.0 + kLookbackBytesPerKey)) + merge_buf +
                             ((n / kMergeTile + 2) * std::min<uint64_t>(p.n_b, kMaxMergeRuns) * 8);
   if (p.n_b <= 1) {
@@ -358,52 +406,65 @@ void sort_bline(GpuCtx& g, CallCtx& c) {
   ed.destroy();
 }
 
+// GPU merge of k resident runs (K4 + K5), chunk by chunk: the co-ranks of chunk c are computed
+// just before its merge, and the DtoH of chunk c overlaps the merge of chunk c+1 (two output
+// slots), so the first bytes leave the GPU one chunk after the last batch is sorted.
 void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std::vector<uint64_t>& h_off,
-                       Acc& acc, double* t_merge_gpu) {
+                       Acc& acc, double* t_merge_gpu, double* t_d2h) {
   const int k = (int)h_off.size() - 1;
   const uint64_t total = h_off[k] - h_off[0];
   g.off.reserve((k + 1) * 8);
   CK(cudaMemcpyAsync(g.off.p, h_off.data(), (k + 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
   const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
-  g.ranks.reserve((tiles + 1) * (uint64_t)k * 8);
-  EvPair em;
-  em.make();
-  CK(cudaEventRecord(em.a, g.s_comp));
-  CK(merge_corank(d_runs, g.off.u64(), k, total, kMergeTile, tiles + 1, g.ranks.u64(), g.s_comp));
-  uint64_t ctiles = std::max<uint64_t>(1, (uint64_t)c.plan.n ? (uint64_t)S().opt.get("merge_chunk") / kMergeTile : 1);
+  const uint64_t ctiles = std::max<uint64_t>(1, (uint64_t)S().opt.get("merge_chunk") / kMergeTile);
   const uint64_t chunk = ctiles * kMergeTile;
   const uint64_t nch = (total + chunk - 1) / chunk;
   const uint64_t slots = nch > 1 ? 2 : 1;
   g.mout.reserve(slots * chunk * 8);
+  g.ranks.reserve(slots * (ctiles + 1) * (uint64_t)k * 8);
   std::vector<cudaEvent_t> ev_done(slots), ev_free(slots);
+  std::vector<EvPair> em(nch), ed(nch);
   for (uint64_t s = 0; s < slots; ++s) {
     CK(cudaEventCreateWithFlags(&ev_done[s], cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ev_free[s], cudaEventDisableTiming));
     CK(cudaEventRecord(ev_free[s], g.s_d2h));
   }
+  for (uint64_t ch = 0; ch < nch; ++ch) {
+    em[ch].make();
+    ed[ch].make();
+  }
   char* B = (char*)c.B;
   auto enqueue_merge = [&](uint64_t ch) {
-    uint64_t s = ch % slots;
-    uint64_t tb = ch * ctiles, tc = std::min(ctiles, tiles - tb);
+    const uint64_t s = ch % slots;
+    const uint64_t tb = ch * ctiles, tc = std::min(ctiles, tiles - tb);
+    uint64_t* rk = g.ranks.u64() + s * (ctiles + 1) * (uint64_t)k;
     CK(cudaStreamWaitEvent(g.s_comp, ev_free[s], 0));
-    CK(merge_tiles(d_runs, g.off.u64(), k, total, g.ranks.u64(), tb, tc,
-                   g.mout.u64() + s * chunk, ch * chunk, c.f64, g.s_comp));
+    CK(cudaEventRecord(em[ch].a, g.s_comp));
+    CK(merge_corank(d_runs, g.off.u64(), k, total, kMergeTile, tb, tc + 1, rk, g.s_comp));
+    CK(merge_tiles(d_runs, g.off.u64(), k, total, rk, tb, tb, tc, g.mout.u64() + s * chunk,
+                   ch * chunk, c.f64, g.s_comp));
+    CK(cudaEventRecord(em[ch].b, g.s_comp));
     CK(cudaEventRecord(ev_done[s], g.s_comp));
   };
   enqueue_merge(0);
   for (uint64_t ch = 0; ch < nch; ++ch) {
     if (ch + 1 < nch) enqueue_merge(ch + 1);
-    if (ch + 1 == nch) CK(cudaEventRecord(em.b, g.s_comp));
-    uint64_t s = ch % slots;
-    uint64_t o = ch * chunk, len = std::min(chunk, total - o);
+    const uint64_t s = ch % slots;
+    const uint64_t o = ch * chunk, len = std::min(chunk, total - o);
     CK(cudaStreamWaitEvent(g.s_d2h, ev_done[s], 0));
+    CK(cudaEventRecord(ed[ch].a, g.s_d2h));
     download(g, B + o * 8, g.mout.u64() + s * chunk, len * 8, g.s_d2h, c.direct_out, c.mc_threads, acc);
+    CK(cudaEventRecord(ed[ch].b, g.s_d2h));
     CK(cudaEventRecord(ev_free[s], g.s_d2h));
   }
   CK(cudaStreamSynchronize(g.s_d2h));
   CK(cudaStreamSynchronize(g.s_comp));
-  *t_merge_gpu += em.ms() / 1e3;
-  em.destroy();
+  for (uint64_t ch = 0; ch < nch; ++ch) {
+    *t_merge_gpu += em[ch].ms() / 1e3;
+    *t_d2h += ed[ch].ms() / 1e3;
+    em[ch].destroy();
+    ed[ch].destroy();
+  }
   for (uint64_t s = 0; s < slots; ++s) {
     cudaEventDestroy(ev_done[s]);
     cudaEventDestroy(ev_free[s]);
@@ -413,6 +474,8 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std:
 void sort_resident(GpuCtx& g, CallCtx& c) {
   CK(cudaSetDevice(g.dev));
   const uint64_t n = c.n, b_s = c.plan.b_s, n_b = c.plan.n_b;
+  const std::vector<uint64_t> h_off = batch_offsets(n, b_s, c.plan.schedule);
+  if (h_off.size() != n_b + 1) throw HsortError(HSORT_ERR_INTERNAL, "batch schedule mismatch");
   g.runs.reserve(n * 8);
   g.alt.reserve(b_s * 8);
   Acc acc;
@@ -422,7 +485,7 @@ void sort_resident(GpuCtx& g, CallCtx& c) {
   auto t0 = Clock::now();
   int passes = 0;
   for (uint64_t i = 0; i < n_b; ++i) {
-    uint64_t o = i * b_s, len = std::min(b_s, n - o);
+    const uint64_t o = h_off[i], len = h_off[i + 1] - h_off[i];
     CK(cudaEventRecord(eh[i].a, g.s_h2d));
     upload(g, g.runs.u64() + o, (const char*)c.A + o * 8, len * 8, g.s_h2d, c.direct_in, c.mc_threads, acc);
     CK(cudaEventRecord(eh[i].b, g.s_h2d));
@@ -435,12 +498,11 @@ void sort_resident(GpuCtx& g, CallCtx& c) {
   passes = g.rs.h_plan->num_active;  // plan of the last batch
   c.st->t_sort_phase = secs_since(t0);
   auto t1 = Clock::now();
-  std::vector<uint64_t> h_off(n_b + 1);
-  for (uint64_t i = 0; i <= n_b; ++i) h_off[i] = std::min(i * b_s, n);
-  double tmg = 0;
-  gpu_merge_to_host(g, c, g.runs.u64(), h_off, acc, &tmg);
+  double tmg = 0, tdh = 0;
+  gpu_merge_to_host(g, c, g.runs.u64(), h_off, acc, &tmg, &tdh);
   c.st->t_merge_phase = secs_since(t1);
   c.st->t_merge_gpu = tmg;
+  c.st->t_d2h = tdh;
   c.st->merge_gpu_fraction = 1.0;
   for (uint64_t i = 0; i < n_b; ++i) {
     c.st->t_h2d += eh[i].ms() / 1e3;
@@ -1009,7 +1071,7 @@ int hsort_device_corank(const uint64_t* d_keys, const uint64_t* h_off, int k, ui
     g.off.reserve((k + 1) * 8);
     cudaStream_t st = (cudaStream_t)stream;
     CK(cudaMemcpyAsync(g.off.p, h_off, (k + 1) * 8, cudaMemcpyHostToDevice, st));
-    CK(merge_corank(d_keys, g.off.u64(), k, h_off[k] - h_off[0], step, n_bounds, d_ranks, st));
+    CK(merge_corank(d_keys, g.off.u64(), k, h_off[k] - h_off[0], step, 0, n_bounds, d_ranks, st));
     CK(cudaStreamSynchronize(st));
     return HSORT_OK;
   });
@@ -1029,8 +1091,8 @@ int hsort_device_merge(const uint64_t* d_keys, const uint64_t* h_off, int k, uin
     CK(cudaMemcpyAsync(g.off.p, h_off, (k + 1) * 8, cudaMemcpyHostToDevice, st));
     const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
     g.ranks.reserve((tiles + 1) * (uint64_t)k * 8);
-    CK(merge_corank(d_keys, g.off.u64(), k, total, kMergeTile, tiles + 1, g.ranks.u64(), st));
-    CK(merge_tiles(d_keys, g.off.u64(), k, total, g.ranks.u64(), 0, tiles, d_out, 0, out_f64 != 0, st));
+    CK(merge_corank(d_keys, g.off.u64(), k, total, kMergeTile, 0, tiles + 1, g.ranks.u64(), st));
+    CK(merge_tiles(d_keys, g.off.u64(), k, total, g.ranks.u64(), 0, 0, tiles, d_out, 0, out_f64 != 0, st));
     CK(cudaStreamSynchronize(st));
     return HSORT_OK;
   });

@@ -68,13 +68,16 @@ cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, 
 constexpr int kMergeTile = 4096;  // output keys per merge CTA
 constexpr int kMaxMergeRuns = 1024;
 
-// K4: ranks[(b)*k + j] for b in [0, n_bounds): co-ranks of o_b = min(b*step, total).
+// K4: ranks[b*k + j] for b in [0, n_bounds): co-ranks of o = min((bound_begin + b)*step, total).
 cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                         uint64_t step, uint64_t n_bounds, uint64_t* ranks, cudaStream_t st);
+                         uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
+                         cudaStream_t st);
 // K5: merge tiles [tile_begin, tile_begin + tile_count) (tile t = output [t*kMergeTile, ...)),
-// given ranks for boundaries of step kMergeTile; writes out[o - out_origin].
+// given co-ranks of boundaries t = rank_tile0, rank_tile0 + 1, ... (row t - rank_tile0 of
+// `ranks`, step kMergeTile); writes out[o - out_origin].
 cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                        const uint64_t* ranks, uint64_t tile_begin, uint64_t tile_count,
-                        uint64_t* out, uint64_t out_origin, bool out_f64, cudaStream_t st);
+                        const uint64_t* ranks, uint64_t rank_tile0, uint64_t tile_begin,
+                        uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
+                        cudaStream_t st);
 
 }  // namespace hsort

@@ -63,12 +63,12 @@ __device__ __forceinline__ uint64_t upper_bound(const uint64_t* a, uint64_t lo, 
 template <int C>
 __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ keys,
                                                 const uint64_t* __restrict__ off, int k,
-                                                uint64_t total, uint64_t step, uint64_t nb,
-                                                uint64_t* __restrict__ ranks) {
+                                                uint64_t total, uint64_t step, uint64_t b0,
+                                                uint64_t nb, uint64_t* __restrict__ ranks) {
   const uint64_t b = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (b >= nb) return;
-  const uint64_t o = b * step < total ? b * step : total;
+  const uint64_t o = (b0 + b) * step < total ? (b0 + b) * step : total;
   uint64_t base[C], lo[C], hi[C];
 #pragma unroll
   for (int c = 0; c < C; ++c) {
@@ -175,8 +175,8 @@ constexpr int kMergeIPT = kMergeTile / kMergeThreads;
 
 __global__ void __launch_bounds__(kMergeThreads) k_merge_tile(
     const uint64_t* __restrict__ keys, const uint64_t* __restrict__ off, int k, uint64_t total,
-    const uint64_t* __restrict__ ranks, uint64_t tile_begin, uint64_t* __restrict__ out,
-    uint64_t out_origin, int out_f64) {
+    const uint64_t* __restrict__ ranks, uint64_t rank_tile0, uint64_t tile_begin,
+    uint64_t* __restrict__ out, uint64_t out_origin, int out_f64) {
   extern __shared__ __align__(16) unsigned char smem[];
   uint64_t* bufA = (uint64_t*)smem;
   uint64_t* bufB = bufA + kMergeTile;
@@ -189,7 +189,7 @@ __global__ void __launch_bounds__(kMergeThreads) k_merge_tile(
   const uint64_t o0 = t * (uint64_t)kMergeTile;
   const uint64_t o1 = (o0 + kMergeTile < total) ? o0 + kMergeTile : total;
   const int L = (int)(o1 - o0);
-  const uint64_t* r0 = ranks + t * (uint64_t)k;
+  const uint64_t* r0 = ranks + (t - rank_tile0) * (uint64_t)k;
   const uint64_t* r1 = r0 + k;
   const int tid = threadIdx.x;
 
@@ -311,22 +311,24 @@ constexpr size_t merge_smem_bytes() {
 }  // namespace
 
 cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                         uint64_t step, uint64_t n_bounds, uint64_t* ranks, cudaStream_t st) {
+                         uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
+                         cudaStream_t st) {
   if (k < 1 || k > kMaxMergeRuns) return cudaErrorInvalidValue;
   if (n_bounds == 0) return cudaSuccess;
   const unsigned grid = (unsigned)((n_bounds * 32 + 127) / 128);
   int C = (k + 31) / 32;
-  if (C <= 1) k_corank<1><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, n_bounds, ranks);
-  else if (C <= 2) k_corank<2><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, n_bounds, ranks);
-  else if (C <= 4) k_corank<4><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, n_bounds, ranks);
-  else if (C <= 8) k_corank<8><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, n_bounds, ranks);
-  else k_corank<kMaxC><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, n_bounds, ranks);
+  if (C <= 1) k_corank<1><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
+  else if (C <= 2) k_corank<2><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
+  else if (C <= 4) k_corank<4><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
+  else if (C <= 8) k_corank<8><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
+  else k_corank<kMaxC><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
   return cudaGetLastError();
 }
 
 cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                        const uint64_t* ranks, uint64_t tile_begin, uint64_t tile_count,
-                        uint64_t* out, uint64_t out_origin, bool out_f64, cudaStream_t st) {
+                        const uint64_t* ranks, uint64_t rank_tile0, uint64_t tile_begin,
+                        uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
+                        cudaStream_t st) {
   if (tile_count == 0) return cudaSuccess;
   static bool attr_set[64] = {false};
   int dev = 0;
@@ -339,8 +341,8 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint
     attr_set[dev] = true;
   }
   k_merge_tile<<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, d_off, k, total, ranks,
-                                                                  tile_begin, out, out_origin,
-                                                                  out_f64 ? 1 : 0);
+                                                                  rank_tile0, tile_begin, out,
+                                                                  out_origin, out_f64 ? 1 : 0);
   return cudaGetLastError();
 }
 

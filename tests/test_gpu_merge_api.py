@@ -114,6 +114,25 @@ def test_hsort_sort_distributions(hs_gpu, oracle_mod, inputs_mod, dist):
         assert np.array_equal(_bits(hs_gpu.hsort_sort(A, batch_elems=b)), want), (dist, b)
 
 
+@pytest.mark.parametrize("dist", ["special", "zipf_dup", "uniform"])
+def test_hsort_sort_auto_pipelined_schedule(hs_gpu, oracle_mod, inputs_mod, dist):
+    """auto plan at n >= 2^24: RESIDENT with b_s batches + halving tail, GPU merge, chunked DtoH."""
+    n = (1 << 24) + 12345
+    A = inputs_mod.generate(dist, n, seed=31)
+    want = _bits(oracle_mod.sort_f64(A))
+    hs_gpu.hsort_set_option("merge_chunk", 1 << 20)  # several merge/DtoH chunks
+    try:
+        B = hs_gpu.hsort_sort(A)
+        st = hs_gpu.hsort_get_stats()
+        Bp = _pinned(np.zeros_like(A))
+        hs_gpu.hsort_sort(_pinned(A.copy()), Bp)
+    finally:
+        hs_gpu.hsort_set_option("merge_chunk", 1 << 26)
+    assert st["mode_name"] == "RESIDENT" and st["n_b"] > 8
+    assert np.array_equal(_bits(B), want)
+    assert np.array_equal(_bits(Bp.numpy()), want)
+
+
 def test_hsort_sort_in_place_and_u64(hs_gpu, oracle_mod, inputs_mod):
     A = inputs_mod.generate("special", 500_001, seed=4)
     want = _bits(oracle_mod.sort_f64(A))

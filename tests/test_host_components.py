@@ -110,8 +110,21 @@ def test_planner_table1_identities(hs):
 
 def test_planner_modes_and_ragged_batches(hs):
     G = 180 << 30
+    # auto plan: pipelined RESIDENT schedule (b_s = 2^27 batches + halving tail)
     p = hs.hsort_plan(1 << 30, 0, 1, G)
-    assert p["mode_name"] == "BLINE" and p["n_b"] == 1 and p["b_s"] == 1 << 30
+    assert p["mode_name"] == "RESIDENT" and p["schedule"] == 1 and p["b_s"] == 1 << 27
+    assert p["n_b"] == 12 and p["last_batch"] == 1 << 23
+    p = hs.hsort_plan(10**9 + 7, 0, 1, G)
+    assert p["mode_name"] == "RESIDENT" and p["schedule"] == 1 and p["n_b"] <= 1024
+    assert p["last_batch"] <= (10**9 + 7) // 128
+    hs.hsort_set_option("auto_pipeline_min", 0)
+    try:
+        p = hs.hsort_plan(1 << 30, 0, 1, G)  # the paper's auto rule: one batch if it fits
+        assert p["mode_name"] == "BLINE" and p["n_b"] == 1 and p["b_s"] == 1 << 30
+    finally:
+        hs.hsort_set_option("auto_pipeline_min", 1 << 24)
+    p = hs.hsort_plan((1 << 24) - 1, 0, 1, G)  # below the threshold: BLINE
+    assert p["mode_name"] == "BLINE"
     p = hs.hsort_plan(10**9 + 7, 250_000_000, 1, G)
     assert p["n_b"] == 5 and p["last_batch"] == 7 and p["mode_name"] == "RESIDENT"
     p = hs.hsort_plan(3 * 10**10, 250_000_000, 1, G)  # 240 GB: runs cannot stay in HBM

@@ -196,6 +196,11 @@ int hsort_device_corank(const uint64_t* d_keys, const uint64_t* h_off, int k, ui
 int hsort_device_merge(const uint64_t* d_keys, const uint64_t* h_off, int k, uint64_t* d_out,
                        int out_f64, void* stream);
 
+/* Splitter partition of one sorted uint64 run (multi-GPU exchange):
+ * d_out[i] = number of keys <= d_values[i] in d_keys[0, n).  Device pointers; synchronous. */
+int hsort_device_upper_bounds(const uint64_t* d_keys, uint64_t n, const uint64_t* d_values,
+                              uint64_t m, uint64_t* d_out, void* stream);
+
 /* ---------------------------------------------------------------------------------------------
  * Host-native components (no GPU needed)
  * ------------------------------------------------------------------------------------------- */
@@ -212,6 +217,10 @@ int hsort_host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t*
 /* Exact co-ranks of output position o over the k host runs (same definition as K4). */
 int hsort_host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o,
                       uint64_t* ranks);
+
+/* Host version of hsort_device_upper_bounds (keys, values, out in host memory). */
+int hsort_host_upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
+                            uint64_t* out);
 
 /* The PIPEMERGE heuristic (reading A-9): number of pair-wise merges overlapped with
  * GPU sorting.  Pure arithmetic. */

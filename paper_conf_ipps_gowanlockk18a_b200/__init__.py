@@ -92,6 +92,8 @@ SIGNATURES = {
     "hsort_pipemerge_count": ([_U64, _I], _U64),
     "hsort_device_count": ([], _I),
     "hsort_get_kernel_times": ([ctypes.POINTER(ctypes.c_float), _I, ctypes.POINTER(_I)], _I),
+    "hsort_device_upper_bounds": ([_P, _U64, _P, _U64, _P, _P], _I),
+    "hsort_host_upper_bounds": ([_P, _U64, _P, _U64, _P], _I),
 }
 
 
@@ -313,6 +315,20 @@ def hsort_get_kernel_times() -> dict:
     out = {"num_active": na.value}
     if m >= 11:
         out.update(hist=v[0], scan=v[1], passes=v[2:10], copy=v[10])
+    return out
+
+
+def hsort_device_upper_bounds(d_keys, d_values, d_out, stream=None) -> None:
+    _check(lib().hsort_device_upper_bounds(_dev_ptr(d_keys), d_keys.numel(), _dev_ptr(d_values),
+                                           d_values.numel(), _dev_ptr(d_out), _stream_ptr(stream)))
+
+
+def hsort_host_upper_bounds(keys: np.ndarray, values: np.ndarray) -> np.ndarray:
+    keys = np.ascontiguousarray(keys, dtype=np.uint64)
+    values = np.ascontiguousarray(values, dtype=np.uint64)
+    out = np.empty(values.size, dtype=np.uint64)
+    _check(lib().hsort_host_upper_bounds(keys.ctypes.data, keys.size, values.ctypes.data,
+                                         values.size, out.ctypes.data))
     return out
 
 

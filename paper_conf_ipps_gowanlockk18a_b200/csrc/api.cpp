@@ -1098,6 +1098,34 @@ int hsort_device_merge(const uint64_t* d_keys, const uint64_t* h_off, int k, uin
   });
 }
 
+int hsort_device_upper_bounds(const uint64_t* d_keys, uint64_t n, const uint64_t* d_values,
+                              uint64_t m, uint64_t* d_out, void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (m && (!d_values || !d_out || (n && !d_keys))) return g_err = "null pointer", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    cudaStream_t st = (cudaStream_t)stream;
+    CK(upper_bounds(d_keys, n, d_values, m, d_out, st));
+    CK(cudaStreamSynchronize(st));
+    return HSORT_OK;
+  });
+}
+
+int hsort_host_upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
+                            uint64_t* out) {
+  if (m && (!values || !out || (n && !keys))) return g_err = "null pointer", HSORT_ERR_INVALID;
+  for (uint64_t i = 0; i < m; ++i) {
+    uint64_t lo = 0, hi = n;
+    while (lo < hi) {
+      const uint64_t mid = lo + ((hi - lo) >> 1);
+      if (keys[mid] <= values[i]) lo = mid + 1;
+      else hi = mid;
+    }
+    out[i] = lo;
+  }
+  return HSORT_OK;
+}
+
 int hsort_par_memcpy(void* dst, const void* src, uint64_t bytes, int threads) {
   if (bytes && (!dst || !src)) return g_err = "null pointer", HSORT_ERR_INVALID;
   return guarded([&]() -> int {

@@ -80,4 +80,8 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint
                         uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
                         cudaStream_t st);
 
+// out[i] = #keys <= values[i] in the sorted run keys[0, n) (device pointers).
+cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
+                         uint64_t* out, cudaStream_t st);
+
 }  // namespace hsort

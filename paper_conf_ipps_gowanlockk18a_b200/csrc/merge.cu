@@ -303,6 +303,15 @@ __global__ void __launch_bounds__(kMergeThreads) k_merge_tile(
   }
 }
 
+// Splitter partition of one sorted run (multi-GPU exchange): out[i] = number of
+// keys <= values[i].  One thread per value; values sorted or not.
+__global__ void k_upper_bounds(const uint64_t* __restrict__ keys, uint64_t n,
+                               const uint64_t* __restrict__ values, uint64_t m,
+                               uint64_t* __restrict__ out) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < m) out[i] = upper_bound(keys, 0, n, values[i]);
+}
+
 constexpr size_t merge_smem_bytes() {
   return 2 * kMergeTile * sizeof(uint64_t) + 2 * (kMaxMergeRuns + 1) * sizeof(uint32_t) +
          kMaxMergeRuns * sizeof(uint64_t);
@@ -322,6 +331,13 @@ cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uin
   else if (C <= 4) k_corank<4><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
   else if (C <= 8) k_corank<8><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
   else k_corank<kMaxC><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
+  return cudaGetLastError();
+}
+
+cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
+                         uint64_t* out, cudaStream_t st) {
+  if (m == 0) return cudaSuccess;
+  k_upper_bounds<<<(unsigned)((m + 255) / 256), 256, 0, st>>>(keys, n, values, m, out);
   return cudaGetLastError();
 }
 

@@ -1,4 +1,6 @@
 """GPU parity: K4 co-ranks, K5 merge, and the host->host hsort_sort in every mode vs the oracle."""
+import os
+
 import numpy as np
 import pytest
 
@@ -58,6 +60,38 @@ def test_device_merge_inverse_transform(hs_gpu, oracle_mod, inputs_mod):
     d_out = torch.empty_like(d_keys)
     hs_gpu.hsort_device_merge(d_keys, off, d_out, True)
     assert np.array_equal(d_out.cpu().numpy(), _bits(oracle_mod.sort_f64(A)))
+
+
+@pytest.mark.parametrize("hi", [2**64, 40])
+def test_device_upper_bounds_match_host(hs_gpu, hi):
+    import torch
+    rng = np.random.default_rng(hi % 1000)
+    keys = np.sort(rng.integers(0, hi, size=100_003, dtype=np.uint64))
+    vals = rng.integers(0, hi, size=1000, dtype=np.uint64)
+    vals[:3] = [0, 2**64 - 1, keys[500]]
+    d_out = torch.empty(vals.size, dtype=torch.uint64, device="cuda")
+    hs_gpu.hsort_device_upper_bounds(torch.from_numpy(keys).cuda(), torch.from_numpy(vals).cuda(), d_out)
+    want = np.searchsorted(keys, vals, side="right").astype(np.uint64)
+    assert np.array_equal(d_out.cpu().numpy(), want)
+    assert np.array_equal(hs_gpu.hsort_host_upper_bounds(keys, vals), want)
+
+
+def test_exchange_single_rank_cuda_path(hs_gpu, oracle_mod, inputs_mod):
+    """dist.exchange_sorted_runs on one NCCL rank (the P == 1 path + device merge)."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_gowanlockk18a_b200 import dist as hd
+    A = inputs_mod.generate("salted", 100_000, seed=5)
+    K = oracle_mod.sort_u64(oracle_mod.keys_from_f64(A))
+    if not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29581")
+        dist.init_process_group("nccl", rank=0, world_size=1)
+    try:
+        out = hd.exchange_sorted_runs(torch.from_numpy(K).cuda(), out_f64=True)
+        assert np.array_equal(out.view(torch.uint64).cpu().numpy(), _bits(oracle_mod.sort_f64(A)))
+    finally:
+        dist.destroy_process_group()
 
 
 # ---- host -> host ------------------------------------------------------------------------------

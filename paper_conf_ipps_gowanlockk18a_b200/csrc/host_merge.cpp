@@ -6,9 +6,12 @@
 // is merged independently by one thread with a loser tree (ceil(log2 k) compares per key); the
 // inverse key transform is fused into the store.  Keys are the order-preserving uint64 view of the
 // float64 bits, so compares are plain unsigned compares.
+#include <emmintrin.h>
+
 #include <algorithm>
 #include <cstdint>
 #include <cstring>
+#include <new>
 #include <vector>
 
 #include "pool.h"
@@ -39,63 +42,92 @@ inline uint64_t lb(const uint64_t* a, uint64_t lo, uint64_t hi, uint64_t v) {
   return lo;
 }
 
-// Loser tree over K (power of two) leaves; dead leaves lose to every live one.
+// Loser tree over K (power of two) leaves, branch-free replay.  Each node holds a (key, src)
+// pair compared lexicographically; a live leaf has src = leaf index (< K) and an exhausted leaf
+// has key = 2^64-1 and src = K + leaf, so it loses to every live key, including a live 2^64-1.
 class LoserTree {
  public:
-  LoserTree(int k) : k_(k) {
+  explicit LoserTree(int k) {
     K_ = 1;
     while (K_ < k) K_ <<= 1;
-    key_.assign(K_, ~0ull);
-    dead_.assign(K_, 1);
-    pos_.assign(K_, 0);
-    end_.assign(K_, 0);
-    tree_.assign(K_, 0);
+    tk_.assign(K_, ~0ull);
+    ts_.assign(K_, 0);
+    cur_.assign(K_, nullptr);
+    end_.assign(K_, nullptr);
   }
   void set_leaf(int j, const uint64_t* p, const uint64_t* e) {
-    pos_[j] = p;
+    cur_[j] = p;
     end_[j] = e;
-    dead_[j] = (p >= e);
-    key_[j] = dead_[j] ? ~0ull : *p;
   }
   void build() {
-    // winners bottom-up, storing losers
-    std::vector<int> win(2 * K_);
-    for (int i = 0; i < K_; ++i) win[K_ + i] = i;
-    for (int n = K_ - 1; n >= 1; --n) {
-      int a = win[2 * n], b = win[2 * n + 1];
-      if (less(b, a)) std::swap(a, b);
-      win[n] = a;
-      tree_[n] = b;
+    std::vector<uint64_t> wk(2 * K_);
+    std::vector<uint32_t> ws(2 * K_);
+    for (int i = 0; i < K_; ++i) {
+      const bool live = cur_[i] && cur_[i] < end_[i];
+      wk[K_ + i] = live ? *cur_[i] : ~0ull;
+      ws[K_ + i] = live ? (uint32_t)i : (uint32_t)(K_ + i);
     }
-    tree_[0] = win[1];
+    for (int v = K_ - 1; v >= 1; --v) {
+      uint64_t ak = wk[2 * v], bk = wk[2 * v + 1];
+      uint32_t as = ws[2 * v], bs = ws[2 * v + 1];
+      const bool bwins = (bk < ak) | ((bk == ak) & (bs < as));
+      wk[v] = bwins ? bk : ak;
+      ws[v] = bwins ? bs : as;
+      tk_[v] = bwins ? ak : bk;
+      ts_[v] = bwins ? as : bs;
+    }
+    win_k_ = wk[1];
+    win_s_ = ws[1];
   }
-  inline bool less(int a, int b) const {
-    if (dead_[a]) return false;
-    if (dead_[b]) return true;
-    return key_[a] < key_[b] || (key_[a] == key_[b] && a < b);
-  }
-  // pop the minimum (caller guarantees one live leaf)
+  // pop the minimum (caller guarantees a live leaf remains)
   inline uint64_t pop() {
-    int w = tree_[0];
-    uint64_t out = key_[w];
-    const uint64_t* p = ++pos_[w];
-    if (p < end_[w]) key_[w] = *p;
-    else dead_[w] = 1;
-    for (int n = (w + K_) >> 1; n >= 1; n >>= 1) {
-      int l = tree_[n];
-      if (less(l, w)) { tree_[n] = w; w = l; }
+    const uint64_t out = win_k_;
+    const uint32_t leaf = win_s_;
+    const uint64_t* p = ++cur_[leaf];
+    uint64_t nk;
+    uint32_t ns;
+    if (__builtin_expect(p < end_[leaf], 1)) {
+      nk = *p;
+      ns = leaf;
+    } else {
+      nk = ~0ull;
+      ns = (uint32_t)K_ + leaf;
     }
-    tree_[0] = w;
+    uint64_t* tk = tk_.data();
+    uint32_t* ts = ts_.data();
+    for (uint32_t v = ((uint32_t)K_ + leaf) >> 1; v >= 1; v >>= 1) {
+      // swap (loser <-> candidate) when the stored loser beats the candidate; masks, no branches
+      const uint64_t lk = tk[v];
+      const uint32_t ls = ts[v];
+      const uint64_t sw = (uint64_t)((lk < nk) | ((lk == nk) & (ls < ns)));
+      const uint64_t mk = 0 - sw;
+      const uint32_t ms = 0u - (uint32_t)sw;
+      const uint64_t dk = (lk ^ nk) & mk;
+      const uint32_t ds = (ls ^ ns) & ms;
+      tk[v] = lk ^ dk;
+      ts[v] = ls ^ ds;
+      nk ^= dk;
+      ns ^= ds;
+    }
+    win_k_ = nk;
+    win_s_ = ns;
     return out;
   }
 
  private:
-  int k_, K_;
-  std::vector<uint64_t> key_;
-  std::vector<uint8_t> dead_;
-  std::vector<const uint64_t*> pos_, end_;
-  std::vector<int> tree_;
+  int K_;
+  std::vector<uint64_t> tk_;
+  std::vector<uint32_t> ts_;
+  std::vector<const uint64_t*> cur_, end_;
+  uint64_t win_k_ = 0;
+  uint32_t win_s_ = 0;
 };
+
+// Non-temporal 8-byte store (MOVNTI): the merge output is written once and not re-read, so it
+// bypasses the cache and avoids the read-for-ownership of B (host DRAM bytes).
+inline void st_nt(uint64_t* p, uint64_t v) {
+  _mm_stream_si64((long long*)p, (long long)v);
+}
 
 }  // namespace
 
@@ -160,11 +192,11 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
   if (live == 0) return;
   if (live == 1) {
     const uint64_t* s = keys + off[last] + ra[last];
-    uint64_t len = rb[last] - ra[last];
+    const uint64_t len = rb[last] - ra[last];
     if (out_f64)
-      for (uint64_t i = 0; i < len; ++i) out[i] = from_key(s[i]);
+      for (uint64_t i = 0; i < len; ++i) st_nt(out + i, from_key(s[i]));
     else
-      std::memcpy(out, s, len * 8);
+      for (uint64_t i = 0; i < len; ++i) st_nt(out + i, s[i]);
     return;
   }
   if (live == 2) {
@@ -175,28 +207,58 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
     const uint64_t *q = keys + off[b] + ra[b], *qe = keys + off[b] + rb[b];
     uint64_t* o = out;
     while (p < pe && q < qe) {
-      uint64_t x = *p, y = *q;
-      bool takep = x <= y;
-      uint64_t v = takep ? x : y;
+      const uint64_t x = *p, y = *q;
+      const bool takep = x <= y;
+      const uint64_t v = takep ? x : y;
       p += takep;
       q += !takep;
-      *o++ = out_f64 ? from_key(v) : v;
+      st_nt(o++, out_f64 ? from_key(v) : v);
     }
-    while (p < pe) { *o++ = out_f64 ? from_key(*p) : *p; ++p; }
-    while (q < qe) { *o++ = out_f64 ? from_key(*q) : *q; ++q; }
+    while (p < pe) { st_nt(o++, out_f64 ? from_key(*p) : *p); ++p; }
+    while (q < qe) { st_nt(o++, out_f64 ? from_key(*q) : *q); ++q; }
     return;
   }
-  LoserTree lt(k);
+  // k >= 3: the range is cut into NI sub-ranges by exact co-ranks and NI loser trees are
+  // advanced in lock step, so NI independent replay chains are in flight (each pop depends on the
+  // previous one of its own tree only).
+  constexpr int NI = 4;
   uint64_t total = 0;
-  for (int j = 0; j < k; ++j) {
-    lt.set_leaf(j, keys + off[j] + ra[j], keys + off[j] + rb[j]);
-    total += rb[j] - ra[j];
+  for (int j = 0; j < k; ++j) total += rb[j] - ra[j];
+  uint64_t oa = 0;
+  for (int j = 0; j < k; ++j) oa += ra[j];  // absolute output position of this range
+  std::vector<uint64_t> cr((NI + 1) * (size_t)k);
+  std::memcpy(&cr[0], ra, k * 8);
+  std::memcpy(&cr[(size_t)NI * k], rb, k * 8);
+  for (int i = 1; i < NI; ++i) host_corank(keys, off, k, oa + total * i / NI, &cr[(size_t)i * k]);
+  LoserTree* lt[NI];
+  alignas(64) unsigned char mem[NI][sizeof(LoserTree)];
+  uint64_t len[NI], pos[NI];
+  for (int i = 0; i < NI; ++i) {
+    lt[i] = new (mem[i]) LoserTree(k);
+    len[i] = 0;
+    for (int j = 0; j < k; ++j) {
+      lt[i]->set_leaf(j, keys + off[j] + cr[(size_t)i * k + j], keys + off[j] + cr[(size_t)(i + 1) * k + j]);
+      len[i] += cr[(size_t)(i + 1) * k + j] - cr[(size_t)i * k + j];
+    }
+    pos[i] = i == 0 ? 0 : pos[i - 1] + len[i - 1];
+    lt[i]->build();
   }
-  lt.build();
-  if (out_f64)
-    for (uint64_t i = 0; i < total; ++i) out[i] = from_key(lt.pop());
-  else
-    for (uint64_t i = 0; i < total; ++i) out[i] = lt.pop();
+  uint64_t m = len[0];
+  for (int i = 1; i < NI; ++i) m = std::min(m, len[i]);
+  if (out_f64) {
+    for (uint64_t t = 0; t < m; ++t)
+      for (int i = 0; i < NI; ++i) st_nt(out + pos[i] + t, from_key(lt[i]->pop()));
+  } else {
+    for (uint64_t t = 0; t < m; ++t)
+      for (int i = 0; i < NI; ++i) st_nt(out + pos[i] + t, lt[i]->pop());
+  }
+  for (int i = 0; i < NI; ++i) {
+    for (uint64_t t = m; t < len[i]; ++t) {
+      const uint64_t v = lt[i]->pop();
+      st_nt(out + pos[i] + t, out_f64 ? from_key(v) : v);
+    }
+    lt[i]->~LoserTree();
+  }
 }
 
 void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, bool out_f64,
@@ -219,6 +281,7 @@ void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out,
     uint64_t o = (uint64_t)((__uint128_t)total * (uint64_t)r / (uint64_t)R);
     merge_range(K, o2.data(), k, &ranks[(uint64_t)r * k], &ranks[(uint64_t)(r + 1) * k], out + o,
                 out_f64);
+    _mm_sfence();
   });
 }
 

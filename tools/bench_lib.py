@@ -1,0 +1,19 @@
+"""Time the device sort with an alternative libhsort build (argv[1] = .so path), 2^30 uniform."""
+import json, os, statistics, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_ipps_gowanlockk18a_b200 as hs
+hs.LIB_PATH = os.path.abspath(sys.argv[1])
+import torch
+import hsort_inputs
+n = 1 << 30
+hs.hsort_set_option("kernel_timing", 1)
+hs.hsort_init()
+A = hsort_inputs.generate("uniform", n, seed=2)
+d_in = torch.from_numpy(A).cuda(); d_out = torch.empty_like(d_in)
+for _ in range(3): hs.hsort_sort_device(d_in, d_out)
+torch.cuda.synchronize()
+ps = []
+for _ in range(5):
+    hs.hsort_sort_device(d_in, d_out); torch.cuda.synchronize()
+    kt = hs.hsort_get_kernel_times(); ps += kt["passes"][:kt["num_active"]]
+print(json.dumps({"lib": sys.argv[1], "pass_ms": statistics.mean(ps), "per_pass": [round(x, 3) for x in kt["passes"]]}))

@@ -83,6 +83,7 @@ typedef struct hsort_stats {
   double t_init;           /* hsort_init() duration (pinned + device allocation) */
   uint64_t bytes_h2d;      /* bytes moved host -> device */
   uint64_t bytes_d2h;      /* bytes moved device -> host */
+  double t_host_alloc;     /* pinned working-memory (W) allocation in this call (cached after) */
 } hsort_stats;
 
 /* Planner output (A1).  Pure host arithmetic; see hsort_plan(). */
@@ -138,7 +139,8 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
  *         "pipeline" (1 = overlapped streams PIPEDATA, 0 = blocking BLINEMULTI ablation),
  *         "merge_chunk" (GPU merge output chunk elements), "device_reserve_mb" (HBM left free),
  *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times),
- *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never).
+ *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never),
+ *         "pin_w" (1 = STREAM-mode W in cached pinned memory, 0 = pageable).
  * ------------------------------------------------------------------------------------------- */
 int hsort_set_option(const char* key, int64_t value);
 int hsort_get_option(const char* key, int64_t* value);

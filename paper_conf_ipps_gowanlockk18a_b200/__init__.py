@@ -55,7 +55,7 @@ class hsort_stats(ctypes.Structure):
         ("t_h2d", ctypes.c_double), ("t_d2h", ctypes.c_double), ("t_stage", ctypes.c_double),
         ("t_merge_cpu", ctypes.c_double), ("t_merge_gpu", ctypes.c_double),
         ("t_init", ctypes.c_double),
-        ("bytes_h2d", _U64), ("bytes_d2h", _U64),
+        ("bytes_h2d", _U64), ("bytes_d2h", _U64), ("t_host_alloc", ctypes.c_double),
     ]
 
 

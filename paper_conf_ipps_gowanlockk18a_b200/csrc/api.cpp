@@ -39,6 +39,8 @@ namespace hsort {
 void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, uint64_t* ranks);
 void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, bool out_f64,
                 int threads);
+void host_merge_range(const uint64_t* keys, const uint64_t* off, int k, uint64_t o_lo,
+                      uint64_t o_hi, uint64_t* out, bool out_f64, int threads);
 }  // namespace hsort
 
 using namespace hsort;
@@ -106,6 +108,7 @@ struct Options {
       {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
       {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
+      {"pin_w", 1},                  // STREAM: W in cached pinned memory (direct DMA) vs pageable
   };
   int64_t get(const char* k) const { return v.at(k); }
 };
@@ -114,7 +117,7 @@ struct GpuCtx {
   int dev = -1;
   cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
   RadixScratch rs;
-  DevBuf runs, alt, mout, ranks, off;
+  DevBuf runs, alt, mout, min, ranks, off;
   std::vector<char*> ring_in, ring_out;
   uint64_t ring_bytes = 0;
   std::vector<cudaEvent_t> ev_in, ev_out;
@@ -130,6 +133,11 @@ struct State {
   Options opt;
   hsort_stats last{};
   double t_init = 0;
+  // pinned working memory W (STREAM mode), allocated once and reused: pinning is expensive
+  // so it is cached like the staging ring
+  void* w_pin = nullptr;
+  size_t w_pin_bytes = 0;
+  double r_cpu_merge = 0;  // last measured CPU merge rate (keys/s), for the A12 split
 };
 State& S() {
   static State s;
@@ -517,26 +525,133 @@ void sort_resident(GpuCtx& g, CallCtx& c) {
   for (auto& e : es) e.destroy();
 }
 
+// GPU share of the STREAM merge: output positions [o_lo, o_hi) of the merge of the k runs in
+// host memory W, in chunks of `merge_chunk` keys: exact co-ranks on the host, HtoD of the k
+// slices (direct from pinned W), K4/K5 on the GPU, DtoH into B.  Two slots: the HtoD of chunk c+1
+// overlaps the merge and DtoH of chunk c.
+void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const uint64_t* W, const std::vector<uint64_t>& off,
+                         uint64_t o_lo, uint64_t o_hi, bool w_direct, double* t_gpu) {
+  CK(cudaSetDevice(g.dev));
+  const int k = (int)off.size() - 1;
+  const uint64_t C = std::max<uint64_t>(
+      kMergeTile, ((uint64_t)S().opt.get("merge_chunk") / kMergeTile) * kMergeTile);
+  const uint64_t nch = (o_hi - o_lo + C - 1) / C;
+  const uint64_t tiles_c = C / kMergeTile;
+  g.min.reserve(2 * C * 8);
+  g.mout.reserve(2 * C * 8);
+  g.ranks.reserve(2 * (tiles_c + 1) * (uint64_t)k * 8);
+  g.off.reserve(2 * (k + 1) * 8);
+  std::vector<uint64_t> cr((nch + 1) * (size_t)k);
+  host_pool().parallel_for((int64_t)nch + 1, host_threads(), [&](int64_t i) {
+    const uint64_t p = std::min(o_lo + (uint64_t)i * C, o_hi);
+    host_corank(W, off.data(), k, p, &cr[(size_t)i * k]);
+  });
+  cudaEvent_t in_ready[2], in_free[2], merged[2], out_free[2];
+  for (int s = 0; s < 2; ++s) {
+    CK(cudaEventCreateWithFlags(&in_ready[s], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&in_free[s], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&merged[s], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&out_free[s], cudaEventDisableTiming));
+    CK(cudaEventRecord(in_free[s], g.s_comp));
+    CK(cudaEventRecord(out_free[s], g.s_d2h));
+  }
+  EvPair em;
+  em.make();
+  std::vector<uint64_t> hoff(2 * (size_t)(k + 1));
+  Acc acc;
+  CK(cudaEventRecord(em.a, g.s_h2d));
+  for (uint64_t ch = 0; ch < nch; ++ch) {
+    const int s = (int)(ch & 1);
+    const uint64_t* r0 = &cr[(size_t)ch * k];
+    const uint64_t* r1 = &cr[(size_t)(ch + 1) * k];
+    uint64_t* din = g.min.u64() + (uint64_t)s * C;
+    uint64_t* ho = &hoff[(size_t)s * (k + 1)];
+    ho[0] = 0;
+    CK(cudaStreamWaitEvent(g.s_h2d, in_free[s], 0));
+    for (int j = 0; j < k; ++j) {
+      const uint64_t len = r1[j] - r0[j];
+      ho[j + 1] = ho[j] + len;
+      if (len) upload(g, din + ho[j], W + off[j] + r0[j], len * 8, g.s_h2d, w_direct, c.mc_threads, acc);
+    }
+    uint64_t* doff = g.off.u64() + (size_t)s * (k + 1);
+    CK(cudaMemcpyAsync(doff, ho, (k + 1) * 8, cudaMemcpyHostToDevice, g.s_h2d));
+    CK(cudaEventRecord(in_ready[s], g.s_h2d));
+    const uint64_t total = ho[k];
+    const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
+    uint64_t* rk = g.ranks.u64() + (uint64_t)s * (tiles_c + 1) * k;
+    uint64_t* dout = g.mout.u64() + (uint64_t)s * C;
+    CK(cudaStreamWaitEvent(g.s_comp, in_ready[s], 0));
+    CK(cudaStreamWaitEvent(g.s_comp, out_free[s], 0));
+    CK(merge_corank(din, doff, k, total, kMergeTile, 0, tiles + 1, rk, g.s_comp));
+    CK(merge_tiles(din, doff, k, total, rk, 0, 0, tiles, dout, 0, c.f64, g.s_comp));
+    CK(cudaEventRecord(in_free[s], g.s_comp));
+    CK(cudaEventRecord(merged[s], g.s_comp));
+    CK(cudaStreamWaitEvent(g.s_d2h, merged[s], 0));
+    const uint64_t p0 = o_lo + ch * C;
+    download(g, (uint64_t*)c.B + p0, dout, total * 8, g.s_d2h, c.direct_out, c.mc_threads, acc);
+    CK(cudaEventRecord(out_free[s], g.s_d2h));
+    // the pageable host offsets of the other slot are rewritten next iteration: its copy must be done
+    if (ch + 1 < nch) CK(cudaEventSynchronize(in_ready[s ^ 1]));
+  }
+  CK(cudaEventRecord(em.b, g.s_d2h));
+  CK(cudaStreamSynchronize(g.s_d2h));
+  CK(cudaStreamSynchronize(g.s_comp));
+  *t_gpu = em.ms() / 1e3;
+  em.destroy();
+  for (int s = 0; s < 2; ++s) {
+    cudaEventDestroy(in_ready[s]);
+    cudaEventDestroy(in_free[s]);
+    cudaEventDestroy(merged[s]);
+    cudaEventDestroy(out_free[s]);
+  }
+}
+
 // STREAM mode: batches -> W (host) through per-GPU uploader/downloader threads, then the CPU
 // multiway merge W -> B.
 void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   const uint64_t n = c.n, b_s = c.plan.b_s, n_b = c.plan.n_b;
   const int n_s = std::max(1, c.plan.n_s);
   const bool pipelined = S().opt.get("pipeline") != 0;
-  // W: working memory for the sorted sublists; transformed uint64 keys
+  // W: working memory for the sorted sublists; transformed uint64 keys.
+  // Pinned and cached across calls when possible (runs then DMA straight into W and the GPU merge
+  // share streams straight out of it); pageable mmap otherwise.
   uint64_t* W = nullptr;
-  {
-    size_t bytes = n * 8;
-    void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  bool w_direct = false;
+  void* w_map = nullptr;
+  if (S().opt.get("pin_w")) {
+    if (S().w_pin_bytes < n * 8) {
+      if (S().w_pin) cudaFreeHost(S().w_pin);
+      S().w_pin = nullptr;
+      S().w_pin_bytes = 0;
+      auto ta = Clock::now();
+      void* p = nullptr;
+      if (cudaHostAlloc(&p, n * 8, cudaHostAllocDefault) == cudaSuccess) {
+        S().w_pin = p;
+        S().w_pin_bytes = n * 8;
+      } else {
+        cudaGetLastError();
+      }
+      c.st->t_host_alloc = secs_since(ta);
+    }
+    if (S().w_pin) {
+      W = (uint64_t*)S().w_pin;
+      w_direct = true;
+    }
+  }
+  if (!W) {
+    void* p = mmap(nullptr, n * 8, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
     if (p == MAP_FAILED) throw HsortError(HSORT_ERR_HOST_OOM, "mmap W failed");
-    madvise(p, bytes, MADV_HUGEPAGE);
+    madvise(p, n * 8, MADV_HUGEPAGE);
     W = (uint64_t*)p;
+    w_map = p;
   }
   struct WFree {
     void* p;
     size_t b;
-    ~WFree() { munmap(p, b); }
-  } wfree{W, n * 8};
+    ~WFree() {
+      if (p) munmap(p, b);
+    }
+  } wfree{w_map, n * 8};
 
   std::atomic<uint64_t> next_batch{0};
   std::mutex err_m;
@@ -600,7 +715,7 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
           CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), len, c.f64, false, g.s_comp));
           CK(cudaEventRecord(it->es.b, g.s_comp));
           CK(cudaEventRecord(it->ed.a, g.s_comp));
-          download(g, W + o, g.runs.p, len * 8, g.s_comp, false, c.mc_threads, P.down);
+          download(g, W + o, g.runs.p, len * 8, g.s_comp, w_direct, c.mc_threads, P.down);
           CK(cudaEventRecord(it->ed.b, g.s_comp));
           CK(cudaStreamSynchronize(g.s_comp));
           P.passes += g.rs.h_plan->num_active;
@@ -621,7 +736,7 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
               uint64_t o = it->batch * b_s, len = std::min(b_s, n - o);
               CK(cudaStreamWaitEvent(g.s_d2h, ev_sorted[it->slot], 0));
               CK(cudaEventRecord(it->ed.a, g.s_d2h));
-              download(g, W + o, g.runs.u64() + (uint64_t)it->slot * b_s, len * 8, g.s_d2h, false,
+              download(g, W + o, g.runs.u64() + (uint64_t)it->slot * b_s, len * 8, g.s_d2h, w_direct,
                        c.mc_threads, P.down);
               CK(cudaEventRecord(it->ed.b, g.s_d2h));
               CK(cudaEventSynchronize(it->ed.b));
@@ -717,14 +832,52 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
     c.st->bytes_d2h += P.down.d2h;
     c.st->passes_run += P.passes;
   }
-  // Merge: CPU multiway merge of the n_b runs in W into B.
+  // Merge with the CPU/GPU split of A12: the GPU merges output positions [0, o_f)
+  // by streaming co-ranked slices of W through HBM (K4/K5), while the host threads merge
+  // [o_f, n) with loser trees; f balances the two measured rates (the split cannot be
+  // derived asymptotically, it must be measured).
   auto t1 = Clock::now();
   std::vector<uint64_t> off(n_b + 1);
   for (uint64_t i = 0; i <= n_b; ++i) off[i] = std::min(i * b_s, n);
-  host_merge(W, off.data(), (int)n_b, (uint64_t*)c.B, c.f64, c.merge_threads);
-  c.st->t_merge_cpu = secs_since(t1);
-  c.st->t_merge_phase = c.st->t_merge_cpu;
-  c.st->merge_gpu_fraction = 0.0;
+  const int k = (int)n_b;
+  double f = 0.0;
+  const int64_t fp = S().opt.get("merge_gpu_permille");
+  if (k <= kMaxMergeRuns && !gs.empty()) {
+    if (fp >= 0) {
+      f = fp / 1000.0;
+    } else {
+      // GPU share is link-bound (HtoD in, DtoH out, duplex); CPU rate from the last STREAM call
+      const double bw_in = c.st->t_h2d > 0 ? c.st->bytes_h2d / c.st->t_h2d : 50e9;
+      const double bw_out = c.st->t_d2h > 0 ? c.st->bytes_d2h / c.st->t_d2h : 50e9;
+      const double r_gpu = 0.85 * std::min(bw_in, bw_out) / 8.0;
+      const double r_cpu = S().r_cpu_merge > 0 ? S().r_cpu_merge : 4e7 * host_threads();
+      f = r_gpu / (r_gpu + r_cpu);
+    }
+  }
+  const uint64_t o_f = std::min<uint64_t>(n, (uint64_t)((double)n * f));
+  double t_cpu = 0, t_gpu = 0;
+  std::thread cpu_part([&] {
+    auto tc = Clock::now();
+    host_merge_range(W, off.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64, c.merge_threads);
+    t_cpu = secs_since(tc);
+  });
+  std::string gpu_err;
+  int gpu_code = 0;
+  if (o_f > 0) {
+    try {
+      gpu_merge_from_host(*gs[0], c, W, off, 0, o_f, w_direct, &t_gpu);
+    } catch (const HsortError& e) {
+      gpu_code = e.code;
+      gpu_err = e.what();
+    }
+  }
+  cpu_part.join();
+  if (gpu_code) throw HsortError(gpu_code, gpu_err);
+  if (n > o_f + (1u << 20) && t_cpu > 0) S().r_cpu_merge = (double)(n - o_f) / t_cpu;
+  c.st->t_merge_cpu = t_cpu;
+  c.st->t_merge_gpu = t_gpu;
+  c.st->t_merge_phase = secs_since(t1);
+  c.st->merge_gpu_fraction = (double)o_f / (double)n;
 }
 
 void ctx_create(GpuCtx& g, int dev, const Options& opt) {
@@ -762,6 +915,7 @@ void ctx_destroy(GpuCtx& g) {
   g.runs.release();
   g.alt.release();
   g.mout.release();
+  g.min.release();
   g.ranks.release();
   g.off.release();
   radix_scratch_release(g.rs);
@@ -923,6 +1077,9 @@ int hsort_init(void) {
 
 int hsort_finalize(void) {
   std::lock_guard<std::mutex> lk(S().m);
+  if (S().w_pin) cudaFreeHost(S().w_pin);
+  S().w_pin = nullptr;
+  S().w_pin_bytes = 0;
   for (auto& g : S().gpus) ctx_destroy(g);
   S().gpus.clear();
   S().inited = false;

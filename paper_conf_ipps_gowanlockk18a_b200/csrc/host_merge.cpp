@@ -261,28 +261,35 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
   }
 }
 
-void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, bool out_f64,
-                int threads) {
+// Merge positions [o_lo, o_hi) of the multiway merge of the k runs keys[off[j] .. off[j+1]) into
+// out[0 .. o_hi - o_lo).  The range is cut into ~4 pieces per thread by exact co-ranks.
+void host_merge_range(const uint64_t* keys, const uint64_t* off, int k, uint64_t o_lo,
+                      uint64_t o_hi, uint64_t* out, bool out_f64, int threads) {
   if (threads <= 0) threads = host_threads();
   const uint64_t total = off[k] - off[0];
-  if (total == 0) return;
-  // normalise offsets to start at 0 relative to keys + off[0]
+  if (o_hi > total) o_hi = total;
+  if (o_lo >= o_hi) return;
   std::vector<uint64_t> o2(k + 1);
   for (int j = 0; j <= k; ++j) o2[j] = off[j] - off[0];
   const uint64_t* K = keys + off[0];
+  const uint64_t span = o_hi - o_lo;
   // ranges: ~4 per thread, each at least 64K keys
-  int64_t R = std::max<int64_t>(1, std::min<int64_t>((int64_t)threads * 4, (int64_t)(total >> 16)));
+  int64_t R = std::max<int64_t>(1, std::min<int64_t>((int64_t)threads * 4, (int64_t)(span >> 16)));
   std::vector<uint64_t> ranks((R + 1) * (uint64_t)k);
+  auto pos = [&](int64_t r) { return o_lo + (uint64_t)((__uint128_t)span * (uint64_t)r / (uint64_t)R); };
   host_pool().parallel_for(R + 1, threads, [&](int64_t r) {
-    uint64_t o = (uint64_t)((__uint128_t)total * (uint64_t)r / (uint64_t)R);
-    host_corank(K, o2.data(), k, o, &ranks[(uint64_t)r * k]);
+    host_corank(K, o2.data(), k, pos(r), &ranks[(uint64_t)r * k]);
   });
   host_pool().parallel_for(R, threads, [&](int64_t r) {
-    uint64_t o = (uint64_t)((__uint128_t)total * (uint64_t)r / (uint64_t)R);
-    merge_range(K, o2.data(), k, &ranks[(uint64_t)r * k], &ranks[(uint64_t)(r + 1) * k], out + o,
-                out_f64);
+    merge_range(K, o2.data(), k, &ranks[(uint64_t)r * k], &ranks[(uint64_t)(r + 1) * k],
+                out + (pos(r) - o_lo), out_f64);
     _mm_sfence();
   });
+}
+
+void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, bool out_f64,
+                int threads) {
+  host_merge_range(keys, off, k, 0, off[k] - off[0], out, out_f64, threads);
 }
 
 }  // namespace hsort

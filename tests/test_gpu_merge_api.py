@@ -167,6 +167,36 @@ def test_hsort_sort_auto_pipelined_schedule(hs_gpu, oracle_mod, inputs_mod, dist
     assert np.array_equal(_bits(Bp.numpy()), want)
 
 
+@pytest.mark.parametrize("permille", [0, 300, 1000, -1])
+@pytest.mark.parametrize("pin_w", [1, 0])
+def test_stream_merge_split(hs_gpu, oracle_mod, inputs_mod, permille, pin_w):
+    """A12: STREAM mode with a GPU share f of the merge streamed from W (K4/K5) and the rest on
+    the CPU loser trees; every split point must give the same bytes."""
+    n = 3_000_017
+    A = inputs_mod.generate("zipf_dup", n, seed=permille + 7)
+    want = _bits(oracle_mod.sort_f64(A))
+    opts = {"resident": 0, "merge_gpu_permille": permille, "pin_w": pin_w, "merge_chunk": 1 << 19}
+    old = {k: hs_gpu.hsort_get_option(k) for k in opts}
+    for k, v in opts.items():
+        hs_gpu.hsort_set_option(k, v)
+    try:
+        for pinned in (False, True):
+            if pinned:
+                Bp = _pinned(np.zeros_like(A))
+                hs_gpu.hsort_sort(_pinned(A.copy()), Bp, batch_elems=400_000)
+                B = Bp.numpy()
+            else:
+                B = hs_gpu.hsort_sort(A, batch_elems=400_000)
+            st = hs_gpu.hsort_get_stats()
+            assert st["mode_name"] == "STREAM" and st["n_b"] == 8
+            assert np.array_equal(_bits(B), want), (permille, pin_w, pinned)
+            if permille >= 0:
+                assert abs(st["merge_gpu_fraction"] - permille / 1000) < 1e-3
+    finally:
+        for k, v in old.items():
+            hs_gpu.hsort_set_option(k, v)
+
+
 def test_hsort_sort_in_place_and_u64(hs_gpu, oracle_mod, inputs_mod):
     A = inputs_mod.generate("special", 500_001, seed=4)
     want = _bits(oracle_mod.sort_f64(A))

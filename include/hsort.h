@@ -140,7 +140,8 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
  *         "merge_chunk" (GPU merge output chunk elements), "device_reserve_mb" (HBM left free),
  *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times),
  *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never),
- *         "pin_w" (1 = STREAM-mode W in cached pinned memory, 0 = pageable).
+ *         "pin_w" (STREAM-mode W: 1 cached pinned, 0 pageable + staging, -1 auto = pinned up to
+ *         "pin_w_max_mb" (16 GiB) or when a large enough pinned W is already cached).
  * ------------------------------------------------------------------------------------------- */
 int hsort_set_option(const char* key, int64_t value);
 int hsort_get_option(const char* key, int64_t* value);

@@ -108,7 +108,8 @@ struct Options {
       {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
       {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
-      {"pin_w", 1},                  // STREAM: W in cached pinned memory (direct DMA) vs pageable
+      {"pin_w", -1},                 // STREAM W: 1 cached pinned, 0 pageable, -1 pinned if <= pin_w_max_mb
+      {"pin_w_max_mb", 16384},       // auto pinning limit: pinning runs at ~2.5 GB/s
   };
   int64_t get(const char* k) const { return v.at(k); }
 };
@@ -618,7 +619,10 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   uint64_t* W = nullptr;
   bool w_direct = false;
   void* w_map = nullptr;
-  if (S().opt.get("pin_w")) {
+  const int64_t pin_w = S().opt.get("pin_w");
+  const bool want_pin = pin_w == 1 ||
+      (pin_w == -1 && (n * 8 <= ((uint64_t)S().opt.get("pin_w_max_mb") << 20) || S().w_pin_bytes >= n * 8));
+  if (want_pin) {
     if (S().w_pin_bytes < n * 8) {
       if (S().w_pin) cudaFreeHost(S().w_pin);
       S().w_pin = nullptr;
@@ -1107,6 +1111,7 @@ int hsort_set_option(const char* key, int64_t value) {
   if (k == "merge_chunk" && value < kMergeTile) return g_err = "merge_chunk too small", HSORT_ERR_INVALID;
   if (k == "merge_gpu_permille" && (value < -1 || value > 1000)) return g_err = "bad permille", HSORT_ERR_INVALID;
   if (k == "resident" && (value < -1 || value > 1)) return g_err = "resident in {-1,0,1}", HSORT_ERR_INVALID;
+  if (k == "pin_w" && (value < -1 || value > 1)) return g_err = "pin_w in {-1,0,1}", HSORT_ERR_INVALID;
   if (S().inited && (k == "p_s" || k == "n_ring")) {
     g_err = k + " must be set before hsort_init";
     return HSORT_ERR_BUSY;

@@ -417,7 +417,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 // per round trip (independent loads in flight) and accumulates aggregates back to the first
 // inclusive prefix.  A serial walk costs one L2 round trip per step and, with tiles claimed a
 // few tens of cycles apart, needs ~latency/interval steps; the window resolves them together.
-template <int W>
+template <int W, int BO = 0>
 __device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__ lookback,
                                                     int64_t j, int d, uint32_t ep) {
   uint64_t excl = 0;
@@ -442,6 +442,7 @@ __device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__
       else ++q;
     }
     if (done) return excl;
+    if (BO > 0 && q == 0) __nanosleep(BO);  // predecessor not published yet: back off the L2
     j -= q;  // all consumed aggregates; re-read from the first unavailable tile
   }
 }
@@ -579,8 +580,26 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
         const bool valid = full || (wofs + (c0 + i) * 32 < tile_n);
         dd[i] = valid ? ((uint32_t)(k[c0 + i] >> shift) & 255u) : (uint32_t)kRadix;
       }
+      // peers (lanes holding the same digit) by an 8-ballot multisplit: on sm_100a MATCH.ANY
+      // over random 8-bit digits costs 1.9 SM-cycles/key, the ballots 1.0
+      // (profiles/r01_microbench_ranking2.txt).  Partial tiles mark invalid items with bit 8.
 #pragma unroll
-      for (int i = 0; i < RC; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+      for (int i = 0; i < RC; ++i) peers[i] = 0xffffffffu;
+#pragma unroll
+      for (int b = 0; b < 8; ++b) {
+#pragma unroll
+        for (int i = 0; i < RC; ++i) {
+          const uint32_t bit = (dd[i] >> b) & 1u;
+          peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+        }
+      }
+      if (!full) {
+#pragma unroll
+        for (int i = 0; i < RC; ++i) {
+          const uint32_t bit = (dd[i] >> 8) & 1u;
+          peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+        }
+      }
 #pragma unroll
       for (int i = 0; i < RC; ++i) {
         const int leader = 31 - __clz(peers[i]);
@@ -629,7 +648,7 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
     if (tid < kRadix) {
       uint64_t excl = 0;
       if (tile > 0) {
-        excl = lookback_window<LBW>(lookback, (int64_t)tile - 1, tid, ep);
+        excl = lookback_window<(LBW & 255), (LBW >> 8)>(lookback, (int64_t)tile - 1, tid, ep);
         st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
       }
       s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)tstart;
@@ -882,7 +901,7 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const bool aligned = !(((uintptr_t)in | (uintptr_t)out | (uintptr_t)(tmp ? tmp : out)) & 15);
   const int v = aligned ? pass_variant() : 0;
-  if (v == 1) return launch_tma_pass<256, 16, 8, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+  if (v == 1) return launch_tma_pass<256, 16, 2, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
   uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
   if (first_in_f64)
     k_onesweep<kPassThreads, kPassItems, true><<<(unsigned)tiles, kPassThreads, 0, st>>>(

@@ -18,7 +18,8 @@ struct RadixPlan {
   int32_t copy_src;     // -1: no final copy; else buffer id copied to out (with conversion)
   int32_t copy_in_f64;  // conversion of the final copy: source is float64 bits
   int32_t copy_out_f64; // conversion of the final copy: destination is float64 bits
-  int32_t pad;
+  int32_t match_mask;   // bit p: pass p ranks with MATCH.ANY (few distinct digits per warp),
+                        // else with the 8-ballot multisplit
 };
 
 struct RadixScratch {

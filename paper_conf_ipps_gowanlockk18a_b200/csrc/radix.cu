@@ -167,6 +167,7 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
                                                    int in_eq_out, int in_f64, int out_f64) {
   __shared__ uint64_t s_warp[8];
   __shared__ int s_nz[kDigits];
+  __shared__ float s_dist[kDigits][8];
   const int t = threadIdx.x;
   for (int p = 0; p < kDigits; ++p) {
     uint64_t v = hist[p * kRadix + t];
@@ -174,6 +175,14 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
     bin_base[p * kRadix + t] = e;
     int nz = __syncthreads_count(v != 0);
     if (t == 0) s_nz[p] = nz;
+    // expected number of distinct digits among 32 keys: D = sum_b 1 - (1 - p_b)^32.  MATCH.ANY
+    // costs ~0.06 SM-cycles/key per distinct value, the ballot multisplit ~1.0 (microbench).
+    float q = n ? 1.0f - (float)v / (float)n : 1.0f;
+    float q2 = q * q, q4 = q2 * q2, q8 = q4 * q4, q16 = q8 * q8;
+    float term = 1.0f - q16 * q16;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) term += __shfl_xor_sync(0xffffffffu, term, o);
+    if ((t & 31) == 0) s_dist[p][t >> 5] = term;
   }
   __syncthreads();
   if (t == 0) {
@@ -186,7 +195,12 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
     P.copy_src = -1;
     P.copy_in_f64 = 0;
     P.copy_out_f64 = 0;
-    P.pad = 0;
+    P.match_mask = 0;
+    for (int q = 0; q < na; ++q) {
+      float dsum = 0;
+      for (int w = 0; w < 8; ++w) dsum += s_dist[P.digit[q]][w];
+      if (dsum < 12.0f) P.match_mask |= 1 << q;
+    }
     // ping-pong assignment: buffers 0 = in, 1 = out, 2 = tmp; the last pass must land in out
     int cur = 0;
     if (!in_eq_out) {
@@ -229,7 +243,7 @@ __global__ void k_force_plan(RadixPlan* plan, int digit) {
   P.src[0] = 0;
   P.dst[0] = 1;
   P.copy_src = -1;
-  P.copy_in_f64 = P.copy_out_f64 = P.pad = 0;
+  P.copy_in_f64 = P.copy_out_f64 = P.match_mask = 0;
   *plan = P;
 }
 
@@ -497,6 +511,7 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
   const int shift = 8 * digit;
   const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
   uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const bool use_match = (plan->match_mask >> p) & 1;
   const bool inv = out_f64 && (p == na - 1);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t num_tiles = (n + TILE - 1) / TILE;
@@ -580,24 +595,30 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
         const bool valid = full || (wofs + (c0 + i) * 32 < tile_n);
         dd[i] = valid ? ((uint32_t)(k[c0 + i] >> shift) & 255u) : (uint32_t)kRadix;
       }
-      // peers (lanes holding the same digit) by an 8-ballot multisplit: on sm_100a MATCH.ANY
-      // over random 8-bit digits costs 1.9 SM-cycles/key, the ballots 1.0
-      // (profiles/r01_microbench_ranking2.txt).  Partial tiles mark invalid items with bit 8.
+      // peers (lanes holding the same digit).  MATCH.ANY costs ~0.06 SM-cycles/key per distinct
+      // value in the warp (1.9 for random 8-bit digits), an 8-ballot multisplit ~1.0
+      // (profiles/r01_microbench_ranking2.txt); K2 picks per pass from the digit histogram.
+      // Partial tiles mark invalid items with bit 8.
+      if (use_match) {
 #pragma unroll
-      for (int i = 0; i < RC; ++i) peers[i] = 0xffffffffu;
+        for (int i = 0; i < RC; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+      } else {
 #pragma unroll
-      for (int b = 0; b < 8; ++b) {
+        for (int i = 0; i < RC; ++i) peers[i] = 0xffffffffu;
 #pragma unroll
-        for (int i = 0; i < RC; ++i) {
-          const uint32_t bit = (dd[i] >> b) & 1u;
-          peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+        for (int b = 0; b < 8; ++b) {
+#pragma unroll
+          for (int i = 0; i < RC; ++i) {
+            const uint32_t bit = (dd[i] >> b) & 1u;
+            peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+          }
         }
-      }
-      if (!full) {
+        if (!full) {
 #pragma unroll
-        for (int i = 0; i < RC; ++i) {
-          const uint32_t bit = (dd[i] >> 8) & 1u;
-          peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+          for (int i = 0; i < RC; ++i) {
+            const uint32_t bit = (dd[i] >> 8) & 1u;
+            peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+          }
         }
       }
 #pragma unroll

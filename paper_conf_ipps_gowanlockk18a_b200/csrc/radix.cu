@@ -482,8 +482,7 @@ struct TmaPassSmem {
   static constexpr size_t bar_off = gofs_off + kRadix * 8;                 // [2] u64
   static constexpr size_t swarp_off = bar_off + 16;                        // [8] u64
   static constexpr size_t tile_off = swarp_off + 64;                       // [2] u32
-  static constexpr size_t thist_off = tile_off + 16;                       // [257] u32 (early counts)
-  static constexpr size_t bytes = thist_off + (kRadix + 1) * 4;
+  static constexpr size_t bytes = tile_off + 16;
 };
 
 template <int THREADS, int ITEMS, bool IN_F64, int LBW, int MINB>
@@ -513,8 +512,6 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
   const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
   uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
   const bool use_match = (plan->match_mask >> p) & 1;
-  constexpr bool EARLY = (LBW >> 16) & 1;  // publish the tile aggregate before ranking
-  uint32_t* s_thist = (uint32_t*)(smem + L::thist_off);
   const bool inv = out_f64 && (p == na - 1);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t num_tiles = (n + TILE - 1) / TILE;
@@ -561,8 +558,6 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
       }
     }
     for (int i = tid; i < WARPS * (kRadix + 1); i += THREADS) whist[i] = 0;
-    if (EARLY)
-      for (int i = tid; i < kRadix + 1; i += THREADS) s_thist[i] = 0;
     mbar_wait(&bars[cb], (phase >> cb) & 1u);
     phase ^= 1u << cb;
     __syncthreads();
@@ -587,27 +582,38 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
       else v = j < bulk_n ? sb[j] : (j < tile_n ? src[tbase + j] : 0);
       k[i] = IN_F64 ? to_key(v) : v;
     }
-    uint64_t cnt = 0;
-    uint32_t tstart = 0;
-    if (EARLY) {
-      // early counts: the aggregate is published before the ranking, so successors' look-backs
-      // never wait on it
+    // ---- early per-warp digit counts -> tile aggregate, published before the ranking (so a
+    // successor's look-back never waits on it), and absolute shared-memory bases per
+    // (warp, digit): tile-local digit start + the counts of the warps before.
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
-        const bool valid = full || (wofs + i * 32 < tile_n);
-        atomicAdd(&s_thist[valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix], 1u);
-      }
-      __syncthreads();
-      if (tid < kRadix) {
-        cnt = s_thist[tid];
-        st_relaxed(&lookback[tile * kRadix + tid],
-                   (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
-      }
-      tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
+    for (int i = 0; i < ITEMS; ++i) {
+      const bool valid = full || (wofs + i * 32 < tile_n);
+      atomicAdd(&wh[valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix], 1u);
     }
-    // ---- rank: per-warp digit counters; the highest peer lane adds the group's count.
-    // Three unrolled phases so the match.any latencies and the leaders' shared atomics of all
-    // ITEMS items are in flight together (same-digit atomics still serialise in hardware order).
+    __syncthreads();
+    uint64_t cnt = 0;
+    if (tid < kRadix) {
+#pragma unroll
+      for (int w = 0; w < WARPS; ++w) cnt += whist[w * (kRadix + 1) + tid];
+      st_relaxed(&lookback[tile * kRadix + tid],
+                 (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+    }
+    const uint32_t tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
+    if (tid < kRadix) {
+      uint32_t run = tstart;
+#pragma unroll
+      for (int w = 0; w < WARPS; ++w) {
+        const uint32_t c = whist[w * (kRadix + 1) + tid];
+        whist[w * (kRadix + 1) + tid] = run;
+        run += c;
+      }
+    }
+    __syncthreads();
+    HSORT_PHASE(2);
+
+    // ---- rank: the highest peer lane's atomic on the warp's base returns the group's first
+    // slot, so r[i] is the key's final position in the digit-ordered tile.  Three unrolled phases
+    // keep the peer computations and the leaders' atomics of all items in flight together.
     uint32_t r[ITEMS];
     constexpr int RC = (MINB >= 3 && ITEMS % 2 == 0) ? ITEMS / 2 : ITEMS;  // ranking chunk
 #pragma unroll
@@ -655,50 +661,12 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
         r[c0 + i] = __shfl_sync(0xffffffffu, r[c0 + i], leader) + __popc(peers[i] & lt);
       }
     }
-    __syncthreads();
-    HSORT_PHASE(2);
-
-    // ---- per digit: warp-exclusive offsets, tile count, aggregate publish, tile-local starts
-    if (EARLY) {
-      if (tid < kRadix) {
-        uint32_t run = tstart;
-#pragma unroll
-        for (int w = 0; w < WARPS; ++w) {
-          const uint32_t c = whist[w * (kRadix + 1) + tid];
-          whist[w * (kRadix + 1) + tid] = run;
-          run += c;
-        }
-      }
-    } else {
-      if (tid < kRadix) {
-        uint32_t run = 0;
-#pragma unroll
-        for (int w = 0; w < WARPS; ++w) {
-          const uint32_t c = whist[w * (kRadix + 1) + tid];
-          whist[w * (kRadix + 1) + tid] = run;
-          run += c;
-        }
-        cnt = run;
-        st_relaxed(&lookback[tile * kRadix + tid],
-                   (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
-      }
-      tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
-      if (tid < kRadix) {
-#pragma unroll
-        for (int w = 0; w < WARPS; ++w) whist[w * (kRadix + 1) + tid] += tstart;
-      }
-    }
-    __syncthreads();
     HSORT_PHASE(3);
 
     // ---- scatter into the (already consumed) stage buffer in digit order
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-      if (full || wofs + i * 32 < tile_n) {
-        const uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
-        sb[wh[d] + r[i]] = k[i];
-      }
-    }
+    for (int i = 0; i < ITEMS; ++i)
+      if (full || wofs + i * 32 < tile_n) sb[r[i]] = k[i];
     // ---- decoupled look-back (thread = digit), LBW predecessors read per round trip
     if (tid < kRadix) {
       uint64_t excl = 0;
@@ -956,8 +924,8 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const bool aligned = !(((uintptr_t)in | (uintptr_t)out | (uintptr_t)(tmp ? tmp : out)) & 15);
   const int v = aligned ? pass_variant() : 0;
-  // window 4 + early aggregates (LBW bit 16); measured best of windows 1..32 with/without
-  if (v == 1) return launch_tma_pass<256, 16, 4 + (1 << 16), 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+  // look-back window 4: measured best of 1..32
+  if (v == 1) return launch_tma_pass<256, 16, 4, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
   uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
   if (first_in_f64)
     k_onesweep<kPassThreads, kPassItems, true><<<(unsigned)tiles, kPassThreads, 0, st>>>(

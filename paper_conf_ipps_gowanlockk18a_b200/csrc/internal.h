@@ -20,6 +20,7 @@ struct RadixPlan {
   int32_t copy_out_f64; // conversion of the final copy: destination is float64 bits
   int32_t match_mask;   // bit p: pass p ranks with MATCH.ANY (few distinct digits per warp),
                         // else with the 8-ballot multisplit
+  int32_t lb_parity;    // 32-bit look-back mode: status array of pass p is (lb_parity + p) & 1
 };
 
 struct RadixScratch {
@@ -35,6 +36,9 @@ struct RadixScratch {
   uint64_t* lookback = nullptr;
   uint64_t max_tiles = 0;
   uint32_t epoch = 0;
+  uint32_t* lb_state = nullptr;  // device word: running count of 32-bit-mode passes (parity)
+  int lb_mode = 0;               // 0 unused/zeroed, 1 64-bit epoch words, 2 32-bit words
+  uint64_t lb_rows = 0;          // 32-bit mode: rows possibly used since the last full clear
   int device = -1;
   // host-pinned mirror of the plan, read back for statistics
   RadixPlan* h_plan = nullptr;

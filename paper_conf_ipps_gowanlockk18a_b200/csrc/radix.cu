@@ -60,6 +60,14 @@ __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
 __device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ uint32_t ld_relaxed32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed32(uint32_t* p, uint32_t v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -164,7 +172,8 @@ __device__ __forceinline__ uint64_t scan256_excl(uint64_t v, uint64_t* s_warp /*
 __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ hist,
                                                    uint64_t* __restrict__ bin_base,
                                                    RadixPlan* __restrict__ plan, uint64_t n,
-                                                   int in_eq_out, int in_f64, int out_f64) {
+                                                   int in_eq_out, int in_f64, int out_f64,
+                                                   uint32_t* __restrict__ lb_state) {
   __shared__ uint64_t s_warp[8];
   __shared__ int s_nz[kDigits];
   __shared__ float s_dist[kDigits][8];
@@ -195,6 +204,8 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
     P.copy_src = -1;
     P.copy_in_f64 = 0;
     P.copy_out_f64 = 0;
+    P.lb_parity = lb_state ? (int32_t)(*lb_state & 1u) : 0;
+    if (lb_state) *lb_state += (uint32_t)na;
     P.match_mask = 0;
     for (int q = 0; q < na; ++q) {
       float dsum = 0;
@@ -235,8 +246,10 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
 }
 
 // Single-pass plan (tests / hsort_device_radix_pass): in -> out by `digit`.
-__global__ void k_force_plan(RadixPlan* plan, int digit) {
+__global__ void k_force_plan(RadixPlan* plan, int digit, uint32_t* lb_state) {
   RadixPlan P;
+  P.lb_parity = (int32_t)(*lb_state & 1u);
+  *lb_state += 1u;
   P.num_active = 1;
   for (int p = 0; p < kDigits; ++p) { P.digit[p] = -1; P.src[p] = -1; P.dst[p] = -1; }
   P.digit[0] = digit;
@@ -461,6 +474,34 @@ __device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__
   }
 }
 
+// 32-bit status words (n <= 2^30): [31:30] flag (1 aggregate, 2 inclusive prefix), [29:0] count.
+// Two arrays alternate between passes and each pass zeroes the rows of the other one, so no
+// epoch tag is needed; half the L2 traffic of the 64-bit words.
+template <int W>
+__device__ __forceinline__ uint32_t lookback_window32(const uint32_t* __restrict__ lb, int64_t j,
+                                                      int d) {
+  uint32_t excl = 0;
+  while (true) {
+    uint32_t w[W];
+#pragma unroll
+    for (int q = 0; q < W; ++q)
+      w[q] = (j - q >= 0) ? ld_relaxed32(&lb[(uint64_t)(j - q) * kRadix + d]) : (2u << 30);
+    int q = 0;
+    bool done = false;
+#pragma unroll
+    for (int u = 0; u < W; ++u) {
+      if (done || q != u) continue;
+      const uint32_t flag = w[u] >> 30;
+      if (flag == 0) continue;  // not yet published: re-read
+      excl += w[u] & 0x3FFFFFFFu;
+      if (flag == 2) done = true;
+      else ++q;
+    }
+    if (done) return excl;
+    j -= q;
+  }
+}
+
 #ifdef HSORT_PHASE_TIMING
 #define HSORT_PHASE(i)                         \
   if (tid == 0) {                              \
@@ -485,14 +526,15 @@ struct TmaPassSmem {
   static constexpr size_t bytes = tile_off + 16;
 };
 
-template <int THREADS, int ITEMS, bool IN_F64, int LBW, int MINB>
+template <int THREADS, int ITEMS, bool IN_F64, int LBW, int MINB, bool S32>
 __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, uint64_t* out, uint64_t* tmp,
                                                            uint64_t n,
                                                            const RadixPlan* __restrict__ plan,
                                                            const uint64_t* __restrict__ bin_base,
                                                            uint64_t* __restrict__ lookback,
                                                            uint32_t* __restrict__ tile_ctr,
-                                                           uint32_t epoch, int p, int out_f64) {
+                                                           uint32_t epoch, int p, int out_f64,
+                                                           uint64_t lb_half, uint64_t lb_rows) {
   using L = TmaPassSmem<THREADS, ITEMS>;
   constexpr int WARPS = L::WARPS;
   constexpr int TILE = L::TILE;
@@ -513,6 +555,8 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
   uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
   const bool use_match = (plan->match_mask >> p) & 1;
   const bool inv = out_f64 && (p == na - 1);
+  uint32_t* lb32 = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p) & 1) * lb_half;
+  uint32_t* lb32_next = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p + 1) & 1) * lb_half;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t num_tiles = (n + TILE - 1) / TILE;
   const uint32_t ep = epoch & kEpochMask;
@@ -595,8 +639,13 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
     if (tid < kRadix) {
 #pragma unroll
       for (int w = 0; w < WARPS; ++w) cnt += whist[w * (kRadix + 1) + tid];
-      st_relaxed(&lookback[tile * kRadix + tid],
-                 (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+      if (S32) {
+        st_relaxed32(&lb32[tile * kRadix + tid], ((tile == 0 ? 2u : 1u) << 30) | (uint32_t)cnt);
+        lb32_next[tile * kRadix + tid] = 0;  // the next pass's array, row of this tile
+      } else {
+        st_relaxed(&lookback[tile * kRadix + tid],
+                   (tile == 0 ? kFlagP : kFlagA) | ((uint64_t)ep << 40) | cnt);
+      }
     }
     const uint32_t tstart = (uint32_t)scan256_excl(cnt, s_warp, nullptr);
     if (tid < kRadix) {
@@ -671,8 +720,13 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
     if (tid < kRadix) {
       uint64_t excl = 0;
       if (tile > 0) {
-        excl = lookback_window<(LBW & 255), ((LBW >> 8) & 255)>(lookback, (int64_t)tile - 1, tid, ep);
-        st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
+        if (S32) {
+          excl = lookback_window32<(LBW & 255)>(lb32, (int64_t)tile - 1, tid);
+          st_relaxed32(&lb32[tile * kRadix + tid], (2u << 30) | (uint32_t)(excl + cnt));
+        } else {
+          excl = lookback_window<(LBW & 255), ((LBW >> 8) & 255)>(lookback, (int64_t)tile - 1, tid, ep);
+          st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
+        }
       }
       s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)tstart;
     }
@@ -717,6 +771,10 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
 #endif
     cb ^= 1;
   }
+  // 32-bit mode: rows beyond this sort's tiles that an earlier, larger sort may have used
+  if (S32)
+    for (uint64_t r = num_tiles + blockIdx.x; r < lb_rows; r += gridDim.x)
+      lb32_next[r * kRadix + tid] = 0;
 #ifdef HSORT_PHASE_TIMING
   if (tid == 0) {
     for (int i = 0; i < 10; ++i) atomicAdd(&g_phase_dbg[p * 16 + (i < 8 ? i : i + 1)], ph_acc[i]);
@@ -884,7 +942,7 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
   return cudaGetLastError();
 }
 
-template <int THREADS, int ITEMS, int LBW = 8, int MINB = ((THREADS * ITEMS <= 2048) ? 4 : ((THREADS * ITEMS <= 4096) ? 2 : 1))>
+template <int THREADS, int ITEMS, int LBW, int MINB, bool S32>
 cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
                             RadixScratch& s, uint32_t ep, int p, bool first_in_f64, bool out_f64,
                             cudaStream_t st) {
@@ -892,8 +950,8 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
   static int blocks_per_sm[64] = {0};
   int dev = 0;
   cudaGetDevice(&dev);
-  auto kt = k_onesweep_tma<THREADS, ITEMS, true, LBW, MINB>;
-  auto kf = k_onesweep_tma<THREADS, ITEMS, false, LBW, MINB>;
+  auto kt = k_onesweep_tma<THREADS, ITEMS, true, LBW, MINB, S32>;
+  auto kf = k_onesweep_tma<THREADS, ITEMS, false, LBW, MINB, S32>;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   if (!blocks_per_sm[dev]) {
     cudaError_t e;
@@ -909,11 +967,40 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
   if (grid > tiles) grid = tiles ? tiles : 1;
   if (first_in_f64)
     kt<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
-                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
+                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0,
+                                                 s.max_tiles * kRadix, s.lb_rows);
   else
     kf<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
-                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0);
+                                                 s.tile_ctr, ep, p, out_f64 ? 1 : 0,
+                                                 s.max_tiles * kRadix, s.lb_rows);
   return cudaGetLastError();
+}
+
+// Look-back status format of one sort: 2 = 32-bit words (TMA pass, n <= 2^30: an active digit
+// has at most n - 1 keys), 1 = 64-bit epoch-tagged words.  Switching formats re-zeroes the array
+// so stale words of the other format can never be read as published.
+int pass_kernel(uint64_t* in, uint64_t* out, uint64_t* tmp) {
+  const bool aligned = !(((uintptr_t)in | (uintptr_t)out | (uintptr_t)(tmp ? tmp : out)) & 15);
+  return aligned ? pass_variant() : 0;
+}
+// 32-bit status words hold flag(2) | count(30).  With n <= 2^30 every prefix a tile actually
+// consumes is < 2^30: a reader that owns keys of digit d reads predecessors' prefixes of d, which
+// exclude its own keys.  The one value that can reach 2^30 (all n keys in one digit, a forced
+// single pass) is only read by tiles without keys of d and decodes as flag 3 = "aggregate", so a
+// reader never spins on it.
+cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t st) {
+  const int mode = (kernel == 1 && n <= (1ull << 30)) ? 2 : 1;
+  if (s.lb_mode != 0 && s.lb_mode != mode) {
+    cudaError_t e = cudaMemsetAsync(s.lookback, 0, s.max_tiles * kRadix * sizeof(uint64_t), st);
+    if (e != cudaSuccess) return e;
+    s.lb_rows = 0;
+  }
+  s.lb_mode = mode;
+  if (mode == 2) {
+    const uint64_t t = (n + kRadixTile - 1) / kRadixTile;
+    if (t > s.lb_rows) s.lb_rows = t;
+  }
+  return cudaSuccess;
 }
 
 cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
@@ -922,10 +1009,13 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   cudaError_t e = next_epoch(s, st, &ep);
   if (e != cudaSuccess) return e;
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
-  const bool aligned = !(((uintptr_t)in | (uintptr_t)out | (uintptr_t)(tmp ? tmp : out)) & 15);
-  const int v = aligned ? pass_variant() : 0;
+  const int v = pass_kernel(in, out, tmp);
   // look-back window 4: measured best of 1..32
-  if (v == 1) return launch_tma_pass<256, 16, 4, 2>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+  if (v == 1) {
+    if (s.lb_mode == 2)
+      return launch_tma_pass<256, 16, 4, 2, true>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+    return launch_tma_pass<256, 16, 4, 2, false>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
+  }
   uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
   if (first_in_f64)
     k_onesweep<kPassThreads, kPassItems, true><<<(unsigned)tiles, kPassThreads, 0, st>>>(
@@ -961,13 +1051,14 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
     // layout (256-byte aligned pieces): hist | plan | tile counters | bin_base
     const size_t hist_b = kDigits * kRadix * sizeof(uint64_t);
     const size_t plan_b = (sizeof(RadixPlan) + 255) & ~(size_t)255;
-    const size_t bytes = hist_b + plan_b + 256 + hist_b;
+    const size_t bytes = hist_b + plan_b + 256 + hist_b + 256;
     if ((e = cudaMalloc(&s.small, bytes)) != cudaSuccess) return e;
     char* b = (char*)s.small;
     s.hist = (uint64_t*)b;
     s.plan = (RadixPlan*)(b + hist_b);
     s.tile_ctr = (uint32_t*)(b + hist_b + plan_b);
     s.bin_base = (uint64_t*)(b + hist_b + plan_b + 256);
+    s.lb_state = (uint32_t*)(b + hist_b + plan_b + 256 + hist_b);  // not zeroed per sort
     s.small_zero_bytes = (char*)s.bin_base - b;
     if ((e = cudaMemset(s.small, 0, bytes)) != cudaSuccess) return e;
     if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)
@@ -984,6 +1075,8 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
     if ((e = cudaMemset(s.lookback, 0, t2 * kRadix * sizeof(uint64_t))) != cudaSuccess) return e;
     s.max_tiles = t2;
     s.epoch = 0;
+    s.lb_mode = 0;  // freshly zeroed
+    s.lb_rows = 0;
   }
   return cudaSuccess;
 }
@@ -1034,8 +1127,9 @@ cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uin
   if ((e = mark(0)) != cudaSuccess) return e;
   if ((e = launch_hist(s, in, n, in_f64, s.hist, st)) != cudaSuccess) return e;
   if ((e = mark(1)) != cudaSuccess) return e;
+  if ((e = select_lb_mode(s, pass_kernel(in, out, tmp), n, st)) != cudaSuccess) return e;
   k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
-                                 out_f64 ? 1 : 0);
+                                 out_f64 ? 1 : 0, s.lb_state);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   if ((e = mark(2)) != cudaSuccess) return e;
   for (int p = 0; p < kDigits; ++p) {
@@ -1066,8 +1160,9 @@ cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, 
   uint64_t* in = const_cast<uint64_t*>(src);
   if ((e = cudaMemsetAsync(s.small, 0, s.small_zero_bytes, st)) != cudaSuccess) return e;
   if ((e = launch_hist(s, in, n, false, s.hist, st)) != cudaSuccess) return e;
-  k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, 0, 0, 0);
-  k_force_plan<<<1, 1, 0, st>>>(s.plan, digit);
+  if ((e = select_lb_mode(s, pass_kernel(in, dst, nullptr), n, st)) != cudaSuccess) return e;
+  k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, 0, 0, 0, nullptr);
+  k_force_plan<<<1, 1, 0, st>>>(s.plan, digit, s.lb_state);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   return launch_pass(s, in, dst, nullptr, n, 0, false, false, st);
 }

@@ -149,3 +149,42 @@ def test_full_size_c2_device_sort(hs_gpu, inputs_mod):
     part = np.partition(A, idx)
     got = d_out[torch.from_numpy(idx).cuda()].cpu().numpy()
     assert np.array_equal(_bits(got), _bits(part[idx]))
+
+
+def test_lookback_state_reuse_across_sizes(hs_gpu, oracle_mod, inputs_mod):
+    """The look-back status arrays persist across calls (32-bit mode alternates two arrays and
+    clears the idle one inside each pass): a large sort, then small ones, then a
+    larger one, with single passes interleaved, must all stay bit-exact."""
+    import torch
+    sizes = [(1 << 22) + 3, 5000, (1 << 20) + 7, 1, 300_001, (1 << 22) + 4096 * 3 + 1, 4097]
+    for i, n in enumerate(sizes):
+        A = inputs_mod.generate("random_bits" if i % 2 else "uniform", n, seed=100 + i)
+        d_in = _to_dev(A)
+        d_out = torch.empty_like(d_in)
+        hs_gpu.hsort_sort_device(d_in, d_out)
+        torch.cuda.synchronize()
+        assert np.array_equal(_bits(d_out.cpu().numpy()), _bits(oracle_mod.sort_f64(A))), n
+        if i % 3 == 1:  # a lone pass between sorts (radix_one_pass path)
+            K = np.random.default_rng(i).integers(0, 2**64, size=2 * n + 11, dtype=np.uint64)
+            src = _to_dev(K)
+            dst = torch.empty_like(src)
+            hs_gpu.hsort_device_radix_pass(src, dst, i % 8)
+            torch.cuda.synchronize()
+            assert np.array_equal(dst.cpu().numpy(), oracle_mod.counting_sort_pass(K, i % 8))
+
+
+def test_device_sort_above_2p30_switches_lookback_mode(hs_gpu, inputs_mod):
+    """n > 2^30 uses 64-bit look-back words (counts above 2^30 do not fit the 32-bit word);
+    alternating with small sorts exercises the mode switch both ways.  Uniform keys: torch.sort
+    is an exact independent reference (see test_full_size_c2_device_sort)."""
+    import torch
+    for n in (70_001, (1 << 30) + 4097, 70_001):
+        A = inputs_mod.generate("uniform", n, seed=n)
+        d_in = torch.from_numpy(A).cuda()
+        d_out = torch.empty_like(d_in)
+        hs_gpu.hsort_sort_device(d_in, d_out)
+        torch.cuda.synchronize()
+        ref = torch.sort(d_in).values
+        assert torch.equal(d_out.view(torch.int64), ref.view(torch.int64)), n
+        del ref, d_in, d_out
+        torch.cuda.empty_cache()

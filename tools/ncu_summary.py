@@ -56,8 +56,18 @@ ap.add_argument("reports", nargs="*")
 ap.add_argument("--n", type=int, required=True)
 ap.add_argument("--out-md", required=True)
 ap.add_argument("--out-json", default=None)
+ap.add_argument("--steps", type=int, default=0,
+                help="keep only the first S device-sort steps (launches up to the S-th k_final_copy)")
 a = ap.parse_args()
 rows = launches(a.csv)
+if a.steps:
+    seen, keep = 0, []
+    for r in rows:
+        keep.append(r)
+        seen += r[0].startswith("k_final_copy")
+        if seen == a.steps:
+            break
+    rows = keep
 agg = OrderedDict()
 for k, ns, g, b in rows:
     e = agg.setdefault(k, [0, 0.0, g, b])
@@ -65,7 +75,8 @@ for k, ns, g, b in rows:
     e[1] += ns
 tot = sum(e[1] for e in agg.values())
 md = ["# ncu launch list summary", "", f"source: `{a.csv}` (gpu__time_duration.sum, --clock-control none; "
-      "cold-cache, serialised launches: compare shares, not absolutes)", "",
+      "cold-cache, serialised launches: compare shares, not absolutes)"
+      + (f"; first {a.steps} device-sort steps of the bench command (warm-up + timed)" if a.steps else ""), "",
       "| kernel | launches | total ms | mean ms | share | grid | block |", "|---|---|---|---|---|---|---|"]
 for k, (c, ns, g, b) in sorted(agg.items(), key=lambda x: -x[1][1]):
     md.append(f"| `{k}` | {c} | {ns/1e6:.3f} | {ns/1e6/c:.3f} | {ns/tot:.1%} | {g} | {b} |")

@@ -27,8 +27,8 @@ L.hsort_debug_phase_counters(buf, 256, 1)
 hs.hsort_sort_device(d_in, d_out)
 torch.cuda.synchronize()
 L.hsort_debug_phase_counters(buf, 256, 1)
-names = {0: "wait+claim", 1: "keys+earlycount", 6: "publish+scan", 7: "match", 9: "atomics",
-         2: "shfl+sync", 3: "offsets", 4: "scatter+lookback", 5: "writeout"}
+names = {0: "wait+claim", 2: "keys+earlycount+scan+bases", 3: "rank", 4: "scatter+lookback",
+         5: "writeout"}
 res = {}
 for p in range(8):
     tiles = buf[p * 16 + 8]

@@ -84,6 +84,10 @@ typedef struct hsort_stats {
   uint64_t bytes_h2d;      /* bytes moved host -> device */
   uint64_t bytes_d2h;      /* bytes moved device -> host */
   double t_host_alloc;     /* pinned working-memory (W) allocation in this call (cached after) */
+  uint64_t pipe_merges;    /* STREAM PIPEMERGE: pair-wise merges done during the sort phase */
+  double t_pipemerge;      /* host: time spent in those pair-wise merges */
+  double t_pipemerge_wait; /* host: wait after the sort phase for the last pair merge (P:422-425
+                              wants 0: pair merges must not delay the final multiway merge) */
 } hsort_stats;
 
 /* Planner output (A1).  Pure host arithmetic; see hsort_plan(). */
@@ -137,6 +141,11 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
  *         MCpy), "merge_threads" (CPU merge threads), "resident" (-1 auto, 0 force
  *         STREAM, 1 force RESIDENT), "merge_gpu_permille" (A12 share f in 1/1000; -1 auto),
  *         "pipeline" (1 = overlapped streams PIPEDATA, 0 = blocking BLINEMULTI ablation),
+ *         "pipemerge" (STREAM mode with pipeline = 1: 1 = PIPEMERGE pair-wise merges of sorted
+ *         batches on the host threads while the GPUs sort, hsort_pipemerge_count(n_b, n_gpus)
+ *         of them; 0 = off (default: slower on a B200 box), the final
+ *         merge takes all n_b runs), "pipemerge_threads"
+ *         (host threads for those pair merges, on their own pool; 0 = half the hardware threads),
  *         "merge_chunk" (GPU merge output chunk elements), "device_reserve_mb" (HBM left free),
  *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times),
  *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never),
@@ -226,7 +235,8 @@ int hsort_host_upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* va
                             uint64_t* out);
 
 /* The PIPEMERGE heuristic (reading A-9): number of pair-wise merges overlapped with
- * GPU sorting.  Pure arithmetic. */
+ * GPU sorting; STREAM mode merges pairs (0,1), (2,3), ... of that many (option "pipemerge").
+ * Pure arithmetic. */
 uint64_t hsort_pipemerge_count(uint64_t n_b, int n_gpus);
 
 /* Number of GPUs visible to the library (0 when none; never an error). */

@@ -56,6 +56,7 @@ class hsort_stats(ctypes.Structure):
         ("t_merge_cpu", ctypes.c_double), ("t_merge_gpu", ctypes.c_double),
         ("t_init", ctypes.c_double),
         ("bytes_h2d", _U64), ("bytes_d2h", _U64), ("t_host_alloc", ctypes.c_double),
+        ("pipe_merges", _U64), ("t_pipemerge", ctypes.c_double), ("t_pipemerge_wait", ctypes.c_double),
     ]
 
 

@@ -41,6 +41,11 @@ void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out,
                 int threads);
 void host_merge_range(const uint64_t* keys, const uint64_t* off, int k, uint64_t o_lo,
                       uint64_t o_hi, uint64_t* out, bool out_f64, int threads);
+void host_corank_runs(const uint64_t* const* run, const uint64_t* len, int k, uint64_t o,
+                      uint64_t* ranks);
+void host_merge_runs_range(const uint64_t* const* run, const uint64_t* len, int k, uint64_t o_lo,
+                           uint64_t o_hi, uint64_t* out, bool out_f64, int threads,
+                           ThreadPool* pool);
 }  // namespace hsort
 
 using namespace hsort;
@@ -104,6 +109,8 @@ struct Options {
       {"resident", -1},              // -1 auto, 0 force STREAM, 1 force RESIDENT
       {"merge_gpu_permille", -1},    // A12 share f (per mille) of merge output on GPUs; -1 auto
       {"pipeline", 1},               // 1 PIPEDATA overlap, 0 blocking BLINEMULTI ablation
+      {"pipemerge", 0},              // STREAM: 1 = pair-wise merges during the sort phase (PIPEMERGE)
+      {"pipemerge_threads", 0},      // threads for those merges (0 = half the hardware threads)
       {"merge_chunk", 1ll << 26},    // GPU merge output chunk (keys)
       {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
@@ -530,10 +537,11 @@ void sort_resident(GpuCtx& g, CallCtx& c) {
 // host memory W, in chunks of `merge_chunk` keys: exact co-ranks on the host, HtoD of the k
 // slices (direct from pinned W), K4/K5 on the GPU, DtoH into B.  Two slots: the HtoD of chunk c+1
 // overlaps the merge and DtoH of chunk c.
-void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const uint64_t* W, const std::vector<uint64_t>& off,
-                         uint64_t o_lo, uint64_t o_hi, bool w_direct, double* t_gpu) {
+void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t*>& run,
+                         const std::vector<uint64_t>& rlen, uint64_t o_lo, uint64_t o_hi,
+                         bool w_direct, double* t_gpu) {
   CK(cudaSetDevice(g.dev));
-  const int k = (int)off.size() - 1;
+  const int k = (int)run.size();
   const uint64_t C = std::max<uint64_t>(
       kMergeTile, ((uint64_t)S().opt.get("merge_chunk") / kMergeTile) * kMergeTile);
   const uint64_t nch = (o_hi - o_lo + C - 1) / C;
@@ -545,7 +553,7 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const uint64_t* W, const std::ve
   std::vector<uint64_t> cr((nch + 1) * (size_t)k);
   host_pool().parallel_for((int64_t)nch + 1, host_threads(), [&](int64_t i) {
     const uint64_t p = std::min(o_lo + (uint64_t)i * C, o_hi);
-    host_corank(W, off.data(), k, p, &cr[(size_t)i * k]);
+    host_corank_runs(run.data(), rlen.data(), k, p, &cr[(size_t)i * k]);
   });
   cudaEvent_t in_ready[2], in_free[2], merged[2], out_free[2];
   for (int s = 0; s < 2; ++s) {
@@ -572,7 +580,7 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const uint64_t* W, const std::ve
     for (int j = 0; j < k; ++j) {
       const uint64_t len = r1[j] - r0[j];
       ho[j + 1] = ho[j] + len;
-      if (len) upload(g, din + ho[j], W + off[j] + r0[j], len * 8, g.s_h2d, w_direct, c.mc_threads, acc);
+      if (len) upload(g, din + ho[j], run[j] + r0[j], len * 8, g.s_h2d, w_direct, c.mc_threads, acc);
     }
     uint64_t* doff = g.off.u64() + (size_t)s * (k + 1);
     CK(cudaMemcpyAsync(doff, ho, (k + 1) * 8, cudaMemcpyHostToDevice, g.s_h2d));
@@ -613,25 +621,36 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   const uint64_t n = c.n, b_s = c.plan.b_s, n_b = c.plan.n_b;
   const int n_s = std::max(1, c.plan.n_s);
   const bool pipelined = S().opt.get("pipeline") != 0;
+  // PIPEMERGE: m pair-wise merges of sorted batches (2j, 2j+1), j < m, run on the
+  // host threads while the GPUs are still sorting; m = hsort_pipemerge_count (reading A-9), so the
+  // last pair (n_b even) or the last batch (n_b odd) is never pre-merged, only full b_s batches
+  // are paired, and merged outputs are never merged again.
+  const uint64_t m_pipe = (pipelined && S().opt.get("pipemerge") != 0 && n_b >= 3)
+                              ? hsort_pipemerge_count(n_b, (int)gs.size()) : 0;
   // W: working memory for the sorted sublists; transformed uint64 keys.
   // Pinned and cached across calls when possible (runs then DMA straight into W and the GPU merge
-  // share streams straight out of it); pageable mmap otherwise.
+  // share streams straight out of it); pageable mmap otherwise.  With PIPEMERGE, W has a 2 b_s
+  // spare region in front: batch i lands at Wb + i b_s (Wb = W + 2 b_s) and pair merge j writes
+  // W[2j b_s, (2j+2) b_s) — the spare for j = 0, else the inputs of pair j-1, already consumed
+  // because the pair merges run one after another.
+  const uint64_t spare = m_pipe ? 2 * b_s : 0;
+  const uint64_t wn = n + spare;
   uint64_t* W = nullptr;
   bool w_direct = false;
   void* w_map = nullptr;
   const int64_t pin_w = S().opt.get("pin_w");
   const bool want_pin = pin_w == 1 ||
-      (pin_w == -1 && (n * 8 <= ((uint64_t)S().opt.get("pin_w_max_mb") << 20) || S().w_pin_bytes >= n * 8));
+      (pin_w == -1 && (wn * 8 <= ((uint64_t)S().opt.get("pin_w_max_mb") << 20) || S().w_pin_bytes >= wn * 8));
   if (want_pin) {
-    if (S().w_pin_bytes < n * 8) {
+    if (S().w_pin_bytes < wn * 8) {
       if (S().w_pin) cudaFreeHost(S().w_pin);
       S().w_pin = nullptr;
       S().w_pin_bytes = 0;
       auto ta = Clock::now();
       void* p = nullptr;
-      if (cudaHostAlloc(&p, n * 8, cudaHostAllocDefault) == cudaSuccess) {
+      if (cudaHostAlloc(&p, wn * 8, cudaHostAllocDefault) == cudaSuccess) {
         S().w_pin = p;
-        S().w_pin_bytes = n * 8;
+        S().w_pin_bytes = wn * 8;
       } else {
         cudaGetLastError();
       }
@@ -643,9 +662,9 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
     }
   }
   if (!W) {
-    void* p = mmap(nullptr, n * 8, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+    void* p = mmap(nullptr, wn * 8, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
     if (p == MAP_FAILED) throw HsortError(HSORT_ERR_HOST_OOM, "mmap W failed");
-    madvise(p, n * 8, MADV_HUGEPAGE);
+    madvise(p, wn * 8, MADV_HUGEPAGE);
     W = (uint64_t*)p;
     w_map = p;
   }
@@ -655,20 +674,36 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
     ~WFree() {
       if (p) munmap(p, b);
     }
-  } wfree{w_map, n * 8};
+  } wfree{w_map, wn * 8};
+  uint64_t* const Wb = W + spare;
 
   std::atomic<uint64_t> next_batch{0};
   std::mutex err_m;
   std::string err_msg;
   int err_code = 0;
   std::atomic<bool> failed{false};
+  std::mutex pm_m;  // PIPEMERGE: which batches have landed in W
+  std::condition_variable pm_cv;
+  std::vector<uint8_t> landed(m_pipe ? n_b : 0, 0);
   auto fail = [&](int code, const std::string& m) {
-    std::lock_guard<std::mutex> gd(err_m);
-    if (!err_code) {
-      err_code = code;
-      err_msg = m;
+    {
+      std::lock_guard<std::mutex> gd(err_m);
+      if (!err_code) {
+        err_code = code;
+        err_msg = m;
+      }
+      failed = true;
     }
-    failed = true;
+    { std::lock_guard<std::mutex> gd(pm_m); }
+    pm_cv.notify_all();
+  };
+  auto mark_landed = [&](uint64_t i) {
+    if (!m_pipe) return;
+    {
+      std::lock_guard<std::mutex> gd(pm_m);
+      landed[i] = 1;
+    }
+    pm_cv.notify_all();
   };
   struct PerGpu {
     Acc up, down;
@@ -719,7 +754,7 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
           CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), len, c.f64, false, g.s_comp));
           CK(cudaEventRecord(it->es.b, g.s_comp));
           CK(cudaEventRecord(it->ed.a, g.s_comp));
-          download(g, W + o, g.runs.p, len * 8, g.s_comp, w_direct, c.mc_threads, P.down);
+          download(g, Wb + o, g.runs.p, len * 8, g.s_comp, w_direct, c.mc_threads, P.down);
           CK(cudaEventRecord(it->ed.b, g.s_comp));
           CK(cudaStreamSynchronize(g.s_comp));
           P.passes += g.rs.h_plan->num_active;
@@ -740,10 +775,11 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
               uint64_t o = it->batch * b_s, len = std::min(b_s, n - o);
               CK(cudaStreamWaitEvent(g.s_d2h, ev_sorted[it->slot], 0));
               CK(cudaEventRecord(it->ed.a, g.s_d2h));
-              download(g, W + o, g.runs.u64() + (uint64_t)it->slot * b_s, len * 8, g.s_d2h, w_direct,
+              download(g, Wb + o, g.runs.u64() + (uint64_t)it->slot * b_s, len * 8, g.s_d2h, w_direct,
                        c.mc_threads, P.down);
               CK(cudaEventRecord(it->ed.b, g.s_d2h));
               CK(cudaEventSynchronize(it->ed.b));
+              mark_landed(it->batch);
               {
                 std::lock_guard<std::mutex> gd(m);
                 slot_busy[it->slot] = 0;
@@ -818,6 +854,36 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
       fail(e.code, e.what());
     }
   };
+  // PIPEMERGE worker: pair j as soon as batches 2j and 2j+1 are in W, one pair at a time, each
+  // merge spread over the merge threads by exact co-ranks (the output stays in key form).
+  double t_pipe = 0;
+  uint64_t pipe_done = 0;
+  const int pm_threads = (int)std::max<int64_t>(
+      1, std::min<int64_t>(S().opt.get("pipemerge_threads") > 0 ? S().opt.get("pipemerge_threads")
+                                                                : host_threads() / 2,
+                           pipe_pool().size() + 1));
+  std::thread merger;
+  if (m_pipe) {
+    merger = std::thread([&] {
+      try {
+        for (uint64_t j = 0; j < m_pipe; ++j) {
+          {
+            std::unique_lock<std::mutex> lk(pm_m);
+            pm_cv.wait(lk, [&] { return failed.load() || (landed[2 * j] && landed[2 * j + 1]); });
+            if (failed) return;
+          }
+          auto tm = Clock::now();
+          const uint64_t* rp[2] = {Wb + 2 * j * b_s, Wb + (2 * j + 1) * b_s};
+          const uint64_t rl[2] = {b_s, b_s};
+          host_merge_runs_range(rp, rl, 2, 0, 2 * b_s, W + 2 * j * b_s, false, pm_threads, &pipe_pool());
+          t_pipe += secs_since(tm);
+          ++pipe_done;
+        }
+      } catch (const std::exception& e) {
+        fail(HSORT_ERR_INTERNAL, e.what());
+      }
+    });
+  }
   if (gs.size() == 1) {
     gpu_main(0);
   } else {
@@ -825,8 +891,12 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
     for (size_t gi = 0; gi < gs.size(); ++gi) th.emplace_back(gpu_main, gi);
     for (auto& t : th) t.join();
   }
-  if (failed) throw HsortError(err_code ? err_code : HSORT_ERR_INTERNAL, err_msg);
   c.st->t_sort_phase = secs_since(t0);
+  if (merger.joinable()) merger.join();
+  if (failed) throw HsortError(err_code ? err_code : HSORT_ERR_INTERNAL, err_msg);
+  c.st->pipe_merges = pipe_done;
+  c.st->t_pipemerge = t_pipe;
+  c.st->t_pipemerge_wait = secs_since(t0) - c.st->t_sort_phase;
   for (auto& P : pg) {
     c.st->t_h2d += P.t_h2d;
     c.st->t_gpu_sort += P.t_sort;
@@ -841,9 +911,19 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   // [o_f, n) with loser trees; f balances the two measured rates (the split cannot be
   // derived asymptotically, it must be measured).
   auto t1 = Clock::now();
-  std::vector<uint64_t> off(n_b + 1);
-  for (uint64_t i = 0; i <= n_b; ++i) off[i] = std::min(i * b_s, n);
-  const int k = (int)n_b;
+  // the sublists of the final merge: m merged pairs, then the batches 2m .. n_b-1
+  std::vector<const uint64_t*> run;
+  std::vector<uint64_t> rlen;
+  for (uint64_t j = 0; j < m_pipe; ++j) {
+    run.push_back(W + 2 * j * b_s);
+    rlen.push_back(2 * b_s);
+  }
+  for (uint64_t i = 2 * m_pipe; i < n_b; ++i) {
+    run.push_back(Wb + i * b_s);
+    rlen.push_back(std::min(b_s, n - i * b_s));
+  }
+  const int k = (int)run.size();
+  c.st->merge_k = k;
   double f = 0.0;
   const int64_t fp = S().opt.get("merge_gpu_permille");
   if (k <= kMaxMergeRuns && !gs.empty()) {
@@ -862,14 +942,15 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   double t_cpu = 0, t_gpu = 0;
   std::thread cpu_part([&] {
     auto tc = Clock::now();
-    host_merge_range(W, off.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64, c.merge_threads);
+    host_merge_runs_range(run.data(), rlen.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64,
+                          c.merge_threads, nullptr);
     t_cpu = secs_since(tc);
   });
   std::string gpu_err;
   int gpu_code = 0;
   if (o_f > 0) {
     try {
-      gpu_merge_from_host(*gs[0], c, W, off, 0, o_f, w_direct, &t_gpu);
+      gpu_merge_from_host(*gs[0], c, run, rlen, 0, o_f, w_direct, &t_gpu);
     } catch (const HsortError& e) {
       gpu_code = e.code;
       gpu_err = e.what();

@@ -132,12 +132,16 @@ inline void st_nt(uint64_t* p, uint64_t v) {
 }  // namespace
 
 // Exact co-ranks of output position o (ties in run order).  Same definition as K4 (merge.cu).
-void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, uint64_t* ranks) {
+// Runs are given as (start pointer, length) pairs, so they may lie anywhere in memory (the
+// PIPEMERGE working memory holds merged pairs and batches at rotating places).
+void host_corank_runs(const uint64_t* const* run, const uint64_t* len, int k, uint64_t o,
+                      uint64_t* ranks) {
   std::vector<uint64_t> lo(k), hi(k);
-  uint64_t total = off[k] - off[0];
+  uint64_t total = 0;
   for (int j = 0; j < k; ++j) {
     lo[j] = 0;
-    hi[j] = off[j + 1] - off[j];
+    hi[j] = len[j];
+    total += len[j];
   }
   if (o >= total) {
     for (int j = 0; j < k; ++j) ranks[j] = hi[j];
@@ -148,7 +152,7 @@ void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, u
     uint64_t mn = ~0ull, mx = 0;
     for (int j = 0; j < k; ++j)
       if (hi[j] > lo[j]) {
-        const uint64_t* r = keys + off[j];
+        const uint64_t* r = run[j];
         mn = std::min(mn, r[lo[j]]);
         mx = std::max(mx, r[hi[j] - 1]);
       }
@@ -158,7 +162,7 @@ void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, u
     uint64_t mid = L + ((H - L) >> 1), s = 0;
     std::vector<uint64_t> u(k);
     for (int j = 0; j < k; ++j) {
-      u[j] = ub(keys + off[j], lo[j], hi[j], mid);
+      u[j] = ub(run[j], lo[j], hi[j], mid);
       s += u[j];
     }
     if (s > o) { H = mid; hi = u; }
@@ -168,7 +172,7 @@ void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, u
   uint64_t lt = 0;
   std::vector<uint64_t> eq(k);
   for (int j = 0; j < k; ++j) {
-    const uint64_t* r = keys + off[j];
+    const uint64_t* r = run[j];
     uint64_t a = lb(r, lo[j], hi[j], v);
     uint64_t z = ub(r, a, hi[j], v);
     lo[j] = a;
@@ -184,14 +188,14 @@ void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, u
 }
 
 // Merge output range [o_a, o_b) given its co-ranks ra (at o_a) and rb (at o_b).
-static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const uint64_t* ra,
+static void merge_range(const uint64_t* const* run, const uint64_t* rlen, int k, const uint64_t* ra,
                         const uint64_t* rb, uint64_t* out, bool out_f64) {
   int live = 0, last = -1;
   for (int j = 0; j < k; ++j)
     if (rb[j] > ra[j]) { ++live; last = j; }
   if (live == 0) return;
   if (live == 1) {
-    const uint64_t* s = keys + off[last] + ra[last];
+    const uint64_t* s = run[last] + ra[last];
     const uint64_t len = rb[last] - ra[last];
     if (out_f64)
       for (uint64_t i = 0; i < len; ++i) st_nt(out + i, from_key(s[i]));
@@ -203,8 +207,8 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
     int a = -1, b = -1;
     for (int j = 0; j < k; ++j)
       if (rb[j] > ra[j]) (a < 0 ? a : b) = j;
-    const uint64_t *p = keys + off[a] + ra[a], *pe = keys + off[a] + rb[a];
-    const uint64_t *q = keys + off[b] + ra[b], *qe = keys + off[b] + rb[b];
+    const uint64_t *p = run[a] + ra[a], *pe = run[a] + rb[a];
+    const uint64_t *q = run[b] + ra[b], *qe = run[b] + rb[b];
     uint64_t* o = out;
     while (p < pe && q < qe) {
       const uint64_t x = *p, y = *q;
@@ -229,7 +233,7 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
   std::vector<uint64_t> cr((NI + 1) * (size_t)k);
   std::memcpy(&cr[0], ra, k * 8);
   std::memcpy(&cr[(size_t)NI * k], rb, k * 8);
-  for (int i = 1; i < NI; ++i) host_corank(keys, off, k, oa + total * i / NI, &cr[(size_t)i * k]);
+  for (int i = 1; i < NI; ++i) host_corank_runs(run, rlen, k, oa + total * i / NI, &cr[(size_t)i * k]);
   LoserTree* lt[NI];
   alignas(64) unsigned char mem[NI][sizeof(LoserTree)];
   uint64_t len[NI], pos[NI];
@@ -237,7 +241,7 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
     lt[i] = new (mem[i]) LoserTree(k);
     len[i] = 0;
     for (int j = 0; j < k; ++j) {
-      lt[i]->set_leaf(j, keys + off[j] + cr[(size_t)i * k + j], keys + off[j] + cr[(size_t)(i + 1) * k + j]);
+      lt[i]->set_leaf(j, run[j] + cr[(size_t)i * k + j], run[j] + cr[(size_t)(i + 1) * k + j]);
       len[i] += cr[(size_t)(i + 1) * k + j] - cr[(size_t)i * k + j];
     }
     pos[i] = i == 0 ? 0 : pos[i - 1] + len[i - 1];
@@ -261,30 +265,54 @@ static void merge_range(const uint64_t* keys, const uint64_t* off, int k, const 
   }
 }
 
-// Merge positions [o_lo, o_hi) of the multiway merge of the k runs keys[off[j] .. off[j+1]) into
+// Merge positions [o_lo, o_hi) of the multiway merge of the k runs run[j][0 .. len[j]) into
 // out[0 .. o_hi - o_lo).  The range is cut into ~4 pieces per thread by exact co-ranks.
-void host_merge_range(const uint64_t* keys, const uint64_t* off, int k, uint64_t o_lo,
-                      uint64_t o_hi, uint64_t* out, bool out_f64, int threads) {
+void host_merge_runs_range(const uint64_t* const* run, const uint64_t* len, int k, uint64_t o_lo,
+                           uint64_t o_hi, uint64_t* out, bool out_f64, int threads,
+                           ThreadPool* pool) {
   if (threads <= 0) threads = host_threads();
-  const uint64_t total = off[k] - off[0];
+  ThreadPool& tp = pool ? *pool : host_pool();
+  uint64_t total = 0;
+  for (int j = 0; j < k; ++j) total += len[j];
   if (o_hi > total) o_hi = total;
   if (o_lo >= o_hi) return;
-  std::vector<uint64_t> o2(k + 1);
-  for (int j = 0; j <= k; ++j) o2[j] = off[j] - off[0];
-  const uint64_t* K = keys + off[0];
   const uint64_t span = o_hi - o_lo;
   // ranges: ~4 per thread, each at least 64K keys
   int64_t R = std::max<int64_t>(1, std::min<int64_t>((int64_t)threads * 4, (int64_t)(span >> 16)));
   std::vector<uint64_t> ranks((R + 1) * (uint64_t)k);
   auto pos = [&](int64_t r) { return o_lo + (uint64_t)((__uint128_t)span * (uint64_t)r / (uint64_t)R); };
-  host_pool().parallel_for(R + 1, threads, [&](int64_t r) {
-    host_corank(K, o2.data(), k, pos(r), &ranks[(uint64_t)r * k]);
+  tp.parallel_for(R + 1, threads, [&](int64_t r) {
+    host_corank_runs(run, len, k, pos(r), &ranks[(uint64_t)r * k]);
   });
-  host_pool().parallel_for(R, threads, [&](int64_t r) {
-    merge_range(K, o2.data(), k, &ranks[(uint64_t)r * k], &ranks[(uint64_t)(r + 1) * k],
+  tp.parallel_for(R, threads, [&](int64_t r) {
+    merge_range(run, len, k, &ranks[(uint64_t)r * k], &ranks[(uint64_t)(r + 1) * k],
                 out + (pos(r) - o_lo), out_f64);
     _mm_sfence();
   });
+}
+
+namespace {
+struct RunView {  // (pointer, length) view of runs stored back to back: keys[off[j] .. off[j+1])
+  std::vector<const uint64_t*> p;
+  std::vector<uint64_t> len;
+  RunView(const uint64_t* keys, const uint64_t* off, int k) : p(k), len(k) {
+    for (int j = 0; j < k; ++j) {
+      p[j] = keys + off[j];
+      len[j] = off[j + 1] - off[j];
+    }
+  }
+};
+}  // namespace
+
+void host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t o, uint64_t* ranks) {
+  RunView v(keys, off, k);
+  host_corank_runs(v.p.data(), v.len.data(), k, o, ranks);
+}
+
+void host_merge_range(const uint64_t* keys, const uint64_t* off, int k, uint64_t o_lo,
+                      uint64_t o_hi, uint64_t* out, bool out_f64, int threads) {
+  RunView v(keys, off, k);
+  host_merge_runs_range(v.p.data(), v.len.data(), k, o_lo, o_hi, out, out_f64, threads, nullptr);
 }
 
 void host_merge(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out, bool out_f64,

@@ -79,6 +79,11 @@ ThreadPool& host_pool() {
   return pool;
 }
 
+ThreadPool& pipe_pool() {
+  static ThreadPool pool(std::max(1, host_threads() / 2 - 1));
+  return pool;
+}
+
 void par_memcpy(void* dst, const void* src, uint64_t bytes, int threads) {
   if (threads <= 0) threads = host_threads();
   constexpr uint64_t kMinChunk = 2ull << 20;

@@ -45,6 +45,9 @@ class ThreadPool {
 
 // Process-wide pool (created on first use, sized to the hardware threads).
 ThreadPool& host_pool();
+// Second pool for the PIPEMERGE pair merges that run during the sort phase, so they never queue
+// ahead of the PARMEMCPY staging jobs on host_pool() (half the hardware threads).
+ThreadPool& pipe_pool();
 int host_threads();
 
 // PARMEMCPY: dst <- src (bytes) split over `threads` workers (0 = all host threads).

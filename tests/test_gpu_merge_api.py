@@ -231,3 +231,35 @@ def test_stats_fields(hs_gpu, inputs_mod):
     assert st["n_b"] == 4 and st["passes_run"] >= 1
     assert st["bytes_h2d"] == A.nbytes and st["bytes_d2h"] == A.nbytes
     assert st["t_total"] > 0 and st["t_gpu_sort"] > 0 and st["t_h2d"] > 0
+
+
+@pytest.mark.parametrize("n,b", [(3 * 100_000, 100_000), (4 * 100_000 - 7, 100_000),
+                                 (5 * 65_536 + 1, 65_536), (6 * 100_000, 100_000),
+                                 (9 * 50_000 + 123, 50_000)])
+@pytest.mark.parametrize("permille,pin_w", [(0, 1), (500, 1), (-1, 0), (1000, 0)])
+def test_stream_pipemerge(hs_gpu, oracle_mod, inputs_mod, n, b, permille, pin_w):
+    """PIPEMERGE (S§8(f) #1): STREAM mode pre-merges pairs (0,1), (2,3), ... of sorted
+    batches on the host threads during the sort phase, pipemerge_count(n_b, 1) of them (reading
+    A-9, pinned by tests/golden/fig3_pipemerge.txt), and the final merge takes the merged pairs plus
+    the remaining batches.  Output bit-exact vs the oracle for even/odd n_b and ragged last
+    batches, with every merge split f."""
+    A = inputs_mod.generate("normal" if n % 2 else "zipf_dup", n, seed=n + permille)
+    want = _bits(oracle_mod.sort_f64(A))
+    n_b = -(-n // b)
+    m = oracle_mod.pipemerge_count(n_b, 1)
+    opts = {"resident": 0, "merge_gpu_permille": permille, "pin_w": pin_w, "merge_chunk": 1 << 18}
+    old = {k: hs_gpu.hsort_get_option(k) for k in list(opts) + ["pipemerge"]}
+    for k, v in opts.items():
+        hs_gpu.hsort_set_option(k, v)
+    try:
+        for pm in (1, 0):
+            hs_gpu.hsort_set_option("pipemerge", pm)
+            B = hs_gpu.hsort_sort(A, batch_elems=b)
+            st = hs_gpu.hsort_get_stats()
+            assert st["mode_name"] == "STREAM" and st["n_b"] == n_b
+            assert np.array_equal(_bits(B), want), (n, b, permille, pm)
+            assert st["pipe_merges"] == (m if pm else 0)
+            assert st["merge_k"] == n_b - (m if pm else 0)
+    finally:
+        for k, v in old.items():
+            hs_gpu.hsort_set_option(k, v)

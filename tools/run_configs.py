@@ -6,6 +6,7 @@ C3s: the paper's out-of-core workflow (STREAM: batches -> W -> CPU/GPU merge) wi
 C4s: normal and zipf-dup skew, auto plan, n = N4.
 C5s: fixed n = N5, sweep b_s and the merge split f in STREAM mode; reports end-to-end time next to
      the "GPU-only" sum (sum HtoD + sum DtoH + sum GPUSort) the paper criticises.
+C6p: PIPEMERGE on/off in STREAM mode at n = N6 over several b_s, CPU-only merge and A12 split.
 Large outputs are verified by sortedness + multiset hash (oracle verifiers; unique answer, A-4).
 Prints one JSON line per run.
 """
@@ -62,7 +63,8 @@ def main():
     ap.add_argument("--n3", type=float, default=4e9)
     ap.add_argument("--n4", type=float, default=4e9)
     ap.add_argument("--n5", type=float, default=2e9)
-    ap.add_argument("--only", default="C1,C3s,C4s,C5s")
+    ap.add_argument("--n6", type=float, default=2e9)
+    ap.add_argument("--only", default="C1,C3s,C4s,C5s,C6p")
     a = ap.parse_args()
     which = set(a.only.split(","))
     hs.hsort_init()
@@ -92,6 +94,18 @@ def main():
             for pm in (0, 250, 500, 750, 1000, -1):
                 run("C5s-sweep", A, B, b, {"resident": 0, "merge_gpu_permille": pm})
         run("C5s-auto", A, B, 0, {})
+        del A, B
+    if "C6p" in which:
+        # PIPEMERGE ablation (S§8(f) #1, Fig. 6): pair-wise merges during the sort
+        # phase on/off, with the paper's CPU-only merge (f = 0) and with the A12 split
+        n = int(a.n6)
+        A = hsort_inputs.generate("uniform", n, seed=7)
+        B = np.empty_like(A)
+        for b in (1 << 26, 1 << 27, 250_000_000):
+            for pm in (0, 1):
+                for f in (0, -1):
+                    run("C6p-pipemerge", A, B, b, {"resident": 0, "pipemerge": pm, "merge_gpu_permille": f,
+                                                   "pin_w_max_mb": 24576}, reps=2)
     hs.hsort_finalize()
 
 

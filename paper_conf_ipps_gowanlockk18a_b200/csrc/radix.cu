@@ -33,6 +33,9 @@ constexpr uint64_t kCountMask = (1ull << 40) - 1;
 constexpr uint32_t kEpochMask = (1u << 22) - 1;
 #ifdef HSORT_PHASE_TIMING
 __device__ unsigned long long g_phase_dbg[256];  // instrumented builds only
+#ifndef HSORT_FAKE
+#define HSORT_FAKE 0  // tools/ab_build.sh timing experiments (1 no look-back, 2 no ranking, 3 no write-out)
+#endif
 #endif
 
 // float64 bits -> key: negative -> ~u, non-negative -> u | 2^63 (IEEE totalOrder as unsigned).
@@ -488,6 +491,13 @@ __device__ __forceinline__ uint32_t lookback_window32(const uint32_t* __restrict
       w[q] = (j - q >= 0) ? ld_relaxed32(&lb[(uint64_t)(j - q) * kRadix + d]) : (2u << 30);
     int q = 0;
     bool done = false;
+#ifdef HSORT_PHASE_TIMING
+    if (d == 0) {
+      atomicAdd(&g_phase_dbg[200], 1ull);                      // rounds
+      if ((w[0] >> 30) == 0) atomicAdd(&g_phase_dbg[201], 1ull);  // nearest unpublished: spin
+      if ((w[0] >> 30) == 2) atomicAdd(&g_phase_dbg[202], 1ull);  // nearest has P
+    }
+#endif
 #pragma unroll
     for (int u = 0; u < W; ++u) {
       if (done || q != u) continue;
@@ -571,6 +581,8 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
     if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bars[b]);
   };
 
+  // this thread's digit base for the pass, loaded once (not an L2 round trip after each look-back)
+  const uint64_t my_bin_base = tid < kRadix ? bin_base[digit * kRadix + tid] : 0;
   uint32_t claim_next = 0;  // thread 0: tile id claimed one iteration ahead (atomic off the path)
   if (tid == 0) {
     mbar_init(&bars[0], 1);
@@ -699,6 +711,10 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
           }
         }
       }
+#if HSORT_FAKE == 2  // timing experiment only: no ranking (wrong output)
+#pragma unroll
+      for (int i = 0; i < RC; ++i) peers[i] = 1u << lane;
+#endif
 #pragma unroll
       for (int i = 0; i < RC; ++i) {
         const int leader = 31 - __clz(peers[i]);
@@ -721,14 +737,18 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
       uint64_t excl = 0;
       if (tile > 0) {
         if (S32) {
+#if HSORT_FAKE == 1  // timing experiment only: no look-back (wrong output)
+          excl = 0;
+#else
           excl = lookback_window32<(LBW & 255)>(lb32, (int64_t)tile - 1, tid);
+#endif
           st_relaxed32(&lb32[tile * kRadix + tid], (2u << 30) | (uint32_t)(excl + cnt));
         } else {
           excl = lookback_window<(LBW & 255), ((LBW >> 8) & 255)>(lookback, (int64_t)tile - 1, tid, ep);
           st_relaxed(&lookback[tile * kRadix + tid], kFlagP | ((uint64_t)ep << 40) | (excl + cnt));
         }
       }
-      s_gofs[tid] = bin_base[digit * kRadix + tid] + excl - (uint64_t)tstart;
+      s_gofs[tid] = my_bin_base + excl - (uint64_t)tstart;
     }
     __syncthreads();
     HSORT_PHASE(4);
@@ -747,8 +767,14 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
 #pragma unroll
           for (int q = 0; q < WC; ++q) dst[g[q] + tid + (c0 + q) * THREADS] = from_key(v[q]);
         } else {
+#if HSORT_FAKE == 3  // timing experiment only: no HBM write-out (wrong output)
+#pragma unroll
+          for (int q = 0; q < WC; ++q)
+            if (v[q] == 0x123456789ull) dst[g[q] + tid + (c0 + q) * THREADS] = v[q];
+#else
 #pragma unroll
           for (int q = 0; q < WC; ++q) dst[g[q] + tid + (c0 + q) * THREADS] = v[q];
+#endif
         }
       }
     } else if (inv) {
@@ -916,8 +942,11 @@ int env_int(const char* name, int dflt) {
   const char* v = getenv(name);
   return v ? atoi(v) : dflt;
 }
+#ifndef HSORT_DEFAULT_PASS_VARIANT
+#define HSORT_DEFAULT_PASS_VARIANT 2
+#endif
 int pass_variant() {
-  static int v = env_int("HSORT_PASS_VARIANT", 1);
+  static int v = env_int("HSORT_PASS_VARIANT", HSORT_DEFAULT_PASS_VARIANT);
   return v;
 }
 int hist_variant() {
@@ -976,6 +1005,377 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------------------------------
+// K3 v3: warp-specialised onesweep pass (default).  CTA = 8 compute warps + 1 look-back warp.
+//
+// The decoupled look-back is the largest single cost of a pass (removing it, output wrong, cuts a
+// 2^30-key pass from 7.3 to 5.0 ms: profiles/r01_pass_floors.txt), and in v2 every thread of the
+// CTA waits for it.  Here the look-back of tile t runs on its own warp (each lane owns 8 digits)
+// while the compute warps rank the next tile; the compute warps write tile t out one iteration
+// later.  The inclusive prefix is still published as soon as the look-back resolves, so
+// successors wait no longer than in v2.  Three 4096-key stage buffers rotate: tile j+2 is
+// prefetched (TMA) while tile j is ranked and tile j-1 is written out.
+//
+// Hand-offs (shared-memory mbarriers): bar_tma[3] TMA completion; bar_a[2] "tile j counted, A
+// published, counts and tile starts in s_cnt" (compute -> look-back warp); bar_g[2] "global
+// offsets of tile j in s_gofs" (look-back warp -> compute).  32-bit status words only (n <= 2^30).
+// Forward progress: a CTA's claims increase, so the smallest tile without an inclusive prefix is
+// either being looked back (its predecessor has P) or queued behind smaller tiles of its own CTA,
+// which all have P, and nothing in the CTA waits on a larger tile.
+template <int CT>
+__device__ __forceinline__ void bar_compute() { asm volatile("bar.sync 1, %0;" ::"n"(CT) : "memory"); }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// exclusive scan of one value per digit thread (threads 0..255) among CT compute threads,
+// named barrier 1 (threads >= 256 pass v = 0 and ignore the result)
+template <int CT>
+__device__ __forceinline__ uint32_t scan256_excl_c(uint32_t v, uint32_t* s_warp /*[8]*/) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31 && warp < 8) s_warp[warp] = x;
+  bar_compute<CT>();
+  uint32_t wpre = 0;
+#pragma unroll
+  for (int w = 0; w < 8; ++w)
+    if (w < warp) wpre += s_warp[w];
+  return wpre + x - v;
+}
+
+template <int CT, int ITEMS>
+struct WsSmem {
+  static constexpr int TILE = CT * ITEMS;
+  static constexpr int CW = CT / 32;                                          // compute warps
+  static constexpr size_t stage_off = 0;                                      // [3][TILE] u64
+  static constexpr size_t whist_off = 3ull * TILE * 8;                        // [CW][257] u32
+  static constexpr size_t gofs_off = (whist_off + CW * (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [2][256] u64
+  static constexpr size_t cnt_off = gofs_off + 2 * kRadix * 8;                // [2][256] u32
+  static constexpr size_t bar_off = cnt_off + 2 * kRadix * 4;                 // [8] u64
+  static constexpr size_t swarp_off = bar_off + 8 * 8;                        // [8] u32 (+pad)
+  static constexpr size_t tile_off = swarp_off + 64;                          // [4] u32
+  static constexpr size_t bytes = tile_off + 16;
+};
+
+#ifndef HSORT_WS_CT
+#define HSORT_WS_CT 480  // compute threads of the warp-specialised pass (15 warps + 1 look-back warp)
+#endif
+#ifndef HSORT_WS_ITEMS
+#define HSORT_WS_ITEMS 17  // keys per compute thread: 8160-key tiles, 3 stages = 191 KB, 1 CTA/SM
+#endif
+#ifndef HSORT_WS_W
+#define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
+#endif
+template <int W>
+__device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64_t tile, int lane,
+                                          uint32_t* excl) {
+  // 8 digits per lane (d = lane + 32 q).  The warp walks back one tile row at a time for all 256
+  // digits together (W rows per round trip): a digit stops at its first inclusive prefix, and the
+  // walk pauses (re-reads from that row) while any still-walking digit's word is unpublished.
+  uint32_t live = 0xffu;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) excl[q] = 0;
+  int64_t j = tile - 1;
+  while (true) {
+    uint32_t w[W][8];
+#pragma unroll
+    for (int u = 0; u < W; ++u)
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        w[u][q] = (j - u >= 0) ? ld_relaxed32(&lb[(uint64_t)(j - u) * kRadix + lane + 32 * q]) : (2u << 30);
+    int u = 0;
+#pragma unroll
+    for (; u < W; ++u) {
+      bool ok = true;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) ok &= !((live >> q) & 1) || (w[u][q] >> 30) != 0u;
+      if (!__all_sync(0xffffffffu, ok)) break;  // warp-uniform
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        if ((live >> q) & 1) {
+          excl[q] += w[u][q] & 0x3FFFFFFFu;
+          if ((w[u][q] >> 30) == 2u) live &= ~(1u << q);
+        }
+      if (!__any_sync(0xffffffffu, live != 0)) return;
+    }
+    j -= u;
+  }
+}
+
+template <int CT, int ITEMS, bool IN_F64>
+__global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in, uint64_t* out, uint64_t* tmp,
+                                                       uint64_t n, const RadixPlan* __restrict__ plan,
+                                                       const uint64_t* __restrict__ bin_base,
+                                                       uint64_t* __restrict__ lookback,
+                                                       uint32_t* __restrict__ tile_ctr, int p,
+                                                       int out_f64, uint64_t lb_half,
+                                                       uint64_t lb_rows) {
+  using L = WsSmem<CT, ITEMS>;
+  constexpr int TILE = L::TILE;
+  constexpr int CW = L::CW;
+  constexpr int THREADS = CT;  // compute threads
+  extern __shared__ __align__(128) unsigned char smem[];
+  uint64_t* stage = (uint64_t*)(smem + L::stage_off);
+  uint32_t* whist = (uint32_t*)(smem + L::whist_off);
+  uint64_t* s_gofs = (uint64_t*)(smem + L::gofs_off);
+  uint32_t* s_cnt = (uint32_t*)(smem + L::cnt_off);
+  uint64_t* bars = (uint64_t*)(smem + L::bar_off);
+  uint32_t* s_warp = (uint32_t*)(smem + L::swarp_off);
+  uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
+  uint64_t* bar_tma = bars;      // [3]
+  uint64_t* bar_a = bars + 3;    // [2]
+  uint64_t* bar_g = bars + 5;    // [2]
+
+  const int na = plan->num_active;
+  if (p >= na) return;
+  const int digit = plan->digit[p];
+  const int shift = 8 * digit;
+  const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
+  uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const bool use_match = (plan->match_mask >> p) & 1;
+  const bool inv = out_f64 && (p == na - 1);
+  uint32_t* lb32 = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p) & 1) * lb_half;
+  uint32_t* lb32_next = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p + 1) & 1) * lb_half;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t num_tiles = (n + TILE - 1) / TILE;
+
+  auto issue = [&](uint64_t t, int b) {  // one thread: stage b <- tile t
+    const uint64_t base = t * (uint64_t)TILE;
+    const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
+    const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
+    mbar_arrive_expect_tx(&bar_tma[b], bytes);
+    if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bar_tma[b]);
+  };
+  if (tid == 0) {
+    for (int b = 0; b < 3; ++b) mbar_init(&bar_tma[b], 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&bar_a[b], 1);
+      mbar_init(&bar_g[b], 1);
+    }
+    mbar_fence_init();
+    for (int b = 0; b < 2; ++b) {
+      const uint32_t t = atomicAdd(&tile_ctr[p], 1u);
+      s_tile[b] = t;
+      if (t < num_tiles) issue(t, b);
+    }
+  }
+  __syncthreads();
+
+  if (warp == CW) {
+    // ================= look-back warp =================
+    uint64_t base[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) base[q] = bin_base[digit * kRadix + lane + 32 * q];
+    for (uint32_t j = 0;; ++j) {
+      mbar_wait(&bar_a[j & 1], (j >> 1) & 1u);
+      const uint64_t tile = s_tile[j % 3];
+      if (tile >= num_tiles) break;
+      uint32_t cw[8], excl[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cw[q] = s_cnt[(j & 1) * kRadix + lane + 32 * q];
+      if (tile > 0) {
+#if HSORT_FAKE == 1
+#pragma unroll
+        for (int q = 0; q < 8; ++q) excl[q] = 0;
+#else
+        lookback8<HSORT_WS_W>(lb32, (int64_t)tile, lane, excl);
+#endif
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          st_relaxed32(&lb32[tile * kRadix + lane + 32 * q], (2u << 30) | (excl[q] + (cw[q] & 0xFFFFu)));
+      } else {
+#pragma unroll
+        for (int q = 0; q < 8; ++q) excl[q] = 0;
+      }
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        s_gofs[(j & 1) * kRadix + lane + 32 * q] = base[q] + excl[q] - (uint64_t)(cw[q] >> 16);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bar_g[j & 1]);
+    }
+    return;
+  }
+
+  // ================= compute warps (256 threads) =================
+  const uint32_t lt = lanemask_lt();
+  uint32_t claim = 0;  // thread 0: tile j+2, claimed at the start of iteration j
+  uint32_t j = 0;
+  auto write_out = [&](uint32_t jj) {  // tile of iteration jj from its stage buffer
+    const uint64_t tile = s_tile[jj % 3];
+    mbar_wait(&bar_g[jj & 1], (jj >> 1) & 1u);
+    const uint64_t* gofs = s_gofs + (jj & 1) * kRadix;
+    const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
+    const uint64_t rem = n - tile * (uint64_t)TILE;
+    const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+    if (tile_n == TILE) {
+#pragma unroll
+      for (int q = 0; q < ITEMS; ++q) {
+        const uint64_t v = sb[tid + q * THREADS];
+        const uint64_t g = gofs[(uint32_t)(v >> shift) & 255u];
+        dst[g + tid + q * THREADS] = inv ? from_key(v) : v;
+      }
+    } else {
+      for (int i = tid; i < tile_n; i += THREADS) {
+        const uint64_t v = sb[i];
+        dst[gofs[(uint32_t)(v >> shift) & 255u] + i] = inv ? from_key(v) : v;
+      }
+    }
+  };
+  while (true) {
+    const int cb = (int)(j % 3);
+    const uint64_t tile = s_tile[cb];
+    if (tile >= num_tiles) break;
+    if (tid == 0) claim = atomicAdd(&tile_ctr[p], 1u);  // consumed at the end of the iteration
+    for (int i = tid; i < CW * (kRadix + 1); i += THREADS) whist[i] = 0;
+    mbar_wait(&bar_tma[cb], (j / 3) & 1u);
+    bar_compute<CT>();
+
+    const uint64_t tbase = tile * (uint64_t)TILE;
+    const uint64_t rem = n - tbase;
+    const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+    const bool full = tile_n == TILE;
+    const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
+    uint64_t* sb = stage + (size_t)cb * TILE;
+    const int wofs = warp * 32 * ITEMS + lane;
+    uint32_t* wh = whist + warp * (kRadix + 1);
+
+    uint64_t k[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      const int jj = wofs + i * 32;
+      uint64_t v;
+      if (full) v = sb[jj];
+      else v = jj < bulk_n ? sb[jj] : (jj < tile_n ? src[tbase + jj] : 0);
+      k[i] = IN_F64 ? to_key(v) : v;
+    }
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      const bool valid = full || (wofs + i * 32 < tile_n);
+      atomicAdd(&wh[valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix], 1u);
+    }
+    bar_compute<CT>();
+    uint32_t cnt = 0;
+    if (tid < kRadix) {
+#pragma unroll
+      for (int w = 0; w < CW; ++w) cnt += whist[w * (kRadix + 1) + tid];
+      st_relaxed32(&lb32[tile * kRadix + tid], ((tile == 0 ? 2u : 1u) << 30) | cnt);
+      lb32_next[tile * kRadix + tid] = 0;  // the next pass's array, row of this tile
+    }
+    const uint32_t tstart = scan256_excl_c<CT>(cnt, s_warp);
+    if (tid < kRadix) {
+      uint32_t run = tstart;
+#pragma unroll
+      for (int w = 0; w < CW; ++w) {
+        const uint32_t c = whist[w * (kRadix + 1) + tid];
+        whist[w * (kRadix + 1) + tid] = run;
+        run += c;
+      }
+      s_cnt[(j & 1) * kRadix + tid] = cnt | (tstart << 16);
+    }
+    bar_compute<CT>();
+    if (tid == 0) mbar_arrive(&bar_a[j & 1]);
+
+    // rank (as v2): the leader's atomic on the warp's base returns the group's first slot
+    uint32_t r[ITEMS];
+    {
+      uint32_t dd[ITEMS], peers[ITEMS];
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const bool valid = full || (wofs + i * 32 < tile_n);
+        dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+      }
+      if (use_match) {
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+      } else {
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) peers[i] = 0xffffffffu;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+#pragma unroll
+          for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t bit = (dd[i] >> b) & 1u;
+            peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+          }
+        }
+        if (!full) {
+#pragma unroll
+          for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t bit = (dd[i] >> 8) & 1u;
+            peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
+          }
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const int leader = 31 - __clz(peers[i]);
+        r[i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+      }
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) {
+        const int leader = 31 - __clz(peers[i]);
+        r[i] = __shfl_sync(0xffffffffu, r[i], leader) + __popc(peers[i] & lt);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i)
+      if (full || wofs + i * 32 < tile_n) sb[r[i]] = k[i];
+
+    if (j >= 1) write_out(j - 1);
+    bar_compute<CT>();  // stage (j-1)%3 fully read; whist free
+    if (tid == 0) {
+      const int nb = (int)((j + 2) % 3);
+      s_tile[nb] = claim;
+      if (claim < num_tiles) issue(claim, nb);
+    }
+    ++j;
+  }
+  // tell the look-back warp to stop, then drain the last tile
+  if (tid == 0) mbar_arrive(&bar_a[j & 1]);
+  if (j >= 1) write_out(j - 1);
+  if (tid < kRadix)
+    for (uint64_t rr = num_tiles + blockIdx.x; rr < lb_rows; rr += gridDim.x)
+      lb32_next[rr * kRadix + tid] = 0;
+}
+
+template <int CT, int ITEMS>
+cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n, RadixScratch& s,
+                           int p, bool first_in_f64, bool out_f64, cudaStream_t st) {
+  using L = WsSmem<CT, ITEMS>;
+  static int blocks_per_sm[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  auto kt = k_onesweep_ws<CT, ITEMS, true>;
+  auto kf = k_onesweep_ws<CT, ITEMS, false>;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  if (!blocks_per_sm[dev]) {
+    cudaError_t e;
+    if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
+    if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L::bytes)) != cudaSuccess) return e;
+    int b = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, CT + 32, L::bytes)) != cudaSuccess) return e;
+    blocks_per_sm[dev] = b > 0 ? b : 1;
+  }
+  const uint64_t tiles = (n + L::TILE - 1) / L::TILE;
+  if (tiles > s.max_tiles) return cudaErrorInvalidValue;
+  uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
+  if (grid > tiles) grid = tiles ? tiles : 1;
+  if (first_in_f64)
+    kt<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
+                                             s.tile_ctr, p, out_f64 ? 1 : 0, s.max_tiles * kRadix,
+                                             s.lb_rows);
+  else
+    kf<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
+                                             s.tile_ctr, p, out_f64 ? 1 : 0, s.max_tiles * kRadix,
+                                             s.lb_rows);
+  return cudaGetLastError();
+}
+
 // Look-back status format of one sort: 2 = 32-bit words (TMA pass, n <= 2^30: an active digit
 // has at most n - 1 keys), 1 = 64-bit epoch-tagged words.  Switching formats re-zeroes the array
 // so stale words of the other format can never be read as published.
@@ -989,7 +1389,7 @@ int pass_kernel(uint64_t* in, uint64_t* out, uint64_t* tmp) {
 // single pass) is only read by tiles without keys of d and decodes as flag 3 = "aggregate", so a
 // reader never spins on it.
 cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t st) {
-  const int mode = (kernel == 1 && n <= (1ull << 30)) ? 2 : 1;
+  const int mode = (kernel >= 1 && n <= (1ull << 30)) ? 2 : 1;
   if (s.lb_mode != 0 && s.lb_mode != mode) {
     cudaError_t e = cudaMemsetAsync(s.lookback, 0, s.max_tiles * kRadix * sizeof(uint64_t), st);
     if (e != cudaSuccess) return e;
@@ -997,7 +1397,8 @@ cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t
   }
   s.lb_mode = mode;
   if (mode == 2) {
-    const uint64_t t = (n + kRadixTile - 1) / kRadixTile;
+    const uint64_t tile = kernel == 2 ? (uint64_t)HSORT_WS_CT * HSORT_WS_ITEMS : (uint64_t)kRadixTile;
+    const uint64_t t = (n + tile - 1) / tile;
     if (t > s.lb_rows) s.lb_rows = t;
   }
   return cudaSuccess;
@@ -1010,8 +1411,10 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   if (e != cudaSuccess) return e;
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const int v = pass_kernel(in, out, tmp);
+  if (v == 2 && s.lb_mode == 2)
+    return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS>(in, out, tmp, n, s, p, first_in_f64, out_f64, st);
   // look-back window 4: measured best of 1..32
-  if (v == 1) {
+  if (v >= 1) {
     if (s.lb_mode == 2)
       return launch_tma_pass<256, 16, 4, 2, true>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);
     return launch_tma_pass<256, 16, 4, 2, false>(in, out, tmp, n, s, ep, p, first_in_f64, out_f64, st);

@@ -36,4 +36,6 @@ for p in range(8):
         res[p] = {nm: round(buf[p * 16 + i] / tiles) for i, nm in names.items()}
         res[p]["tiles"] = tiles
 print(json.dumps(res))
-print("lookback windows (digit 0) per tile:", buf[200] / max(1, sum(buf[p * 16 + 8] for p in range(8))))
+T = max(1, sum(buf[p * 16 + 8] for p in range(8)))
+print("lookback rounds (digit 0) per tile:", buf[200] / T, " rounds whose nearest window tile was unpublished:",
+      buf[201] / T, " rounds whose nearest tile had P:", buf[202] / T)

@@ -1068,43 +1068,87 @@ struct WsSmem {
 #ifndef HSORT_WS_ITEMS
 #define HSORT_WS_ITEMS 17  // keys per compute thread: 8160-key tiles, 3 stages = 191 KB, 1 CTA/SM
 #endif
+#ifndef HSORT_WS_RC
+#define HSORT_WS_RC 0  // ranking chunk (0 = all items at once)
+#endif
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
 #endif
+__device__ __forceinline__ void ld_relaxed_v4(const uint32_t* p, uint32_t* v) {
+  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
+               : "l"(p)
+               : "memory");
+}
+__device__ __forceinline__ void st_relaxed_v4(uint32_t* p, const uint32_t* v) {
+  asm volatile("st.relaxed.gpu.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v[0]), "r"(v[1]),
+               "r"(v[2]), "r"(v[3])
+               : "memory");
+}
+
 template <int W>
 __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64_t tile, int lane,
                                           uint32_t* excl) {
-  // 8 digits per lane (d = lane + 32 q).  The warp walks back one tile row at a time for all 256
-  // digits together (W rows per round trip): a digit stops at its first inclusive prefix, and the
-  // walk pauses (re-reads from that row) while any still-walking digit's word is unpublished.
-  uint32_t live = 0xffu;
+  // Lane owns digits 8 lane .. 8 lane + 7 (two 16-byte loads per tile row).  The warp walks back
+  // one tile row at a time for all 256 digits together, W rows per round trip.  Fast path: a row
+  // whose 256 words are all aggregates is summed raw (flag bits removed once at the end).  Else
+  // per digit: a digit stops at its first inclusive prefix, and the walk pauses (re-reads from
+  // that row) while any still-walking digit's word is unpublished.
+  uint32_t raw[8], msk[8];
 #pragma unroll
-  for (int q = 0; q < 8; ++q) excl[q] = 0;
+  for (int q = 0; q < 8; ++q) raw[q] = msk[q] = 0;
+  uint32_t live = 0xffu, n_raw = 0;
+  const uint32_t* row0 = lb + lane * 8;
   int64_t j = tile - 1;
   while (true) {
+#ifdef HSORT_PHASE_TIMING
+    if (lane == 0) atomicAdd(&g_phase_dbg[216], 1ull);
+#endif
     uint32_t w[W][8];
 #pragma unroll
-    for (int u = 0; u < W; ++u)
+    for (int u = 0; u < W; ++u) {
+      if (j - u >= 0) {
+        ld_relaxed_v4(row0 + (uint64_t)(j - u) * kRadix, &w[u][0]);
+        ld_relaxed_v4(row0 + (uint64_t)(j - u) * kRadix + 4, &w[u][4]);
+      } else {
 #pragma unroll
-      for (int q = 0; q < 8; ++q)
-        w[u][q] = (j - u >= 0) ? ld_relaxed32(&lb[(uint64_t)(j - u) * kRadix + lane + 32 * q]) : (2u << 30);
+        for (int q = 0; q < 8; ++q) w[u][q] = 2u << 30;  // before tile 0: prefix 0
+      }
+    }
     int u = 0;
 #pragma unroll
     for (; u < W; ++u) {
+      uint32_t a = w[u][0], o = w[u][0];
+#pragma unroll
+      for (int q = 1; q < 8; ++q) {
+        a &= w[u][q];
+        o |= w[u][q];
+      }
+      // every word of the row an aggregate (flag 01) and every digit still walking
+      const bool allA = live == 0xffu && (a >> 30) == 1u && (o >> 31) == 0u;
+      if (__all_sync(0xffffffffu, allA)) {
+#pragma unroll
+        for (int q = 0; q < 8; ++q) raw[q] += w[u][q];
+        ++n_raw;
+        continue;
+      }
       bool ok = true;
 #pragma unroll
       for (int q = 0; q < 8; ++q) ok &= !((live >> q) & 1) || (w[u][q] >> 30) != 0u;
-      if (!__all_sync(0xffffffffu, ok)) break;  // warp-uniform
+      if (!__all_sync(0xffffffffu, ok)) break;  // warp-uniform: re-read from row u
 #pragma unroll
       for (int q = 0; q < 8; ++q)
         if ((live >> q) & 1) {
-          excl[q] += w[u][q] & 0x3FFFFFFFu;
+          msk[q] += w[u][q] & 0x3FFFFFFFu;
           if ((w[u][q] >> 30) == 2u) live &= ~(1u << q);
         }
-      if (!__any_sync(0xffffffffu, live != 0)) return;
+      if (!__any_sync(0xffffffffu, live != 0)) break;
     }
+    if (!__any_sync(0xffffffffu, live != 0)) break;
     j -= u;
   }
+#pragma unroll
+  for (int q = 0; q < 8; ++q) excl[q] = raw[q] - (n_raw << 30) + msk[q];
 }
 
 template <int CT, int ITEMS, bool IN_F64>
@@ -1170,14 +1214,24 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     // ================= look-back warp =================
     uint64_t base[8];
 #pragma unroll
-    for (int q = 0; q < 8; ++q) base[q] = bin_base[digit * kRadix + lane + 32 * q];
+    for (int q = 0; q < 8; ++q) base[q] = bin_base[digit * kRadix + lane * 8 + q];
+#ifdef HSORT_PHASE_TIMING
+    unsigned long long t_wait = 0, t_lb = 0, n_lb = 0;
+#endif
     for (uint32_t j = 0;; ++j) {
+#ifdef HSORT_PHASE_TIMING
+      long long c0 = clock64();
+#endif
       mbar_wait(&bar_a[j & 1], (j >> 1) & 1u);
+#ifdef HSORT_PHASE_TIMING
+      long long c1 = clock64();
+      t_wait += c1 - c0;
+#endif
       const uint64_t tile = s_tile[j % 3];
       if (tile >= num_tiles) break;
       uint32_t cw[8], excl[8];
 #pragma unroll
-      for (int q = 0; q < 8; ++q) cw[q] = s_cnt[(j & 1) * kRadix + lane + 32 * q];
+      for (int q = 0; q < 8; ++q) cw[q] = s_cnt[(j & 1) * kRadix + lane * 8 + q];
       if (tile > 0) {
 #if HSORT_FAKE == 1
 #pragma unroll
@@ -1185,19 +1239,32 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #else
         lookback8<HSORT_WS_W>(lb32, (int64_t)tile, lane, excl);
 #endif
+#ifdef HSORT_PHASE_TIMING
+        t_lb += clock64() - c1;
+        ++n_lb;
+#endif
+        uint32_t pv[8];
 #pragma unroll
-        for (int q = 0; q < 8; ++q)
-          st_relaxed32(&lb32[tile * kRadix + lane + 32 * q], (2u << 30) | (excl[q] + (cw[q] & 0xFFFFu)));
+        for (int q = 0; q < 8; ++q) pv[q] = (2u << 30) | (excl[q] + (cw[q] & 0xFFFFu));
+        st_relaxed_v4(&lb32[tile * kRadix + lane * 8], pv);
+        st_relaxed_v4(&lb32[tile * kRadix + lane * 8 + 4], pv + 4);
       } else {
 #pragma unroll
         for (int q = 0; q < 8; ++q) excl[q] = 0;
       }
 #pragma unroll
       for (int q = 0; q < 8; ++q)
-        s_gofs[(j & 1) * kRadix + lane + 32 * q] = base[q] + excl[q] - (uint64_t)(cw[q] >> 16);
+        s_gofs[(j & 1) * kRadix + lane * 8 + q] = base[q] + excl[q] - (uint64_t)(cw[q] >> 16);
       __syncwarp();
       if (lane == 0) mbar_arrive(&bar_g[j & 1]);
     }
+#ifdef HSORT_PHASE_TIMING
+    if (lane == 0) {
+      atomicAdd(&g_phase_dbg[214], t_wait);
+      atomicAdd(&g_phase_dbg[215], t_lb);
+      atomicAdd(&g_phase_dbg[217], n_lb);
+    }
+#endif
     return;
   }
 
@@ -1205,9 +1272,19 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   const uint32_t lt = lanemask_lt();
   uint32_t claim = 0;  // thread 0: tile j+2, claimed at the start of iteration j
   uint32_t j = 0;
+#ifdef HSORT_PHASE_TIMING
+  unsigned long long t_g = 0, t_t = 0, t_all = 0, t_rank = 0, t_cnt = 0, t_wo = 0, n_t = 0;
+  long long c_start = clock64();
+#endif
   auto write_out = [&](uint32_t jj) {  // tile of iteration jj from its stage buffer
     const uint64_t tile = s_tile[jj % 3];
+#ifdef HSORT_PHASE_TIMING
+    long long cw0 = clock64();
+#endif
     mbar_wait(&bar_g[jj & 1], (jj >> 1) & 1u);
+#ifdef HSORT_PHASE_TIMING
+    t_g += clock64() - cw0;
+#endif
     const uint64_t* gofs = s_gofs + (jj & 1) * kRadix;
     const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
     const uint64_t rem = n - tile * (uint64_t)TILE;
@@ -1217,6 +1294,9 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       for (int q = 0; q < ITEMS; ++q) {
         const uint64_t v = sb[tid + q * THREADS];
         const uint64_t g = gofs[(uint32_t)(v >> shift) & 255u];
+#if HSORT_FAKE == 3
+        if (v == 0x123456789ull)
+#endif
         dst[g + tid + q * THREADS] = inv ? from_key(v) : v;
       }
     } else {
@@ -1232,8 +1312,18 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     if (tile >= num_tiles) break;
     if (tid == 0) claim = atomicAdd(&tile_ctr[p], 1u);  // consumed at the end of the iteration
     for (int i = tid; i < CW * (kRadix + 1); i += THREADS) whist[i] = 0;
+#ifdef HSORT_PHASE_TIMING
+    long long ct0 = clock64();
+#endif
     mbar_wait(&bar_tma[cb], (j / 3) & 1u);
+#ifdef HSORT_PHASE_TIMING
+    t_t += clock64() - ct0;
+    ++n_t;
+#endif
     bar_compute<CT>();
+#ifdef HSORT_PHASE_TIMING
+    long long cc0 = clock64();
+#endif
 
     const uint64_t tbase = tile * (uint64_t)TILE;
     const uint64_t rem = n - tbase;
@@ -1279,54 +1369,75 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     }
     bar_compute<CT>();
     if (tid == 0) mbar_arrive(&bar_a[j & 1]);
+#ifdef HSORT_PHASE_TIMING
+    long long cr0 = clock64();
+    t_cnt += cr0 - cc0;
+#endif
 
-    // rank (as v2): the leader's atomic on the warp's base returns the group's first slot
+    // rank (as v2): the leader's atomic on the warp's base returns the group's first slot.
+    // Items are ranked in chunks of RC (fewer live peer masks -> fewer registers).
     uint32_t r[ITEMS];
-    {
-      uint32_t dd[ITEMS], peers[ITEMS];
+    constexpr int RC = HSORT_WS_RC > 0 && HSORT_WS_RC < ITEMS ? HSORT_WS_RC : ITEMS;
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
-        const bool valid = full || (wofs + i * 32 < tile_n);
-        dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+    for (int c0 = 0; c0 < ITEMS; c0 += RC) {
+      constexpr int RCX = RC;
+      uint32_t dd[RCX], peers[RCX];
+#pragma unroll
+      for (int i = 0; i < RCX; ++i) {
+        const bool valid = (c0 + i < ITEMS) && (full || (wofs + (c0 + i) * 32 < tile_n));
+        dd[i] = valid ? ((uint32_t)(k[c0 + i < ITEMS ? c0 + i : 0] >> shift) & 255u) : (uint32_t)kRadix;
       }
       if (use_match) {
 #pragma unroll
-        for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+        for (int i = 0; i < RCX; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
       } else {
 #pragma unroll
-        for (int i = 0; i < ITEMS; ++i) peers[i] = 0xffffffffu;
+        for (int i = 0; i < RCX; ++i) peers[i] = 0xffffffffu;
 #pragma unroll
         for (int b = 0; b < 8; ++b) {
 #pragma unroll
-          for (int i = 0; i < ITEMS; ++i) {
+          for (int i = 0; i < RCX; ++i) {
             const uint32_t bit = (dd[i] >> b) & 1u;
             peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
           }
         }
-        if (!full) {
+        if (!full || (c0 + RCX > ITEMS)) {
 #pragma unroll
-          for (int i = 0; i < ITEMS; ++i) {
+          for (int i = 0; i < RCX; ++i) {
             const uint32_t bit = (dd[i] >> 8) & 1u;
             peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
           }
         }
       }
+#if HSORT_FAKE == 2
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
+      for (int i = 0; i < RCX; ++i) peers[i] = 1u << lane;
+#endif
+      uint32_t rr[RCX];
+#pragma unroll
+      for (int i = 0; i < RCX; ++i) {
         const int leader = 31 - __clz(peers[i]);
-        r[i] = (lane == leader) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+        rr[i] = (lane == leader && dd[i] < kRadix) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
       }
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) {
+      for (int i = 0; i < RCX; ++i) {
         const int leader = 31 - __clz(peers[i]);
-        r[i] = __shfl_sync(0xffffffffu, r[i], leader) + __popc(peers[i] & lt);
+        const uint32_t v = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
+        if (c0 + i < ITEMS) r[c0 + i] = v;
       }
     }
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i)
       if (full || wofs + i * 32 < tile_n) sb[r[i]] = k[i];
 
+#ifdef HSORT_PHASE_TIMING
+    long long cw1 = clock64();
+    t_rank += cw1 - cr0;
+#endif
     if (j >= 1) write_out(j - 1);
+#ifdef HSORT_PHASE_TIMING
+    t_wo += clock64() - cw1;
+#endif
     bar_compute<CT>();  // stage (j-1)%3 fully read; whist free
     if (tid == 0) {
       const int nb = (int)((j + 2) % 3);
@@ -1338,6 +1449,18 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   // tell the look-back warp to stop, then drain the last tile
   if (tid == 0) mbar_arrive(&bar_a[j & 1]);
   if (j >= 1) write_out(j - 1);
+#ifdef HSORT_PHASE_TIMING
+  t_all = clock64() - c_start;
+  if (tid == 0) {
+    atomicAdd(&g_phase_dbg[210], t_g);
+    atomicAdd(&g_phase_dbg[211], t_t);
+    atomicAdd(&g_phase_dbg[212], t_all);
+    atomicAdd(&g_phase_dbg[213], n_t);
+    atomicAdd(&g_phase_dbg[218], t_rank);
+    atomicAdd(&g_phase_dbg[219], t_cnt);
+    atomicAdd(&g_phase_dbg[220], t_wo);
+  }
+#endif
   if (tid < kRadix)
     for (uint64_t rr = num_tiles + blockIdx.x; rr < lb_rows; rr += gridDim.x)
       lb32_next[rr * kRadix + tid] = 0;

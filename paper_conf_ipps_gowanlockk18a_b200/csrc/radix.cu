@@ -1071,6 +1071,9 @@ struct WsSmem {
 #ifndef HSORT_WS_RC
 #define HSORT_WS_RC 0  // ranking chunk (0 = all items at once)
 #endif
+#ifndef HSORT_WS_NMATCH
+#define HSORT_WS_NMATCH 5  // items ranked with match.any in high-entropy passes (best of 0..7)
+#endif
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
 #endif
@@ -1391,19 +1394,24 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
         for (int i = 0; i < RCX; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
       } else {
+        // high-entropy digits: an 8-ballot multisplit for most items; the first NM items use
+        // match.any, which runs on another pipe, so both proceed in parallel
+        constexpr int NM = HSORT_WS_NMATCH < RCX ? HSORT_WS_NMATCH : RCX;
 #pragma unroll
-        for (int i = 0; i < RCX; ++i) peers[i] = 0xffffffffu;
+        for (int i = 0; i < NM; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+#pragma unroll
+        for (int i = NM; i < RCX; ++i) peers[i] = 0xffffffffu;
 #pragma unroll
         for (int b = 0; b < 8; ++b) {
 #pragma unroll
-          for (int i = 0; i < RCX; ++i) {
+          for (int i = NM; i < RCX; ++i) {
             const uint32_t bit = (dd[i] >> b) & 1u;
             peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
           }
         }
         if (!full || (c0 + RCX > ITEMS)) {
 #pragma unroll
-          for (int i = 0; i < RCX; ++i) {
+          for (int i = NM; i < RCX; ++i) {
             const uint32_t bit = (dd[i] >> 8) & 1u;
             peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
           }

@@ -19,6 +19,7 @@
 
 #include <cstdint>
 #include <cstdlib>
+#include <type_traits>
 
 #include "internal.h"
 
@@ -1089,6 +1090,24 @@ __device__ __forceinline__ void st_relaxed_v4(uint32_t* p, const uint32_t* v) {
                : "memory");
 }
 
+__device__ __forceinline__ void st_global_u64(uint64_t addr, uint64_t v) {
+  asm volatile("st.global.u64 [%0], %1;" ::"l"(addr), "l"(v) : "memory");
+}
+// One bit of the ballot multisplit: peers &= (bit b of d) ? ballot(bit) : ~ballot(bit).
+__device__ __forceinline__ uint32_t peer_bit(uint32_t peers, uint32_t d, uint32_t bm) {
+  uint32_t out;
+  asm("{\n\t.reg .pred p;\n\t.reg .b32 B, t, m;\n\t"
+      "and.b32 t, %1, %2;\n\t"
+      "setp.ne.u32 p, t, 0;\n\t"
+      "vote.sync.ballot.b32 B, p, 0xffffffff;\n\t"
+      "selp.b32 m, 0, 0xffffffff, p;\n\t"
+      "xor.b32 B, B, m;\n\t"
+      "and.b32 %0, %3, B;\n\t}"
+      : "=r"(out)
+      : "r"(d), "r"(bm), "r"(peers));
+  return out;
+}
+
 template <int W>
 __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64_t tile, int lane,
                                           uint32_t* excl) {
@@ -1257,7 +1276,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       }
 #pragma unroll
       for (int q = 0; q < 8; ++q)
-        s_gofs[(j & 1) * kRadix + lane * 8 + q] = base[q] + excl[q] - (uint64_t)(cw[q] >> 16);
+        s_gofs[(j & 1) * kRadix + lane * 8 + q] =
+            (uint64_t)dst + 8ull * (base[q] + excl[q] - (uint64_t)(cw[q] >> 16));  // byte address (mod 2^64)
       __syncwarp();
       if (lane == 0) mbar_arrive(&bar_g[j & 1]);
     }
@@ -1279,7 +1299,10 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   unsigned long long t_g = 0, t_t = 0, t_all = 0, t_rank = 0, t_cnt = 0, t_wo = 0, n_t = 0;
   long long c_start = clock64();
 #endif
-  auto write_out = [&](uint32_t jj) {  // tile of iteration jj from its stage buffer
+  // write-out of the tile of iteration jj from its (digit-ordered) stage buffer.  s_gofs holds,
+  // per digit, the byte address of the tile-local position 0 of that digit's run in dst, so a key
+  // at stage position i goes to s_gofs[d] + 8 i (one 64-bit add, the q offset is an immediate).
+  auto write_out = [&](uint32_t jj) {
     const uint64_t tile = s_tile[jj % 3];
 #ifdef HSORT_PHASE_TIMING
     long long cw0 = clock64();
@@ -1292,65 +1315,51 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
     const uint64_t rem = n - tile * (uint64_t)TILE;
     const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
-    if (tile_n == TILE) {
+    auto wo_full = [&](auto inv_tag) {
+      constexpr bool INV = decltype(inv_tag)::value;
+      const uint64_t t8 = 8ull * (uint64_t)tid;
 #pragma unroll
       for (int q = 0; q < ITEMS; ++q) {
         const uint64_t v = sb[tid + q * THREADS];
-        const uint64_t g = gofs[(uint32_t)(v >> shift) & 255u];
+        const uint64_t ga = gofs[(uint32_t)(v >> shift) & 255u] + t8;
 #if HSORT_FAKE == 3
         if (v == 0x123456789ull)
 #endif
-        dst[g + tid + q * THREADS] = inv ? from_key(v) : v;
+        st_global_u64(ga + 8ull * (uint64_t)(q * THREADS), INV ? from_key(v) : v);
       }
+    };
+    if (tile_n == TILE) {
+      if (inv) wo_full(std::true_type{});
+      else wo_full(std::false_type{});
     } else {
       for (int i = tid; i < tile_n; i += THREADS) {
         const uint64_t v = sb[i];
-        dst[gofs[(uint32_t)(v >> shift) & 255u] + i] = inv ? from_key(v) : v;
+        st_global_u64(gofs[(uint32_t)(v >> shift) & 255u] + 8ull * (uint64_t)i, inv ? from_key(v) : v);
       }
     }
   };
-  while (true) {
-    const int cb = (int)(j % 3);
-    const uint64_t tile = s_tile[cb];
-    if (tile >= num_tiles) break;
-    if (tid == 0) claim = atomicAdd(&tile_ctr[p], 1u);  // consumed at the end of the iteration
-    for (int i = tid; i < CW * (kRadix + 1); i += THREADS) whist[i] = 0;
-#ifdef HSORT_PHASE_TIMING
-    long long ct0 = clock64();
-#endif
-    mbar_wait(&bar_tma[cb], (j / 3) & 1u);
-#ifdef HSORT_PHASE_TIMING
-    t_t += clock64() - ct0;
-    ++n_t;
-#endif
-    bar_compute<CT>();
-#ifdef HSORT_PHASE_TIMING
-    long long cc0 = clock64();
-#endif
-
+  // one tile: load from the stage, per-warp digit counts, tile aggregate + scan, warp ranking,
+  // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
+  auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, uint64_t* sb) {
+    constexpr bool FULL = decltype(full_tag)::value;
     const uint64_t tbase = tile * (uint64_t)TILE;
-    const uint64_t rem = n - tbase;
-    const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
-    const bool full = tile_n == TILE;
     const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
-    uint64_t* sb = stage + (size_t)cb * TILE;
     const int wofs = warp * 32 * ITEMS + lane;
     uint32_t* wh = whist + warp * (kRadix + 1);
-
     uint64_t k[ITEMS];
+    uint32_t dd[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int jj = wofs + i * 32;
       uint64_t v;
-      if (full) v = sb[jj];
+      if (FULL) v = sb[jj];
       else v = jj < bulk_n ? sb[jj] : (jj < tile_n ? src[tbase + jj] : 0);
       k[i] = IN_F64 ? to_key(v) : v;
+      const bool valid = FULL || jj < tile_n;
+      dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
     }
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-      const bool valid = full || (wofs + i * 32 < tile_n);
-      atomicAdd(&wh[valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix], 1u);
-    }
+    for (int i = 0; i < ITEMS; ++i) atomicAdd(&wh[dd[i]], 1u);
     bar_compute<CT>();
     uint32_t cnt = 0;
     if (tid < kRadix) {
@@ -1374,69 +1383,80 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     if (tid == 0) mbar_arrive(&bar_a[j & 1]);
 #ifdef HSORT_PHASE_TIMING
     long long cr0 = clock64();
-    t_cnt += cr0 - cc0;
 #endif
 
-    // rank (as v2): the leader's atomic on the warp's base returns the group's first slot.
-    // Items are ranked in chunks of RC (fewer live peer masks -> fewer registers).
-    uint32_t r[ITEMS];
-    constexpr int RC = HSORT_WS_RC > 0 && HSORT_WS_RC < ITEMS ? HSORT_WS_RC : ITEMS;
+    // rank: peers = lanes of this item with the same digit; the leader's atomic on the warp's
+    // base returns the group's first slot.
+    uint32_t peers[ITEMS];
+    if (use_match) {
 #pragma unroll
-    for (int c0 = 0; c0 < ITEMS; c0 += RC) {
-      constexpr int RCX = RC;
-      uint32_t dd[RCX], peers[RCX];
+      for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+    } else {
+      // high-entropy digits: an 8-ballot multisplit (4 instructions per bit: test -> predicate,
+      // vote, select, and) for most items; the first NM items use match.any, which runs on another
+      // pipe, so both proceed in parallel
+      constexpr int NM = HSORT_WS_NMATCH < ITEMS ? HSORT_WS_NMATCH : ITEMS;
 #pragma unroll
-      for (int i = 0; i < RCX; ++i) {
-        const bool valid = (c0 + i < ITEMS) && (full || (wofs + (c0 + i) * 32 < tile_n));
-        dd[i] = valid ? ((uint32_t)(k[c0 + i < ITEMS ? c0 + i : 0] >> shift) & 255u) : (uint32_t)kRadix;
-      }
-      if (use_match) {
+      for (int i = 0; i < NM; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
 #pragma unroll
-        for (int i = 0; i < RCX; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
-      } else {
-        // high-entropy digits: an 8-ballot multisplit for most items; the first NM items use
-        // match.any, which runs on another pipe, so both proceed in parallel
-        constexpr int NM = HSORT_WS_NMATCH < RCX ? HSORT_WS_NMATCH : RCX;
+      for (int i = NM; i < ITEMS; ++i) peers[i] = 0xffffffffu;
 #pragma unroll
-        for (int i = 0; i < NM; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+      for (int b = 0; b < (FULL ? 8 : 9); ++b) {
 #pragma unroll
-        for (int i = NM; i < RCX; ++i) peers[i] = 0xffffffffu;
-#pragma unroll
-        for (int b = 0; b < 8; ++b) {
-#pragma unroll
-          for (int i = NM; i < RCX; ++i) {
-            const uint32_t bit = (dd[i] >> b) & 1u;
-            peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
-          }
-        }
-        if (!full || (c0 + RCX > ITEMS)) {
-#pragma unroll
-          for (int i = NM; i < RCX; ++i) {
-            const uint32_t bit = (dd[i] >> 8) & 1u;
-            peers[i] &= __ballot_sync(0xffffffffu, bit) ^ (bit - 1u);
-          }
-        }
-      }
-#if HSORT_FAKE == 2
-#pragma unroll
-      for (int i = 0; i < RCX; ++i) peers[i] = 1u << lane;
-#endif
-      uint32_t rr[RCX];
-#pragma unroll
-      for (int i = 0; i < RCX; ++i) {
-        const int leader = 31 - __clz(peers[i]);
-        rr[i] = (lane == leader && dd[i] < kRadix) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
-      }
-#pragma unroll
-      for (int i = 0; i < RCX; ++i) {
-        const int leader = 31 - __clz(peers[i]);
-        const uint32_t v = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
-        if (c0 + i < ITEMS) r[c0 + i] = v;
+        for (int i = NM; i < ITEMS; ++i) peers[i] = peer_bit(peers[i], dd[i], 1u << b);
       }
     }
+#if HSORT_FAKE == 2
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i)
-      if (full || wofs + i * 32 < tile_n) sb[r[i]] = k[i];
+    for (int i = 0; i < ITEMS; ++i) peers[i] = 1u << lane;
+#endif
+    uint32_t rr[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      const int leader = 31 - __clz(peers[i]);
+      rr[i] = (lane == leader && (FULL || dd[i] < kRadix)) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+    }
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      const int leader = 31 - __clz(peers[i]);
+      const uint32_t r = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
+      if (FULL || dd[i] < kRadix) sb[r] = k[i];
+    }
+#ifdef HSORT_PHASE_TIMING
+    return cr0;
+#else
+    return 0ll;
+#endif
+  };
+  while (true) {
+    const int cb = (int)(j % 3);
+    const uint64_t tile = s_tile[cb];
+    if (tile >= num_tiles) break;
+    if (tid == 0) claim = atomicAdd(&tile_ctr[p], 1u);  // consumed at the end of the iteration
+    for (int i = tid; i < CW * (kRadix + 1); i += THREADS) whist[i] = 0;
+#ifdef HSORT_PHASE_TIMING
+    long long ct0 = clock64();
+#endif
+    mbar_wait(&bar_tma[cb], (j / 3) & 1u);
+#ifdef HSORT_PHASE_TIMING
+    t_t += clock64() - ct0;
+    ++n_t;
+#endif
+    bar_compute<CT>();
+#ifdef HSORT_PHASE_TIMING
+    long long cc0 = clock64();
+#endif
+    const uint64_t rem = n - tile * (uint64_t)TILE;
+    const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+    uint64_t* sb = stage + (size_t)cb * TILE;
+    long long cr0;
+    if (tile_n == TILE) cr0 = rank_tile(std::true_type{}, tile, tile_n, sb);
+    else cr0 = rank_tile(std::false_type{}, tile, tile_n, sb);
+#ifdef HSORT_PHASE_TIMING
+    t_cnt += cr0 - cc0;
+#else
+    (void)cr0;
+#endif
 
 #ifdef HSORT_PHASE_TIMING
     long long cw1 = clock64();

@@ -16,4 +16,5 @@ ps = []
 for _ in range(5):
     hs.hsort_sort_device(d_in, d_out); torch.cuda.synchronize()
     kt = hs.hsort_get_kernel_times(); ps += kt["passes"][:kt["num_active"]]
-print(json.dumps({"lib": sys.argv[1], "pass_ms": statistics.mean(ps), "per_pass": [round(x, 3) for x in kt["passes"]]}))
+ok = bool((d_out[1:] >= d_out[:-1]).all().item()) and torch.equal(torch.sort(d_in)[0], d_out)
+print(json.dumps({"lib": sys.argv[1], "pass_ms": statistics.mean(ps), "sort_ms": sum(kt["passes"][:kt["num_active"]]) + kt["hist"], "ok": ok, "per_pass": [round(x, 3) for x in kt["passes"]]}))

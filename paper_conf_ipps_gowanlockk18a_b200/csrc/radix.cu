@@ -1055,10 +1055,10 @@ struct WsSmem {
   static constexpr int CW = CT / 32;                                          // compute warps
   static constexpr size_t stage_off = 0;                                      // [3][TILE] u64
   static constexpr size_t whist_off = 3ull * TILE * 8;                        // [CW][257] u32
-  static constexpr size_t gofs_off = (whist_off + CW * (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [2][256] u64
-  static constexpr size_t cnt_off = gofs_off + 2 * kRadix * 8;                // [2][256] u32
-  static constexpr size_t bar_off = cnt_off + 2 * kRadix * 4;                 // [8] u64
-  static constexpr size_t swarp_off = bar_off + 8 * 8;                        // [8] u32 (+pad)
+  static constexpr size_t gofs_off = (whist_off + CW * (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [2][256] i32
+  static constexpr size_t cnt_off = gofs_off + 2 * kRadix * 4;                // [2][256] u32
+  static constexpr size_t bar_off = cnt_off + 2 * kRadix * 4;                 // [12] u64
+  static constexpr size_t swarp_off = bar_off + 12 * 8;                       // [8] u32 (+pad)
   static constexpr size_t tile_off = swarp_off + 64;                          // [4] u32
   static constexpr size_t bytes = tile_off + 16;
 };
@@ -1188,14 +1188,15 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* stage = (uint64_t*)(smem + L::stage_off);
   uint32_t* whist = (uint32_t*)(smem + L::whist_off);
-  uint64_t* s_gofs = (uint64_t*)(smem + L::gofs_off);
+  int32_t* s_gofs = (int32_t*)(smem + L::gofs_off);
   uint32_t* s_cnt = (uint32_t*)(smem + L::cnt_off);
   uint64_t* bars = (uint64_t*)(smem + L::bar_off);
   uint32_t* s_warp = (uint32_t*)(smem + L::swarp_off);
   uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
-  uint64_t* bar_tma = bars;      // [3]
-  uint64_t* bar_a = bars + 3;    // [2]
-  uint64_t* bar_g = bars + 5;    // [2]
+  uint64_t* bar_tma = bars;       // [3] stage s holds its tile (TMA done, or "no tile")
+  uint64_t* bar_a = bars + 3;     // [2] tile j counted, A published, counts in s_cnt
+  uint64_t* bar_g = bars + 5;     // [2] offsets of tile j in s_gofs
+  uint64_t* bar_free = bars + 7;  // [3] stage s read out by every compute warp
 
   const int na = plan->num_active;
   if (p >= na) return;
@@ -1210,30 +1211,39 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t num_tiles = (n + TILE - 1) / TILE;
 
-  auto issue = [&](uint64_t t, int b) {  // one thread: stage b <- tile t
-    const uint64_t base = t * (uint64_t)TILE;
-    const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
-    const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
-    mbar_arrive_expect_tx(&bar_tma[b], bytes);
-    if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bar_tma[b]);
+  // stage b <- tile t (one thread); a claim past the end completes the phase without a copy
+  auto issue = [&](uint32_t t, int b) {
+    s_tile[b] = t;
+    if (t < num_tiles) {
+      const uint64_t base = (uint64_t)t * TILE;
+      const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
+      const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
+      mbar_arrive_expect_tx(&bar_tma[b], bytes);
+      if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bar_tma[b]);
+    } else {
+      mbar_arrive(&bar_tma[b]);
+    }
   };
+  for (int i = tid; i < CW * (kRadix + 1); i += blockDim.x) whist[i] = 0;
   if (tid == 0) {
-    for (int b = 0; b < 3; ++b) mbar_init(&bar_tma[b], 1);
+    for (int b = 0; b < 3; ++b) {
+      mbar_init(&bar_tma[b], 1);
+      mbar_init(&bar_free[b], CW);
+    }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&bar_a[b], 1);
       mbar_init(&bar_g[b], 1);
     }
     mbar_fence_init();
-    for (int b = 0; b < 2; ++b) {
-      const uint32_t t = atomicAdd(&tile_ctr[p], 1u);
-      s_tile[b] = t;
-      if (t < num_tiles) issue(t, b);
-    }
+    for (int b = 0; b < 2; ++b) issue(atomicAdd(&tile_ctr[p], 1u), b);
   }
   __syncthreads();
 
   if (warp == CW) {
     // ================= look-back warp =================
+    // Per tile j: wait for its counts, look back, publish the inclusive prefix, hand the global
+    // offsets to the compute warps; then claim tile j+2 and issue its TMA into the stage that
+    // tile j-1 used, once every compute warp has written tile j-1 out.
     uint64_t base[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) base[q] = bin_base[digit * kRadix + lane * 8 + q];
@@ -1241,6 +1251,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     unsigned long long t_wait = 0, t_lb = 0, n_lb = 0;
 #endif
     for (uint32_t j = 0;; ++j) {
+      const uint64_t tile = s_tile[j % 3];  // written by this warp (or thread 0) before
+      if (tile >= num_tiles) break;
 #ifdef HSORT_PHASE_TIMING
       long long c0 = clock64();
 #endif
@@ -1249,8 +1261,6 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       long long c1 = clock64();
       t_wait += c1 - c0;
 #endif
-      const uint64_t tile = s_tile[j % 3];
-      if (tile >= num_tiles) break;
       uint32_t cw[8], excl[8];
 #pragma unroll
       for (int q = 0; q < 8; ++q) cw[q] = s_cnt[(j & 1) * kRadix + lane * 8 + q];
@@ -1274,12 +1284,18 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
         for (int q = 0; q < 8; ++q) excl[q] = 0;
       }
+      // offset of the digit's run relative to tile-local position 0 (n <= 2^30: fits in int32)
 #pragma unroll
       for (int q = 0; q < 8; ++q)
-        s_gofs[(j & 1) * kRadix + lane * 8 + q] =
-            (uint64_t)dst + 8ull * (base[q] + excl[q] - (uint64_t)(cw[q] >> 16));  // byte address (mod 2^64)
+        s_gofs[(j & 1) * kRadix + lane * 8 + q] = (int32_t)(base[q] + excl[q] - (uint64_t)(cw[q] >> 16));
       __syncwarp();
-      if (lane == 0) mbar_arrive(&bar_g[j & 1]);
+      if (lane == 0) {
+        mbar_arrive(&bar_g[j & 1]);
+        const int nb = (int)((j + 2) % 3);
+        if (j >= 1) mbar_wait(&bar_free[nb], ((j - 1) / 3) & 1u);
+        issue(atomicAdd(&tile_ctr[p], 1u), nb);
+      }
+      __syncwarp();
     }
 #ifdef HSORT_PHASE_TIMING
     if (lane == 0) {
@@ -1291,19 +1307,18 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     return;
   }
 
-  // ================= compute warps (256 threads) =================
+  // ================= compute warps =================
   const uint32_t lt = lanemask_lt();
-  uint32_t claim = 0;  // thread 0: tile j+2, claimed at the start of iteration j
   uint32_t j = 0;
+  uint64_t prev_tile = 0;
 #ifdef HSORT_PHASE_TIMING
   unsigned long long t_g = 0, t_t = 0, t_all = 0, t_rank = 0, t_cnt = 0, t_wo = 0, n_t = 0;
   long long c_start = clock64();
 #endif
-  // write-out of the tile of iteration jj from its (digit-ordered) stage buffer.  s_gofs holds,
-  // per digit, the byte address of the tile-local position 0 of that digit's run in dst, so a key
-  // at stage position i goes to s_gofs[d] + 8 i (one 64-bit add, the q offset is an immediate).
-  auto write_out = [&](uint32_t jj) {
-    const uint64_t tile = s_tile[jj % 3];
+  uint64_t* const dst_t = dst + tid;
+  // write-out of the tile of iteration jj from its (digit-ordered) stage buffer: a key at stage
+  // position i with digit d goes to dst[s_gofs[d] + i]; then this warp releases the stage
+  auto write_out = [&](uint32_t jj, uint64_t tile) {
 #ifdef HSORT_PHASE_TIMING
     long long cw0 = clock64();
 #endif
@@ -1311,21 +1326,20 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #ifdef HSORT_PHASE_TIMING
     t_g += clock64() - cw0;
 #endif
-    const uint64_t* gofs = s_gofs + (jj & 1) * kRadix;
+    const int32_t* gofs = s_gofs + (jj & 1) * kRadix;
     const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
     const uint64_t rem = n - tile * (uint64_t)TILE;
     const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
     auto wo_full = [&](auto inv_tag) {
       constexpr bool INV = decltype(inv_tag)::value;
-      const uint64_t t8 = 8ull * (uint64_t)tid;
 #pragma unroll
       for (int q = 0; q < ITEMS; ++q) {
         const uint64_t v = sb[tid + q * THREADS];
-        const uint64_t ga = gofs[(uint32_t)(v >> shift) & 255u] + t8;
+        uint64_t* a = dst_t + gofs[(uint32_t)(v >> shift) & 255u];
 #if HSORT_FAKE == 3
         if (v == 0x123456789ull)
 #endif
-        st_global_u64(ga + 8ull * (uint64_t)(q * THREADS), INV ? from_key(v) : v);
+        st_global_u64((uint64_t)(a + q * THREADS), INV ? from_key(v) : v);
       }
     };
     if (tile_n == TILE) {
@@ -1334,9 +1348,11 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     } else {
       for (int i = tid; i < tile_n; i += THREADS) {
         const uint64_t v = sb[i];
-        st_global_u64(gofs[(uint32_t)(v >> shift) & 255u] + 8ull * (uint64_t)i, inv ? from_key(v) : v);
+        st_global_u64((uint64_t)(dst + gofs[(uint32_t)(v >> shift) & 255u] + i), inv ? from_key(v) : v);
       }
     }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&bar_free[jj % 3]);
   };
   // one tile: load from the stage, per-warp digit counts, tile aggregate + scan, warp ranking,
   // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
@@ -1345,7 +1361,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     const uint64_t tbase = tile * (uint64_t)TILE;
     const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
     const int wofs = warp * 32 * ITEMS + lane;
-    uint32_t* wh = whist + warp * (kRadix + 1);
+    uint32_t* wh = whist + warp * (kRadix + 1);  // this warp's row: zero on entry
     uint64_t k[ITEMS];
     uint32_t dd[ITEMS];
 #pragma unroll
@@ -1422,6 +1438,9 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       const uint32_t r = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
       if (FULL || dd[i] < kRadix) sb[r] = k[i];
     }
+    // the row is private to this warp from here to the next tile's counts: clear it now
+    __syncwarp();
+    for (int i = lane; i < kRadix + 1; i += 32) wh[i] = 0;
 #ifdef HSORT_PHASE_TIMING
     return cr0;
 #else
@@ -1430,10 +1449,6 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   };
   while (true) {
     const int cb = (int)(j % 3);
-    const uint64_t tile = s_tile[cb];
-    if (tile >= num_tiles) break;
-    if (tid == 0) claim = atomicAdd(&tile_ctr[p], 1u);  // consumed at the end of the iteration
-    for (int i = tid; i < CW * (kRadix + 1); i += THREADS) whist[i] = 0;
 #ifdef HSORT_PHASE_TIMING
     long long ct0 = clock64();
 #endif
@@ -1442,7 +1457,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     t_t += clock64() - ct0;
     ++n_t;
 #endif
-    bar_compute<CT>();
+    const uint64_t tile = s_tile[cb];
+    if (tile >= num_tiles) break;
 #ifdef HSORT_PHASE_TIMING
     long long cc0 = clock64();
 #endif
@@ -1454,29 +1470,21 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     else cr0 = rank_tile(std::false_type{}, tile, tile_n, sb);
 #ifdef HSORT_PHASE_TIMING
     t_cnt += cr0 - cc0;
+    long long cw1 = clock64();
+    t_rank += cw1 - cr0;
 #else
     (void)cr0;
 #endif
-
-#ifdef HSORT_PHASE_TIMING
-    long long cw1 = clock64();
-    t_rank += cw1 - cr0;
-#endif
-    if (j >= 1) write_out(j - 1);
+    if (j >= 1) write_out(j - 1, prev_tile);
 #ifdef HSORT_PHASE_TIMING
     t_wo += clock64() - cw1;
 #endif
-    bar_compute<CT>();  // stage (j-1)%3 fully read; whist free
-    if (tid == 0) {
-      const int nb = (int)((j + 2) % 3);
-      s_tile[nb] = claim;
-      if (claim < num_tiles) issue(claim, nb);
-    }
+    prev_tile = tile;
     ++j;
   }
-  // tell the look-back warp to stop, then drain the last tile
-  if (tid == 0) mbar_arrive(&bar_a[j & 1]);
-  if (j >= 1) write_out(j - 1);
+  // drain the last tile (every warp's scatter of it must be complete: no tile barrier since)
+  bar_compute<CT>();
+  if (j >= 1) write_out(j - 1, prev_tile);
 #ifdef HSORT_PHASE_TIMING
   t_all = clock64() - c_start;
   if (tid == 0) {

@@ -12,7 +12,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 import paper_conf_ipps_gowanlockk18a_b200 as hs  # noqa: E402
 
-hs.LIB_PATH = os.path.join(ROOT, "paper_conf_ipps_gowanlockk18a_b200", "libhsort_timing.so")
+hs.LIB_PATH = os.environ.get("HSORT_LIB", os.path.join(ROOT, "paper_conf_ipps_gowanlockk18a_b200", "libhsort_timing.so"))
 import torch  # noqa: E402
 
 import hsort_inputs  # noqa: E402

@@ -1073,7 +1073,7 @@ struct WsSmem {
 #define HSORT_WS_RC 0  // ranking chunk (0 = all items at once)
 #endif
 #ifndef HSORT_WS_NMATCH
-#define HSORT_WS_NMATCH 5  // items ranked with match.any in high-entropy passes (best of 0..7)
+#define HSORT_WS_NMATCH 3  // items ranked with match.any in high-entropy passes (best of 0..7)
 #endif
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass

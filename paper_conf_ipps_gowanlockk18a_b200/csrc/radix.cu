@@ -1064,10 +1064,10 @@ struct WsSmem {
 };
 
 #ifndef HSORT_WS_CT
-#define HSORT_WS_CT 480  // compute threads of the warp-specialised pass (15 warps + 1 look-back warp)
+#define HSORT_WS_CT 576  // compute threads of the warp-specialised pass (18 warps + 1 look-back warp)
 #endif
 #ifndef HSORT_WS_ITEMS
-#define HSORT_WS_ITEMS 17  // keys per compute thread: 8160-key tiles, 3 stages = 191 KB, 1 CTA/SM
+#define HSORT_WS_ITEMS 15  // keys per compute thread: 8640-key tiles, 3 stages = 203 KB, 1 CTA/SM
 #endif
 #ifndef HSORT_WS_RC
 #define HSORT_WS_RC 0  // ranking chunk (0 = all items at once)

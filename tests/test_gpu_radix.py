@@ -8,7 +8,8 @@ import pytest
 
 pytestmark = pytest.mark.gpu
 
-SIZES = [1, 2, 3, 255, 4095, 4096, 4097, 3 * 4096 + 17, 100_003, (1 << 20) + 5]
+# 4096: tile of the register-load / v2 passes; 8640 = 576 x 15: tile of the default warp-specialised pass
+SIZES = [1, 2, 3, 255, 4095, 4096, 4097, 3 * 4096 + 17, 8639, 8640, 8641, 2 * 8640 + 4097, 100_003, (1 << 20) + 5]
 DISTS = ["uniform", "normal", "zipf_dup", "special", "random_bits", "salted", "sorted", "reverse",
          "all_equal", "few_distinct", "closed_form", "uniform_pm1"]
 
@@ -49,7 +50,7 @@ def test_histograms_misaligned(hs_gpu, oracle_mod):
 
 
 @pytest.mark.parametrize("digit", range(8))
-@pytest.mark.parametrize("n", [4096, 3 * 4096 + 17, 300_001])
+@pytest.mark.parametrize("n", [4096, 3 * 4096 + 17, 8640, 2 * 8640 + 5, 300_001])
 def test_single_pass_is_stable_counting_sort(hs_gpu, oracle_mod, digit, n):
     import torch
     rng = np.random.default_rng(digit * 31 + n)

@@ -812,7 +812,7 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
 
 // K1 v2: per-warp entropy probe picks, for each digit, either direct shared atomics (spread
 // digits) or the register run-length cache (low-entropy digits, e.g. the exponent byte).
-template <bool IN_F64, uint32_t MASK>
+template <bool IN_F64, uint32_t MASK, int SH = 0>
 __device__ __forceinline__ void hist2_key(uint64_t k, uint32_t* sh, uint32_t* cd, uint32_t* cc,
                                           uint32_t mask) {
   if (IN_F64) k = to_key(k);
@@ -825,17 +825,17 @@ __device__ __forceinline__ void hist2_key(uint64_t k, uint32_t* sh, uint32_t* cd
       if (d == cd[p]) {
         ++cc[p];
       } else {
-        if (cc[p]) atomicAdd(&sh[p * kRadix + cd[p]], cc[p]);
+        if (cc[p]) atomicAdd(&sh[(p * kRadix + cd[p]) << SH], cc[p]);
         cd[p] = d;
         cc[p] = 1;
       }
     } else {
-      atomicAdd(&sh[p * kRadix + d], 1u);
+      atomicAdd(&sh[(p * kRadix + d) << SH], 1u);
     }
   }
 }
 
-template <bool IN_F64, uint32_t MASK>
+template <bool IN_F64, uint32_t MASK, int SH = 0>
 __device__ __forceinline__ void hist2_loop(const uint64_t* base, uint64_t pairs, uint64_t i,
                                            uint64_t stride, uint32_t* sh, uint32_t* cd,
                                            uint32_t* cc, uint32_t mask) {
@@ -844,13 +844,13 @@ __device__ __forceinline__ void hist2_loop(const uint64_t* base, uint64_t pairs,
 #pragma unroll
     for (int u = 0; u < 4; ++u) ld_stream2(base + 2 * (i + u * stride), a[2 * u], a[2 * u + 1]);
 #pragma unroll
-    for (int u = 0; u < 8; ++u) hist2_key<IN_F64, MASK>(a[u], sh, cd, cc, mask);
+    for (int u = 0; u < 8; ++u) hist2_key<IN_F64, MASK, SH>(a[u], sh, cd, cc, mask);
   }
   for (; i < pairs; i += stride) {
     uint64_t a0, a1;
     ld_stream2(base + 2 * i, a0, a1);
-    hist2_key<IN_F64, MASK>(a0, sh, cd, cc, mask);
-    hist2_key<IN_F64, MASK>(a1, sh, cd, cc, mask);
+    hist2_key<IN_F64, MASK, SH>(a0, sh, cd, cc, mask);
+    hist2_key<IN_F64, MASK, SH>(a1, sh, cd, cc, mask);
   }
 }
 
@@ -896,6 +896,61 @@ __global__ void __launch_bounds__(kHistThreads) k_hist2(const uint64_t* __restri
   __syncthreads();
   for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
     uint32_t c = sh[j];
+    if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
+  }
+}
+
+// K1 v3: as v2, but the shared histograms are replicated 8 times, interleaved so that counter
+// (p, v) of copy c sits at word 8 (256 p + v) + c; lane L uses copy L & 7.  A warp's 32 atomics
+// then spread over 32 banks by (v & 3, L & 7): only the 4 lanes sharing a copy can conflict (v2:
+// all 32 lanes over 32 banks, ~3.7 wavefronts per atomic for random digits; K1 v2 was
+// shared-atomic-bound at 99% of the L1 data pipe).  64 KB per CTA.
+constexpr int kHist3Copies = 8;
+template <bool IN_F64>
+__global__ void __launch_bounds__(kHistThreads) k_hist3(const uint64_t* __restrict__ src, uint64_t n,
+                                                       uint64_t* __restrict__ hist) {
+  extern __shared__ uint32_t sh3[];  // [8 * 256][8]
+  for (int i = threadIdx.x; i < kDigits * kRadix * kHist3Copies; i += kHistThreads) sh3[i] = 0;
+  __syncthreads();
+  uint32_t* sh = sh3 + (threadIdx.x & (kHist3Copies - 1));
+  uint32_t cd[kDigits], cc[kDigits];
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p) { cd[p] = 0; cc[p] = 0; }
+  const uint64_t head = (((uintptr_t)src & 15) && n) ? 1 : 0;
+  const uint64_t* base = src + head;
+  const uint64_t m = n - head;
+  const uint64_t pairs = m / 2;
+  const uint64_t stride = (uint64_t)gridDim.x * kHistThreads;
+  const uint64_t i0 = (uint64_t)blockIdx.x * kHistThreads + threadIdx.x;
+  // entropy probe on this warp's first keys: <= 4 distinct values among 32 lanes -> run cache
+  uint32_t mask = 0;
+  {
+    uint64_t k = i0 < pairs ? base[2 * i0] : (m ? base[0] : 0);
+    if (IN_F64) k = to_key(k);
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int p = 0; p < kDigits; ++p) {
+      const uint32_t d = (uint32_t)(k >> (8 * p)) & 255u;
+      const uint32_t peers = __match_any_sync(0xffffffffu, d);
+      const uint32_t leaders = __ballot_sync(0xffffffffu, lane == 31 - __clz(peers));
+      if (__popc(leaders) <= 4) mask |= 1u << p;
+    }
+  }
+  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist2_key<IN_F64, 0xFFFFFFFFu, 3>(src[0], sh, cd, cc, 0xFF);
+  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else if (mask == 0u) hist2_loop<IN_F64, 0u, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else hist2_loop<IN_F64, 0xFFFFFFFFu, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
+  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == kHistThreads - 1)
+    hist2_key<IN_F64, 0xFFFFFFFFu, 3>(base[m - 1], sh, cd, cc, 0xFF);
+#pragma unroll
+  for (int p = 0; p < kDigits; ++p)
+    if (cc[p]) atomicAdd(&sh[(p * kRadix + cd[p]) << 3], cc[p]);
+  __syncthreads();
+  for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
+    const uint4 a = *(const uint4*)&sh3[j * kHist3Copies];
+    const uint4 b = *(const uint4*)&sh3[j * kHist3Copies + 4];
+    const uint32_t c = a.x + a.y + a.z + a.w + b.x + b.y + b.z + b.w;
     if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
   }
 }
@@ -951,7 +1006,7 @@ int pass_variant() {
   return v;
 }
 int hist_variant() {
-  static int v = env_int("HSORT_HIST_VARIANT", 1);
+  static int v = env_int("HSORT_HIST_VARIANT", 2);
   return v;
 }
 
@@ -960,14 +1015,27 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
   int dev = 0;
   cudaGetDevice(&dev);
   uint64_t want = (n / 2 + kHistThreads * 8 - 1) / (kHistThreads * 8);
-  uint64_t cap = (uint64_t)num_sms(dev) * 2;
+  static const int ctas = env_int("HSORT_HIST_CTAS", 2);  // CTAs per SM (experiments)
+  uint64_t cap = (uint64_t)num_sms(dev) * ctas;
   int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
   if (hist_variant() == 0) {
     if (in_f64) k_hist<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
     else k_hist<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
-  } else {
+  } else if (hist_variant() == 1) {
     if (in_f64) k_hist2<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
     else k_hist2<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
+  } else {
+    constexpr int smem = kDigits * kRadix * kHist3Copies * 4;
+    static bool attr[64] = {false};  // per device
+    if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+    if (!attr[dev]) {
+      cudaError_t e;
+      if ((e = cudaFuncSetAttribute(k_hist3<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(k_hist3<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      attr[dev] = true;
+    }
+    if (in_f64) k_hist3<true><<<grid, kHistThreads, smem, st>>>(in, n, hist);
+    else k_hist3<false><<<grid, kHistThreads, smem, st>>>(in, n, hist);
   }
   return cudaGetLastError();
 }

@@ -1380,7 +1380,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   uint32_t j = 0;
   uint64_t prev_tile = 0;
 #ifdef HSORT_PHASE_TIMING
-  unsigned long long t_g = 0, t_t = 0, t_all = 0, t_rank = 0, t_cnt = 0, t_wo = 0, n_t = 0;
+  unsigned long long t_g = 0, t_t = 0, t_all = 0, t_rank = 0, t_cnt = 0, t_wo = 0, n_t = 0, t_peers = 0;
   long long c_start = clock64();
 #endif
   uint64_t* const dst_t = dst + tid;
@@ -1494,6 +1494,15 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) peers[i] = 1u << lane;
 #endif
+#ifdef HSORT_PHASE_TIMING
+    {  // force the peers to be computed before the clock read
+      uint32_t x = 0;
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) x ^= peers[i];
+      asm volatile("" ::"r"(x));
+    }
+    t_peers += clock64() - cr0;
+#endif
     uint32_t rr[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -1563,6 +1572,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     atomicAdd(&g_phase_dbg[218], t_rank);
     atomicAdd(&g_phase_dbg[219], t_cnt);
     atomicAdd(&g_phase_dbg[220], t_wo);
+    atomicAdd(&g_phase_dbg[221], t_peers);
   }
 #endif
   if (tid < kRadix)

@@ -34,7 +34,7 @@ L.hsort_debug_phase_counters(buf, 256, 1)
 T = max(1, buf[213])
 res = {"tiles": T,
        "compute_total": buf[212] / T, "wait_tma": buf[211] / T, "count+publish": buf[219] / T,
-       "rank+scatter": buf[218] / T, "writeout(incl wait)": buf[220] / T, "wait_lookback": buf[210] / T,
+       "rank+scatter": buf[218] / T, "  of which peers": buf[221] / T, "writeout(incl wait)": buf[220] / T, "wait_lookback": buf[210] / T,
        "lb_idle": buf[214] / max(1, buf[217]), "lb_time": buf[215] / max(1, buf[217]),
        "lb_rounds": buf[216] / max(1, buf[217])}
 print(json.dumps({k: round(v, 1) if isinstance(v, float) else v for k, v in res.items()}))

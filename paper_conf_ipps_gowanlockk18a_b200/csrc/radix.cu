@@ -905,14 +905,22 @@ __global__ void __launch_bounds__(kHistThreads) k_hist2(const uint64_t* __restri
 // then spread over 32 banks by (v & 3, L & 7): only the 4 lanes sharing a copy can conflict (v2:
 // all 32 lanes over 32 banks, ~3.7 wavefronts per atomic for random digits; K1 v2 was
 // shared-atomic-bound at 99% of the L1 data pipe).  64 KB per CTA.
-constexpr int kHist3Copies = 8;
-template <bool IN_F64>
-__global__ void __launch_bounds__(kHistThreads) k_hist3(const uint64_t* __restrict__ src, uint64_t n,
+#ifndef HSORT_HIST_COPIES
+#define HSORT_HIST_COPIES 16  // 16 copies: a half-warp's 16 lanes use 16 distinct banks
+#endif
+#ifndef HSORT_HIST_THREADS
+#define HSORT_HIST_THREADS 1024  // 1 CTA (128 KB of copies) per SM
+#endif
+constexpr int kHist3Copies = HSORT_HIST_COPIES;
+constexpr int kHist3Threads = HSORT_HIST_THREADS;
+template <bool IN_F64, int THREADS, int COPIES>
+__global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ src, uint64_t n,
                                                        uint64_t* __restrict__ hist) {
-  extern __shared__ uint32_t sh3[];  // [8 * 256][8]
-  for (int i = threadIdx.x; i < kDigits * kRadix * kHist3Copies; i += kHistThreads) sh3[i] = 0;
+  constexpr int SHC = COPIES == 16 ? 4 : 3;
+  extern __shared__ uint32_t sh3[];  // [8 * 256][COPIES]
+  for (int i = threadIdx.x; i < kDigits * kRadix * COPIES; i += THREADS) sh3[i] = 0;
   __syncthreads();
-  uint32_t* sh = sh3 + (threadIdx.x & (kHist3Copies - 1));
+  uint32_t* sh = sh3 + (threadIdx.x & (COPIES - 1));
   uint32_t cd[kDigits], cc[kDigits];
 #pragma unroll
   for (int p = 0; p < kDigits; ++p) { cd[p] = 0; cc[p] = 0; }
@@ -920,8 +928,8 @@ __global__ void __launch_bounds__(kHistThreads) k_hist3(const uint64_t* __restri
   const uint64_t* base = src + head;
   const uint64_t m = n - head;
   const uint64_t pairs = m / 2;
-  const uint64_t stride = (uint64_t)gridDim.x * kHistThreads;
-  const uint64_t i0 = (uint64_t)blockIdx.x * kHistThreads + threadIdx.x;
+  const uint64_t stride = (uint64_t)gridDim.x * THREADS;
+  const uint64_t i0 = (uint64_t)blockIdx.x * THREADS + threadIdx.x;
   // entropy probe on this warp's first keys: <= 4 distinct values among 32 lanes -> run cache
   uint32_t mask = 0;
   {
@@ -936,21 +944,24 @@ __global__ void __launch_bounds__(kHistThreads) k_hist3(const uint64_t* __restri
       if (__popc(leaders) <= 4) mask |= 1u << p;
     }
   }
-  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist2_key<IN_F64, 0xFFFFFFFFu, 3>(src[0], sh, cd, cc, 0xFF);
-  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else if (mask == 0u) hist2_loop<IN_F64, 0u, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else hist2_loop<IN_F64, 0xFFFFFFFFu, 3>(base, pairs, i0, stride, sh, cd, cc, mask);
-  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == kHistThreads - 1)
-    hist2_key<IN_F64, 0xFFFFFFFFu, 3>(base[m - 1], sh, cd, cc, 0xFF);
+  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist2_key<IN_F64, 0xFFFFFFFFu, SHC>(src[0], sh, cd, cc, 0xFF);
+  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else if (mask == 0u) hist2_loop<IN_F64, 0u, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
+  else hist2_loop<IN_F64, 0xFFFFFFFFu, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
+  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == THREADS - 1)
+    hist2_key<IN_F64, 0xFFFFFFFFu, SHC>(base[m - 1], sh, cd, cc, 0xFF);
 #pragma unroll
   for (int p = 0; p < kDigits; ++p)
-    if (cc[p]) atomicAdd(&sh[(p * kRadix + cd[p]) << 3], cc[p]);
+    if (cc[p]) atomicAdd(&sh[(p * kRadix + cd[p]) << SHC], cc[p]);
   __syncthreads();
-  for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
-    const uint4 a = *(const uint4*)&sh3[j * kHist3Copies];
-    const uint4 b = *(const uint4*)&sh3[j * kHist3Copies + 4];
-    const uint32_t c = a.x + a.y + a.z + a.w + b.x + b.y + b.z + b.w;
+  for (int j = threadIdx.x; j < kDigits * kRadix; j += THREADS) {
+    uint32_t c = 0;
+#pragma unroll
+    for (int q = 0; q < COPIES; q += 4) {
+      const uint4 a = *(const uint4*)&sh3[j * COPIES + q];
+      c += a.x + a.y + a.z + a.w;
+    }
     if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
   }
 }
@@ -1026,16 +1037,23 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
     else k_hist2<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
   } else {
     constexpr int smem = kDigits * kRadix * kHist3Copies * 4;
-    static bool attr[64] = {false};  // per device
+    auto kt = k_hist3<true, kHist3Threads, kHist3Copies>;
+    auto kf = k_hist3<false, kHist3Threads, kHist3Copies>;
+    static int per_sm[64] = {0};  // resident CTAs per SM, per device
     if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
-    if (!attr[dev]) {
+    if (!per_sm[dev]) {
       cudaError_t e;
-      if ((e = cudaFuncSetAttribute(k_hist3<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-      if ((e = cudaFuncSetAttribute(k_hist3<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-      attr[dev] = true;
+      if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      int b = 0;
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, kHist3Threads, smem)) != cudaSuccess) return e;
+      per_sm[dev] = b > 0 ? b : 1;
     }
-    if (in_f64) k_hist3<true><<<grid, kHistThreads, smem, st>>>(in, n, hist);
-    else k_hist3<false><<<grid, kHistThreads, smem, st>>>(in, n, hist);
+    const uint64_t want3 = (n / 2 + kHist3Threads * 8 - 1) / (kHist3Threads * 8);
+    const uint64_t cap3 = (uint64_t)num_sms(dev) * per_sm[dev];
+    const int grid3 = (int)(want3 < 1 ? 1 : (want3 > cap3 ? cap3 : want3));
+    if (in_f64) kt<<<grid3, kHist3Threads, smem, st>>>(in, n, hist);
+    else kf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist);
   }
   return cudaGetLastError();
 }

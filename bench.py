@@ -137,6 +137,51 @@ def cpu_baseline_oracle(n_sample: int):
     }
 
 
+MERGE_K = 12  # runs of the RESIDENT auto plan at n = 2^30 (2^27-key batches + halving tail)
+
+
+def stage_rooflines(hs, torch, d_in, d_out, n, peak, hist_ms, pass_ms, stream):
+    """Per-stage HBM rooflines (outside the timed region): K1 and K3 from the timed steps, and the
+    GPU merge of k = MERGE_K device-resident sorted runs of the same workload (K4 co-ranks + K5
+    tile merge, the RESIDENT mode's merge), timed with CUDA events on the launching stream.
+    Algorithmic bytes: K1 8 B/key, K3 16 B/key per pass, K5 16 B/key (read once, write once).
+    Overwrites d_in/d_out."""
+    cuts = [n * j // MERGE_K for j in range(MERGE_K + 1)]
+    for j in range(MERGE_K):
+        hs.hsort_sort_device_keys(d_in[cuts[j]:cuts[j + 1]], d_out[cuts[j]:cuts[j + 1]], True, False,
+                                  stream)
+    tiles = (n + 4095) // 4096
+    d_ranks = torch.empty((tiles + 1) * MERGE_K, dtype=torch.int64, device=d_in.device)
+    hs.hsort_device_merge(d_out, cuts, d_in, True, stream)  # warm
+    tc, tm = [], []
+    for _ in range(3):
+        e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        e[0].record(stream)
+        hs.hsort_device_corank(d_out, cuts, 4096, tiles + 1, d_ranks, stream)
+        e[1].record(stream)
+        hs.hsort_device_merge(d_out, cuts, d_in, True, stream)
+        e[2].record(stream)
+        e[2].synchronize()
+        tc.append(e[0].elapsed_time(e[1]))
+        tm.append(e[1].elapsed_time(e[2]))
+    o = d_in[:: max(1, n // (1 << 20))]
+    assert bool((o[1:] >= o[:-1]).all()), "merged output not sorted"
+    k4, merge = statistics.median(tc), statistics.median(tm)
+    k5 = merge - k4
+
+    def hbm(ms, bpk, what):
+        gbs = bpk * n / (ms / 1e3) / 1e9
+        return {"kernel": what, "bound": "hbm", "ms": ms, "alg_bytes_per_key": bpk,
+                "achieved": gbs, "unit": "GB/s", "peak": peak, "frac": gbs / peak}
+
+    return {
+        "K1_hist": hbm(hist_ms, 8, "k_hist3 (8 digit histograms, one read)"),
+        "K3_onesweep": hbm(pass_ms, 16, "k_onesweep_ws (one 8-bit LSD pass)"),
+        "K5_merge": dict(hbm(k5, 16, f"k_merge_tile (k = {MERGE_K} resident runs, 2^30 keys)"),
+                         k4_corank_ms=k4, k4_k5_frac=16 * n / (merge / 1e3) / 1e9 / peak),
+    }
+
+
 def run_reference(args):
     ws, rank, _ = dist_env()
     if rank != 0:
@@ -294,6 +339,9 @@ def main():
     e2e_total = max_over_ranks(sum(e2e_t))
     e2e_value = ws * n * e2e_steps / e2e_total
 
+    stages = stage_rooflines(hs, torch, d_in, d_out, n, peak, statistics.mean(hist_ms), avg_pass_ms,
+                             stream)
+
     line = {
         "metric": METRIC,
         "value": value,
@@ -344,6 +392,7 @@ def main():
             "link_floor_ms": 1e3 * link_floor_s,
             "link_frac": link_floor_s / (e2e_total / e2e_steps),
         },
+        "stages": stages,
         "gpu_launches": args.steps * 11,
         "clocks": sampler.summary(),
         "init_s": t_init,

@@ -92,6 +92,8 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
   }
   // Find v = the key at merged position o: smallest v with count(<= v) > o.
   // Invariant: lo[c] = #(< L) in run, hi[c] = #(<= H) in run, count(<= H) > o, count(< L) <= o.
+  // (An interpolated two-pivot variant was measured: 1.9x slower at k = 12 -- the float64 key
+  // space is not uniform across binades, so the interpolation misses -- and removed.)
   uint64_t L = 0, H = ~0ull;
   while (true) {
     // tighten [L, H] to the keys still inside the windows
@@ -117,8 +119,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
       ub[c] = upper_bound(K + base[c], lo[c], hi[c], mid);
       s += ub[c];
     }
-    // elements <= mid overall = (elements < L, i.e. sum lo) + (in-window <= mid): the window
-    // search counts from index 0 because lo/hi are absolute.
+    // elements <= mid overall: the window searches count from index 0 (lo/hi are absolute)
     s = warp_sum(s);
     if (s > o) {
       H = mid;
@@ -169,21 +170,68 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
   }
 }
 
-// K5.  One CTA per output tile.  Dynamic smem: 2 x kMergeTile keys + bounds.
-constexpr int kMergeThreads = 256;
-constexpr int kMergeIPT = kMergeTile / kMergeThreads;
+// K5.  One CTA per output tile of kMergeTile keys, T threads x IPT = kMergeTile / T keys.
+//   1. slice table: len_j = r1[j] - r0[j], bnd = exclusive prefix of len (tile-local starts);
+//   2. gather: the k slices are copied into buf0 back to back.  Thread tid loads elements
+//      p = q T + tid (q < IPT, coalesced within a slice); the run of p, max{j : bnd[j] <= p}, only
+//      grows with q, so it is found once and then advanced; all IPT loads are issued before any
+//      store, so IPT HBM reads per thread are in flight;
+//   3. ceil(log2 k) pairwise merge-path rounds between buf0 and buf1: in round r the sequences are
+//      the groups of 2^r consecutive runs, so sequence m starts at bnd[min(m 2^r, k)] and no
+//      boundary table is rewritten; the pair holding a thread's first output in round r is
+//      j0 >> (r + 1), j0 the run holding it.  A thread owns outputs [IPT tid, IPT tid + IPT),
+//      finds its split (A wins ties: stable, runs in order) by a merge-path search, and merges with
+//      one shared-memory load per output;
+//   4. the merged tile is stored with coalesced stores (inverse key transform fused).
+// Shared-memory index of tile element p: one 8-byte pad after every IPT keys.  A thread's outputs
+// start IPT keys after its neighbour's; without the pad (IPT = 8: 64 B stride) 16 lanes of a warp
+// share one 8-byte bank pair on every merge-round load and store; with it the stride is IPT + 1
+// keys (odd) and a half-warp hits 16 distinct bank pairs.
+// Dynamic smem: 2 x (kMergeTile + kMergeTile / IPT) keys + k slice sources + (k + 1) bounds.
+__device__ __forceinline__ uint64_t ld_stream_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.global.cs.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
 
-__global__ void __launch_bounds__(kMergeThreads) k_merge_tile(
+template <int T>
+struct MergeCfg {
+  static constexpr int IPT = kMergeTile / T;
+  static_assert(T * IPT == kMergeTile, "merge tile");
+  static constexpr int BUF = kMergeTile + kMergeTile / IPT;
+  static __device__ __forceinline__ int pp(int p) { return p + p / IPT; }
+};
+
+// largest j >= a with bnd[j] <= p (j < cnt), starting from a valid j = a: two linear steps (the
+// usual distance when slices are longer than a thread's stride), then bisection of the rest
+__device__ __forceinline__ int advance_run(const uint32_t* bnd, int a, int cnt, uint32_t p) {
+#pragma unroll
+  for (int s = 0; s < 2; ++s) {
+    if (a + 1 >= cnt || bnd[a + 1] > p) return a;
+    ++a;
+  }
+  int z = cnt;
+  while (z - a > 1) {
+    const int m = (a + z) >> 1;
+    if (bnd[m] <= p) a = m;
+    else z = m;
+  }
+  return a;
+}
+
+template <int T>
+__global__ void __launch_bounds__(T) k_merge_tile(
     const uint64_t* __restrict__ keys, const uint64_t* __restrict__ off, int k, uint64_t total,
     const uint64_t* __restrict__ ranks, uint64_t rank_tile0, uint64_t tile_begin,
     uint64_t* __restrict__ out, uint64_t out_origin, int out_f64) {
+  using Cfg = MergeCfg<T>;
+  constexpr int IPT = Cfg::IPT;
   extern __shared__ __align__(16) unsigned char smem[];
-  uint64_t* bufA = (uint64_t*)smem;
-  uint64_t* bufB = bufA + kMergeTile;
-  uint32_t* bnd = (uint32_t*)(bufB + kMergeTile);   // k+1 sequence boundaries
-  uint32_t* bnd2 = bnd + (kMaxMergeRuns + 1);        // scratch for compaction
-  uint64_t* s_src = (uint64_t*)(bnd2 + (kMaxMergeRuns + 1));  // absolute start of slice j
-  __shared__ uint32_t s_carry;
+  uint64_t* buf0 = (uint64_t*)smem;
+  uint64_t* buf1 = buf0 + Cfg::BUF;
+  uint64_t* s_src = buf1 + Cfg::BUF;            // [k] absolute start of slice j (minus bnd[j])
+  uint32_t* bnd = (uint32_t*)(s_src + k);       // [k + 1] tile-local slice starts
+  __shared__ uint32_t s_w[T / 32];
 
   const uint64_t t = tile_begin + blockIdx.x;
   const uint64_t o0 = t * (uint64_t)kMergeTile;
@@ -191,115 +239,145 @@ __global__ void __launch_bounds__(kMergeThreads) k_merge_tile(
   const int L = (int)(o1 - o0);
   const uint64_t* r0 = ranks + (t - rank_tile0) * (uint64_t)k;
   const uint64_t* r1 = r0 + k;
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
 
-  // slice lengths -> exclusive prefix (sequential chunks of 256 runs)
-  if (tid == 0) s_carry = 0;
-  __syncthreads();
-  for (int c0 = 0; c0 < k; c0 += kMergeThreads) {
-    int j = c0 + tid;
+  // 1. slice table (chunks of T runs, block scan); s_src[j] - bnd[j] is stored, so element p of
+  //    slice j is keys[s_src[j] + p]
+  uint32_t carry = 0;
+  for (int c0 = 0; c0 < k; c0 += T) {
+    const int j = c0 + tid;
     uint32_t len = 0;
+    uint64_t srcj = 0;
     if (j < k) {
-      len = (uint32_t)(r1[j] - r0[j]);
-      s_src[j] = off[j] + r0[j];
+      const uint64_t a = r0[j];
+      len = (uint32_t)(r1[j] - a);
+      srcj = off[j] + a;
     }
-    // block inclusive scan of len
     uint32_t x = len;
-    const int lane = tid & 31, w = tid >> 5;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-      uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
       if (lane >= d) x += y;
     }
-    __shared__ uint32_t s_w[kMergeThreads / 32];
+    if (k <= 32) {  // one warp holds every run: no block scan
+      if (j < k) {
+        bnd[j] = x - len;
+        s_src[j] = srcj - (x - len);
+      }
+      break;
+    }
     if (lane == 31) s_w[w] = x;
     __syncthreads();
     uint32_t pre = 0, tot = 0;
-    for (int q = 0; q < kMergeThreads / 32; ++q) {
-      if (q < w) pre += s_w[q];
-      tot += s_w[q];
+#pragma unroll
+    for (int q = 0; q < T / 32; ++q) {
+      const uint32_t sq = s_w[q];
+      pre += q < w ? sq : 0;
+      tot += sq;
     }
-    if (j < k) bnd[j] = s_carry + pre + x - len;
-    __syncthreads();
-    if (tid == 0) s_carry += tot;
+    if (j < k) {
+      const uint32_t bj = carry + pre + x - len;
+      bnd[j] = bj;
+      s_src[j] = srcj - bj;
+    }
+    carry += tot;
     __syncthreads();
   }
   if (tid == 0) bnd[k] = (uint32_t)L;
   __syncthreads();
 
-  // gather slices into bufA (element p belongs to run j with bnd[j] <= p < bnd[j+1])
-  for (int p = tid; p < L; p += kMergeThreads) {
-    int a = 0, z = k;  // largest j with bnd[j] <= p
-    while (z - a > 1) {
-      int m = (a + z) >> 1;
-      if (bnd[m] <= (uint32_t)p) a = m;
-      else z = m;
-    }
-    // skip empty runs sharing the same boundary: a is the largest j with bnd[j] <= p, and since
-    // p < bnd[k] = L, run a is non-empty at p
-    bufA[p] = keys[s_src[a] + (p - bnd[a])];
-  }
-  __syncthreads();
+  uint64_t* o = out + (o0 - out_origin);
+  const uint64_t xmask = out_f64 ? ~0ull : 0ull;  // from_key applied iff out_f64
 
-  // pairwise merge-path tree in shared memory
-  int nseq = k;
-  uint64_t* srcb = bufA;
-  uint64_t* dstb = bufB;
-  while (nseq > 1) {
-    const int npair = (nseq + 1) >> 1;
-    const int p0 = tid * kMergeIPT;
-    if (p0 < L) {
-      int p = p0;
-      int pend = p0 + kMergeIPT < L ? p0 + kMergeIPT : L;
-      while (p < pend) {
-        // pair m: largest m with bnd[2m] <= p
-        int a = 0, z = npair;
-        while (z - a > 1) {
-          int m = (a + z) >> 1;
-          if (bnd[2 * m] <= (uint32_t)p) a = m;
-          else z = m;
-        }
-        const int m = a;
-        const int s0 = bnd[2 * m];
-        const int s1 = (2 * m + 1 <= nseq) ? bnd[2 * m + 1 < nseq ? 2 * m + 1 : nseq] : L;
-        const int s2 = bnd[2 * m + 2 <= nseq ? 2 * m + 2 : nseq];
-        const int lenA = s1 - s0, lenB = s2 - s1;
-        const uint64_t* A = srcb + s0;
-        const uint64_t* B = srcb + s1;
-        const int d = p - s0;
-        int lo = d > lenB ? d - lenB : 0, hi = d < lenA ? d : lenA;
-        while (lo < hi) {
-          int mid = (lo + hi) >> 1;
-          if (A[mid] <= B[d - 1 - mid]) lo = mid + 1;
-          else hi = mid;
-        }
-        int i = lo, jb = d - lo;
-        const int stop = pend < s2 ? pend : s2;
-        for (; p < stop; ++p) {
-          uint64_t x;
-          if (i < lenA && (jb >= lenB || A[i] <= B[jb])) x = A[i++];
-          else x = B[jb++];
-          dstb[p] = x;
-        }
+  // 2. gather (k == 1: straight copy)
+  uint64_t v[IPT];
+  {
+    int a = 0;
+#pragma unroll
+    for (int q = 0; q < IPT; ++q) {
+      const int p = q * T + tid;
+      if (p < L) {
+        if (k > 1) a = advance_run(bnd, a, k, (uint32_t)p);
+        v[q] = ld_stream_u64(keys + s_src[a] + p);
       }
     }
+  }
+  if (k == 1) {
+#pragma unroll
+    for (int q = 0; q < IPT; ++q) {
+      const int p = q * T + tid;
+      if (p < L) o[p] = out_f64 ? from_key(v[q]) : v[q];
+    }
+    return;
+  }
+#pragma unroll
+  for (int q = 0; q < IPT; ++q) {
+    const int p = q * T + tid;
+    if (p < L) buf0[Cfg::pp(p)] = v[q];
+  }
+  const int p0 = tid * IPT;
+  const int pend = p0 + IPT < L ? p0 + IPT : L;
+  const int j0 = p0 < L ? advance_run(bnd, 0, k, (uint32_t)p0) : 0;  // run holding output p0
+  __syncthreads();
+
+  // 3. pairwise merge-path rounds
+  uint64_t* src = buf0;
+  uint64_t* dst = buf1;
+  for (int sh = 0; (1 << sh) < k; ++sh) {
+    const int nseq = (k + (1 << sh) - 1) >> sh;
+    const int npair = (nseq + 1) >> 1;
+    const bool last = npair == 1;
+    int p = p0;
+    int m = j0 >> (sh + 1);
+    while (p < pend) {
+      // pair m holds p: bnd[start(m)] <= p < bnd[start(m + 1)]; advance past pairs ending <= p
+      const int q0 = (2 * m) << sh, q1 = (2 * m + 1) << sh, q2 = (2 * m + 2) << sh;
+      const int s0 = bnd[q0 < k ? q0 : k];
+      const int s1 = bnd[q1 < k ? q1 : k];
+      const int s2 = bnd[q2 < k ? q2 : k];
+      if (s2 <= p) {
+        ++m;
+        continue;
+      }
+      const int lenA = s1 - s0, lenB = s2 - s1;
+      const int d = p - s0;
+      int lo = d > lenB ? d - lenB : 0, hi = d < lenA ? d : lenA;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (src[Cfg::pp(s0 + mid)] <= src[Cfg::pp(s1 + d - 1 - mid)]) lo = mid + 1;
+        else hi = mid;
+      }
+      int i = lo, jb = d - lo;
+      const int stop = pend < s2 ? pend : s2;
+      // heads (indices clamped into the pair; an exhausted side is never taken)
+      uint64_t a = src[Cfg::pp(s0 + i < s2 - 1 ? s0 + i : s2 - 1)];
+      uint64_t b = src[Cfg::pp(s1 + jb < s2 - 1 ? s1 + jb : s2 - 1)];
+      for (; p < stop; ++p) {
+        const bool ta = jb >= lenB || (i < lenA && a <= b);
+        const uint64_t x = ta ? a : b;
+        dst[Cfg::pp(p)] =
+            last ? (x ^ (xmask & ((uint64_t)((int64_t)(~x) >> 63) | 0x8000000000000000ull))) : x;
+        i += ta;
+        jb += !ta;
+        int nx = ta ? s0 + i : s1 + jb;
+        nx = nx < s2 - 1 ? nx : s2 - 1;
+        const uint64_t y = src[Cfg::pp(nx)];
+        a = ta ? y : a;
+        b = ta ? b : y;
+      }
+      ++m;
+    }
     __syncthreads();
-    // new boundaries: bnd'[m] = bnd[2m], bnd'[npair] = L
-    for (int m = tid; m <= npair; m += kMergeThreads) bnd2[m] = (m < npair) ? bnd[2 * m] : (uint32_t)L;
-    __syncthreads();
-    for (int m = tid; m <= npair; m += kMergeThreads) bnd[m] = bnd2[m];
-    __syncthreads();
-    nseq = npair;
-    uint64_t* tsw = srcb;
-    srcb = dstb;
-    dstb = tsw;
+    uint64_t* tsw = src;
+    src = dst;
+    dst = tsw;
   }
 
-  uint64_t* o = out + (o0 - out_origin);
-  if (out_f64) {
-    for (int p = tid; p < L; p += kMergeThreads) o[p] = from_key(srcb[p]);
-  } else {
-    for (int p = tid; p < L; p += kMergeThreads) o[p] = srcb[p];
+  // 4. coalesced store of the tile (src holds the merged, transformed keys)
+#pragma unroll
+  for (int q = 0; q < IPT; ++q) {
+    const int p = q * T + tid;
+    if (p < L) __stcs(o + p, src[Cfg::pp(p)]);
   }
 }
 
@@ -312,9 +390,14 @@ __global__ void k_upper_bounds(const uint64_t* __restrict__ keys, uint64_t n,
   if (i < m) out[i] = upper_bound(keys, 0, n, values[i]);
 }
 
-constexpr size_t merge_smem_bytes() {
-  return 2 * kMergeTile * sizeof(uint64_t) + 2 * (kMaxMergeRuns + 1) * sizeof(uint32_t) +
-         kMaxMergeRuns * sizeof(uint64_t);
+#ifndef HSORT_MERGE_THREADS
+#define HSORT_MERGE_THREADS 256  // 256 x 16 keys: 12.9 ms vs 14.8 ms (512 x 8) per 2^30 keys, k = 12
+#endif
+constexpr int kMergeThreads = HSORT_MERGE_THREADS;
+
+size_t merge_smem_bytes(int k) {
+  return 2 * MergeCfg<kMergeThreads>::BUF * sizeof(uint64_t) + (size_t)k * sizeof(uint64_t) +
+         ((size_t)k + 1) * sizeof(uint32_t);
 }
 
 }  // namespace
@@ -349,14 +432,14 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint
   static bool attr_set[64] = {false};
   int dev = 0;
   cudaGetDevice(&dev);
-  const size_t smem = merge_smem_bytes();
+  const size_t smem = merge_smem_bytes(k);
   if (dev >= 0 && dev < 64 && !attr_set[dev]) {
-    cudaError_t e = cudaFuncSetAttribute(k_merge_tile, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_merge_tile<kMergeThreads>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)merge_smem_bytes(kMaxMergeRuns));
     if (e != cudaSuccess) return e;
     attr_set[dev] = true;
   }
-  k_merge_tile<<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, d_off, k, total, ranks,
+  k_merge_tile<kMergeThreads><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, d_off, k, total, ranks,
                                                                   rank_tile0, tile_begin, out,
                                                                   out_origin, out_f64 ? 1 : 0);
   return cudaGetLastError();

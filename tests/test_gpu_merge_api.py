@@ -50,6 +50,21 @@ def test_device_merge_matches_oracle(hs_gpu, oracle_mod, k, hi):
     assert np.array_equal(d_out.cpu().numpy(), oracle_mod.merge_runs(runs))
 
 
+@pytest.mark.parametrize("k", [31, 32, 33, 511, 512, 513])
+@pytest.mark.parametrize("misaligned", [False, True])
+def test_device_merge_slice_table_paths(hs_gpu, oracle_mod, k, misaligned):
+    """K5 slice-table scan: one warp (k <= 32) vs block scan in chunks of 512 runs; 16-byte
+    vector store vs the scalar store of a misaligned output; tiles with many empty slices."""
+    import torch
+    rng = np.random.default_rng(k + 1000 * misaligned)
+    runs, keys, off = _runs(rng, k, 9000 if k <= 33 else 60)
+    d_keys = torch.from_numpy(keys).cuda()
+    d_buf = torch.zeros(keys.size + 1, dtype=torch.uint64, device="cuda")
+    d_out = d_buf[1:] if misaligned else d_buf[:-1]
+    hs_gpu.hsort_device_merge(d_keys, off, d_out, False)
+    assert np.array_equal(d_out.cpu().numpy(), oracle_mod.merge_runs(runs))
+
+
 def test_device_merge_inverse_transform(hs_gpu, oracle_mod, inputs_mod):
     import torch
     A = inputs_mod.generate("special", 200_000, seed=12)

@@ -146,6 +146,25 @@ def stage_rooflines(hs, torch, d_in, d_out, n, peak, hist_ms, pass_ms, stream):
     tile merge, the RESIDENT mode's merge), timed with CUDA events on the launching stream.
     Algorithmic bytes: K1 8 B/key, K3 16 B/key per pass, K5 16 B/key (read once, write once).
     Overwrites d_in/d_out."""
+    # key/value GPUSort (S§8(f) #3): 2^30 (key, index) pairs, 32 B/pair per pass
+    vals = torch.arange(n, dtype=torch.int64, device=d_in.device)
+    kout, vout = torch.empty_like(d_in), torch.empty_like(vals)
+    hs.hsort_sort_device_pairs(d_in, vals, kout, vout, True, stream)  # warm
+    kv_ms, kv_pass = [], []
+    for _ in range(3):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        hs.hsort_sort_device_pairs(d_in, vals, kout, vout, True, stream)
+        e1.record(stream)
+        e1.synchronize()
+        kv_ms.append(e0.elapsed_time(e1))
+        kt = hs.hsort_get_kernel_times()
+        kv_pass.extend(kt["passes"][:kt["num_active"]])
+    assert bool((kout[1:] >= kout[:-1]).all()), "pairs output not sorted"
+    del vals, kout, vout
+    kv = statistics.median(kv_ms)
+    kv_pass_ms = statistics.mean(kv_pass)
+
     cuts = [n * j // MERGE_K for j in range(MERGE_K + 1)]
     for j in range(MERGE_K):
         hs.hsort_sort_device_keys(d_in[cuts[j]:cuts[j + 1]], d_out[cuts[j]:cuts[j + 1]], True, False,
@@ -177,6 +196,8 @@ def stage_rooflines(hs, torch, d_in, d_out, n, peak, hist_ms, pass_ms, stream):
     return {
         "K1_hist": hbm(hist_ms, 8, "k_hist3 (8 digit histograms, one read)"),
         "K3_onesweep": hbm(pass_ms, 16, "k_onesweep_ws (one 8-bit LSD pass)"),
+        "K3_kv_pass": dict(hbm(kv_pass_ms, 32, "k_onesweep_ws<KV> (one LSD pass over key/value pairs)"),
+                           sort_ms=kv, pairs_per_s=n / (kv / 1e3)),
         "K5_merge": dict(hbm(k5, 16, f"k_merge_tile (k = {MERGE_K} resident runs, 2^30 keys)"),
                          k4_corank_ms=k4, k4_k5_frac=16 * n / (merge / 1e3) / 1e9 / peak),
     }

@@ -135,6 +135,21 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
                    int n_gpus);
 
 /* ---------------------------------------------------------------------------------------------
+ * Key/value sort (the [5] workload of 64-bit keys with 64-bit values,
+ * P:743-761).  B/VB = the pairs (A[i], V[i]) ordered by A under IEEE totalOrder, STABLY: pairs
+ * with equal keys keep their input order, so the result is unique (V = 0..n-1 gives the stable
+ * argsort).  Values are opaque 64-bit payloads, never transformed.  One GPU, one batch (BLINE):
+ * 1 <= n <= 2^30 pairs and 32 B/pair + 0.5 B/pair of HBM; larger n -> HSORT_ERR_INVALID (a merge
+ * that carries values is not built).  B == A and VB == V allowed together or separately; any
+ * other overlap among A, V, B, VB -> HSORT_ERR_INVALID.  Synchronous; retains no pointer.
+ * ------------------------------------------------------------------------------------------- */
+int hsort_sort_pairs(const double* A_host, const uint64_t* V_host, double* B_host, uint64_t* VB_host,
+                     uint64_t n);
+/* Same with raw uint64 keys (ascending unsigned). */
+int hsort_sort_pairs_u64(const uint64_t* A_host, const uint64_t* V_host, uint64_t* B_host,
+                         uint64_t* VB_host, uint64_t n);
+
+/* ---------------------------------------------------------------------------------------------
  * Options, statistics, errors
  *   keys: "n_s" (batch slots per GPU, default 2), "p_s" (pinned staging chunk bytes),
  *         "n_ring" (pinned slots per direction), "memcpy_threads" (PARMEMCPY threads; 1 = serial
@@ -184,6 +199,15 @@ int hsort_sort_device(const double* d_in, double* d_out, uint64_t n, void* strea
  * float64 bits (inverse transform fused into the last pass). */
 int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, int in_f64,
                            int out_f64, void* stream);
+
+/* Key/value GPUSort, device -> device (current device, stream-ordered): (d_keys_out,
+ * d_vals_out) = the pairs stably sorted by key (float64 totalOrder bits in and out if keys_f64,
+ * else ascending uint64).  n <= 2^30; all four buffers 16-byte aligned (TMA tile loads); keys in
+ * place iff values in place.  Same K1/K2 as hsort_sort_device, then the key/value onesweep pass
+ * (4032-pair tiles) per active digit: 32 HBM bytes per pair per pass. */
+int hsort_sort_device_pairs(const uint64_t* d_keys_in, const uint64_t* d_vals_in,
+                            uint64_t* d_keys_out, uint64_t* d_vals_out, uint64_t n, int keys_f64,
+                            void* stream);
 
 /* K1 alone: d_hist[8*256] (uint64, device) = per-digit histograms of the keys (digit d =
  * bits [8d, 8d+8) of key(x) if in_f64 else of the raw uint64).  Synchronous. */

@@ -55,6 +55,8 @@ def _load():
                 "oracle_pipemerge_count": ([_U64, ctypes.c_int], _U64),
                 "oracle_is_sorted_f64": ([_P, _U64], ctypes.c_int),
                 "oracle_multiset_hash": ([_P, _U64, _P], None),
+                "oracle_sort_pairs_f64": ([_P, _P, _P, _P, _U64], None),
+                "oracle_sort_pairs_u64": ([_P, _P, _P, _P, _U64], None),
             }
             for name, (args, res) in sig.items():
                 f = getattr(lib, name)
@@ -130,6 +132,27 @@ def _pack_runs(runs):
         off[j + 1] = off[j] + r.size
     keys = np.concatenate(runs) if runs else np.zeros(0, dtype=np.uint64)
     return _c(keys, np.uint64), off
+
+
+def sort_pairs_f64(A, V):
+    """(B, VB): the pairs stably sorted by A under IEEE totalOrder (oracle.cpp)."""
+    A = np.ascontiguousarray(A, dtype=np.float64)
+    V = np.ascontiguousarray(V, dtype=np.uint64)
+    assert A.size == V.size
+    B = np.empty_like(A)
+    VB = np.empty_like(V)
+    _load().oracle_sort_pairs_f64(A.ctypes.data, V.ctypes.data, B.ctypes.data, VB.ctypes.data, A.size)
+    return B, VB
+
+
+def sort_pairs_u64(A, V):
+    A = np.ascontiguousarray(A, dtype=np.uint64)
+    V = np.ascontiguousarray(V, dtype=np.uint64)
+    assert A.size == V.size
+    B = np.empty_like(A)
+    VB = np.empty_like(V)
+    _load().oracle_sort_pairs_u64(A.ctypes.data, V.ctypes.data, B.ctypes.data, VB.ctypes.data, A.size)
+    return B, VB
 
 
 def merge_runs(runs) -> np.ndarray:

@@ -23,6 +23,10 @@
 //   oracle_corank              pinned: co-rank invariants (sum, boundary) + brute force.
 //   oracle_pipemerge_count     pinned: Fig. 3 worked example (tests/golden/fig3_pipemerge.txt).
 //   oracle_is_sorted_f64 / oracle_multiset_hash: pinned by planted faults.
+//   oracle_sort_pairs_f64/_u64 pinned: keys = oracle_sort; values = numpy stable argsort on
+//                              NaN/-0-free keys; brute force over all permutations of small
+//                              duplicate-heavy inputs vs a Python insertion sort (stable by
+//                              construction) under the IEEE clause predicate; pair multiset.
 #include <algorithm>
 #include <compare>
 #include <cstdint>
@@ -53,6 +57,39 @@ int oracle_total_order_cmp(double a, double b) {
 void oracle_sort_f64(const double* A, double* B, uint64_t n) {
   if (B != A) std::memcpy(B, A, n * sizeof(double));
   std::sort(B, B + n, total_less);
+}
+
+// ---------------------------------------------------------------------------------------------
+// Key/value sort (the [5] workload of 64-bit keys with values):
+// the pairs (A[i], V[i]) ordered by A under totalOrder, STABLY (equal keys keep input order), so
+// the result is unique.  Definition: std::stable_sort of the index sequence 0..n-1 by A[i], then
+// gather.
+void oracle_sort_pairs_f64(const double* A, const uint64_t* V, double* B, uint64_t* VB, uint64_t n) {
+  std::vector<uint64_t> idx(n);
+  for (uint64_t i = 0; i < n; ++i) idx[i] = i;
+  std::stable_sort(idx.begin(), idx.end(), [&](uint64_t x, uint64_t y) { return total_less(A[x], A[y]); });
+  std::vector<double> b(n);
+  std::vector<uint64_t> vb(n);
+  for (uint64_t i = 0; i < n; ++i) {
+    b[i] = A[idx[i]];
+    vb[i] = V[idx[i]];
+  }
+  std::memcpy(B, b.data(), n * sizeof(double));
+  std::memcpy(VB, vb.data(), n * sizeof(uint64_t));
+}
+
+// Same on raw uint64 keys, ascending unsigned.
+void oracle_sort_pairs_u64(const uint64_t* A, const uint64_t* V, uint64_t* B, uint64_t* VB, uint64_t n) {
+  std::vector<uint64_t> idx(n);
+  for (uint64_t i = 0; i < n; ++i) idx[i] = i;
+  std::stable_sort(idx.begin(), idx.end(), [&](uint64_t x, uint64_t y) { return A[x] < A[y]; });
+  std::vector<uint64_t> b(n), vb(n);
+  for (uint64_t i = 0; i < n; ++i) {
+    b[i] = A[idx[i]];
+    vb[i] = V[idx[i]];
+  }
+  std::memcpy(B, b.data(), n * sizeof(uint64_t));
+  std::memcpy(VB, vb.data(), n * sizeof(uint64_t));
 }
 
 // ---------------------------------------------------------------------------------------------

@@ -75,6 +75,9 @@ SIGNATURES = {
     "hsort_finalize": ([], _I),
     "hsort_sort": ([_P, _P, _U64, _U64, _I], _I),
     "hsort_sort_u64": ([_P, _P, _U64, _U64, _I], _I),
+    "hsort_sort_pairs": ([_P, _P, _P, _P, _U64], _I),
+    "hsort_sort_pairs_u64": ([_P, _P, _P, _P, _U64], _I),
+    "hsort_sort_device_pairs": ([_P, _P, _P, _P, _U64, _I, _P], _I),
     "hsort_set_option": ([ctypes.c_char_p, ctypes.c_int64], _I),
     "hsort_get_option": ([ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64)], _I),
     "hsort_get_stats": ([ctypes.POINTER(hsort_stats)], _I),
@@ -213,6 +216,38 @@ def hsort_sort_u64(A, B=None, batch_elems: int = 0, n_gpus: int = 0):
     return B
 
 
+def hsort_sort_pairs(A, V, B=None, VB=None):
+    """(B, VB) = the pairs (A[i], V[i]) stably sorted by A under IEEE totalOrder (host -> host,
+    one GPU, n <= 2^30).  A float64, V uint64 payloads (e.g. np.arange(n): stable argsort)."""
+    a, n = _host_ptr(A, np.float64)
+    v, nv = _host_ptr(V, np.uint64)
+    if B is None:
+        B = np.empty(n, dtype=np.float64)
+    if VB is None:
+        VB = np.empty(n, dtype=np.uint64)
+    b, nb = _host_ptr(B, np.float64)
+    vb, nvb = _host_ptr(VB, np.uint64)
+    if not (n == nv == nb == nvb):
+        raise ValueError("A, V, B, VB must have the same length")
+    _check(lib().hsort_sort_pairs(a, v, b, vb, n))
+    return B, VB
+
+
+def hsort_sort_pairs_u64(A, V, B=None, VB=None):
+    a, n = _host_ptr(A, np.uint64)
+    v, nv = _host_ptr(V, np.uint64)
+    if B is None:
+        B = np.empty(n, dtype=np.uint64)
+    if VB is None:
+        VB = np.empty(n, dtype=np.uint64)
+    b, nb = _host_ptr(B, np.uint64)
+    vb, nvb = _host_ptr(VB, np.uint64)
+    if not (n == nv == nb == nvb):
+        raise ValueError("A, V, B, VB must have the same length")
+    _check(lib().hsort_sort_pairs_u64(a, v, b, vb, n))
+    return B, VB
+
+
 def hsort_set_option(key: str, value: int) -> None:
     _check(lib().hsort_set_option(key.encode(), int(value)))
 
@@ -252,6 +287,17 @@ def hsort_sort_device_keys(d_in, d_out, in_f64: bool, out_f64: bool, stream=None
     n = d_in.numel()
     _check(lib().hsort_sort_device_keys(_dev_ptr(d_in), _dev_ptr(d_out), n, int(in_f64),
                                         int(out_f64), _stream_ptr(stream)))
+
+
+def hsort_sort_device_pairs(d_keys_in, d_vals_in, d_keys_out, d_vals_out, keys_f64: bool = True,
+                            stream=None) -> None:
+    """(d_keys_out, d_vals_out) = pairs stably sorted by key; 8-byte CUDA tensors, stream-ordered."""
+    n = d_keys_in.numel()
+    if not (d_vals_in.numel() == d_keys_out.numel() == d_vals_out.numel() == n):
+        raise ValueError("length mismatch")
+    _check(lib().hsort_sort_device_pairs(_dev_ptr(d_keys_in), _dev_ptr(d_vals_in),
+                                         _dev_ptr(d_keys_out), _dev_ptr(d_vals_out), n,
+                                         int(keys_f64), _stream_ptr(stream)))
 
 
 def hsort_device_histograms(d_keys, in_f64: bool, d_hist, stream=None) -> None:

@@ -126,6 +126,7 @@ struct GpuCtx {
   cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
   RadixScratch rs;
   DevBuf runs, alt, mout, min, ranks, off;
+  DevBuf vruns, valt;  // key/value sorts: values and their ping-pong scratch
   std::vector<char*> ring_in, ring_out;
   uint64_t ring_bytes = 0;
   std::vector<cudaEvent_t> ev_in, ev_out;
@@ -999,6 +1000,8 @@ void ctx_destroy(GpuCtx& g) {
   for (auto e : g.ev_out) cudaEventDestroy(e);
   g.runs.release();
   g.alt.release();
+  g.vruns.release();
+  g.valt.release();
   g.mout.release();
   g.min.release();
   g.ranks.release();
@@ -1108,6 +1111,104 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
   });
 }
 
+// Key/value host->host sort (S§8(f) #3, the [5] workload of P:743-761): BLINE on one GPU --
+// HtoD of keys and values, the key/value GPUSort in place, DtoH of both.  Out-of-core pairs (a
+// merge that carries values) are not built: n must fit one GPU (32 B/pair + look-back).
+int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint64_t n, bool f64) {
+  int rc = check_ready();
+  if (rc) return rc;
+  BusyGuard busy;
+  if (!busy.ok) {
+    g_err = "hsort_sort already running";
+    return HSORT_ERR_BUSY;
+  }
+  if (n == 0) {
+    S().last = hsort_stats{};
+    return HSORT_OK;
+  }
+  if (!A || !B || !V || !VB) {
+    g_err = "null A, V, B or VB with n > 0";
+    return HSORT_ERR_INVALID;
+  }
+  if ((((uintptr_t)A | (uintptr_t)B | (uintptr_t)V | (uintptr_t)VB) & 7) != 0) {
+    g_err = "A, V, B, VB must be 8-byte aligned";
+    return HSORT_ERR_INVALID;
+  }
+  const uint64_t bytes = n * 8;
+  auto overlap = [&](const void* x, const void* y) {
+    const uintptr_t a0 = (uintptr_t)x, b0 = (uintptr_t)y;
+    return x != y && a0 < b0 + bytes && b0 < a0 + bytes;
+  };
+  if (overlap(A, B) || overlap(V, VB) || overlap(A, V) || overlap(A, VB) || overlap(B, V) ||
+      overlap(B, VB) || (const void*)A == (const void*)V || (const void*)B == (const void*)VB ||
+      (const void*)A == (const void*)VB || (const void*)B == (const void*)V) {
+    g_err = "key and value arrays must not overlap (B == A and VB == V are allowed)";
+    return HSORT_ERR_INVALID;
+  }
+  if (n > (1ull << 30)) {
+    g_err = "key/value sort: n <= 2^30 pairs (one GPU, no out-of-core merge of pairs)";
+    return HSORT_ERR_INVALID;
+  }
+  return guarded([&]() -> int {
+    auto t0 = Clock::now();
+    GpuCtx& g = S().gpus[0];
+    CK(cudaSetDevice(g.dev));
+    hsort_stats st{};
+    st.n = n;
+    st.b_s = n;
+    st.n_b = 1;
+    st.n_gpus = 1;
+    st.n_s = 1;
+    st.mode = HSORT_MODE_BLINE;
+    st.merge_k = 1;
+    st.t_init = S().t_init;
+    const bool din = is_pinned(A, bytes) && is_pinned(V, bytes);
+    const bool dout = is_pinned(B, bytes) && is_pinned(VB, bytes);
+    const int mc = (int)S().opt.get("memcpy_threads");
+    st.direct_in = din;
+    st.direct_out = dout;
+    g.runs.reserve(bytes);
+    g.alt.reserve(bytes);
+    g.vruns.reserve(bytes);
+    g.valt.reserve(bytes);
+    Acc acc;
+    EvPair eh, es, ed;
+    eh.make();
+    es.make();
+    ed.make();
+    CK(cudaEventRecord(eh.a, g.s_h2d));
+    upload(g, g.runs.p, A, bytes, g.s_h2d, din, mc, acc);
+    upload(g, g.vruns.p, V, bytes, g.s_h2d, din, mc, acc);
+    CK(cudaEventRecord(eh.b, g.s_h2d));
+    CK(cudaStreamWaitEvent(g.s_comp, eh.b, 0));
+    CK(cudaEventRecord(es.a, g.s_comp));
+    CK(radix_sort_pairs(g.rs, g.runs.u64(), g.vruns.u64(), g.runs.u64(), g.vruns.u64(), g.alt.u64(),
+                        g.valt.u64(), n, f64, f64, g.s_comp));
+    CK(cudaEventRecord(es.b, g.s_comp));
+    CK(cudaStreamWaitEvent(g.s_d2h, es.b, 0));
+    CK(cudaEventRecord(ed.a, g.s_d2h));
+    download(g, B, g.runs.p, bytes, g.s_d2h, dout, mc, acc);
+    download(g, VB, g.vruns.p, bytes, g.s_d2h, dout, mc, acc);
+    CK(cudaEventRecord(ed.b, g.s_d2h));
+    CK(cudaStreamSynchronize(g.s_d2h));
+    st.t_sort_phase = secs_since(t0);
+    st.t_h2d = eh.ms() / 1e3;
+    st.t_gpu_sort = es.ms() / 1e3;
+    st.t_d2h = ed.ms() / 1e3;
+    st.t_stage = acc.t_stage;
+    st.bytes_h2d = acc.h2d;
+    st.bytes_d2h = acc.d2h;
+    st.passes_run = g.rs.h_plan->num_active;
+    st.passes_skipped = 8 - g.rs.h_plan->num_active;
+    eh.destroy();
+    es.destroy();
+    ed.destroy();
+    st.t_total = secs_since(t0);
+    S().last = st;
+    return HSORT_OK;
+  });
+}
+
 }  // namespace
 
 // =============================================================================================
@@ -1179,6 +1280,16 @@ int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_
 int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_t batch_elems,
                    int n_gpus) {
   return do_sort(A_host, B_host, n, batch_elems, n_gpus, false);
+}
+
+int hsort_sort_pairs(const double* A_host, const uint64_t* V_host, double* B_host, uint64_t* VB_host,
+                     uint64_t n) {
+  return do_sort_pairs(A_host, V_host, B_host, VB_host, n, true);
+}
+
+int hsort_sort_pairs_u64(const uint64_t* A_host, const uint64_t* V_host, uint64_t* B_host,
+                         uint64_t* VB_host, uint64_t n) {
+  return do_sort_pairs(A_host, V_host, B_host, VB_host, n, false);
 }
 
 int hsort_set_option(const char* key, int64_t value) {
@@ -1274,6 +1385,30 @@ int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, in
     g.alt.reserve(n * 8);
     CK(radix_sort(g.rs, d_in, d_out, g.alt.u64(), n, in_f64 != 0, out_f64 != 0,
                   (cudaStream_t)stream));
+    return HSORT_OK;
+  });
+}
+
+int hsort_sort_device_pairs(const uint64_t* d_keys_in, const uint64_t* d_vals_in,
+                            uint64_t* d_keys_out, uint64_t* d_vals_out, uint64_t n, int keys_f64,
+                            void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (n && (!d_keys_in || !d_vals_in || !d_keys_out || !d_vals_out))
+    return g_err = "null device pointer", HSORT_ERR_INVALID;
+  if (n > (1ull << 30)) return g_err = "key/value sort: n <= 2^30", HSORT_ERR_INVALID;
+  if ((((uintptr_t)d_keys_in | (uintptr_t)d_vals_in | (uintptr_t)d_keys_out |
+        (uintptr_t)d_vals_out) & 15) != 0)
+    return g_err = "key/value sort: device buffers must be 16-byte aligned", HSORT_ERR_INVALID;
+  if ((d_keys_in == d_keys_out) != (d_vals_in == d_vals_out))
+    return g_err = "key/value sort: keys and values must both be in place or both not",
+           HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    g.alt.reserve(n * 8);
+    g.valt.reserve(n * 8);
+    CK(radix_sort_pairs(g.rs, d_keys_in, d_vals_in, d_keys_out, d_vals_out, g.alt.u64(),
+                        g.valt.u64(), n, keys_f64 != 0, keys_f64 != 0, (cudaStream_t)stream));
     return HSORT_OK;
   });
 }

@@ -50,6 +50,7 @@ struct RadixScratch {
 constexpr int kNumKernelEvents = 12;
 
 constexpr int kRadixTile = 4096;  // keys per onesweep tile (THREADS x ITEMS), see radix.cu
+constexpr int kKvTile = 4032;     // pairs per key/value onesweep tile (576 x 7), see radix.cu
 
 cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n);
 cudaError_t radix_set_timing(RadixScratch& s, bool on);
@@ -62,6 +63,12 @@ void radix_scratch_release(RadixScratch& s);
 // pass).  out_f64: store float64 bits (inverse transform fused into the last pass).
 cudaError_t radix_sort(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,
                        uint64_t n, bool in_f64, bool out_f64, cudaStream_t st);
+// Key/value GPUSort (S§8(f) #3): (out, vout) = (in, vin) stably sorted by key; n <= 2^30, every
+// buffer 16-byte aligned, tmp/vtmp n-element scratch; in == out iff vin == vout.  The values are
+// opaque 64-bit payloads (e.g. indices: argsort).
+cudaError_t radix_sort_pairs(RadixScratch& s, const uint64_t* in, const uint64_t* vin, uint64_t* out,
+                             uint64_t* vout, uint64_t* tmp, uint64_t* vtmp, uint64_t n, bool in_f64,
+                             bool out_f64, cudaStream_t st);
 // K1 only (hist zeroed first); d_hist receives 8*256 counts.
 cudaError_t radix_histograms(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
                              uint64_t* d_hist, cudaStream_t st);

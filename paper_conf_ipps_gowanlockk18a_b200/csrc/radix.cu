@@ -967,17 +967,21 @@ __global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ 
 }
 
 // Final conversion/copy (P_eff == 0, or odd P_eff with in == out).
+// Key/value sorts pass the value buffers (same buffer ids); keys-only sorts pass nullptr.
 __global__ void k_final_copy(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
-                             const RadixPlan* __restrict__ plan) {
+                             const RadixPlan* __restrict__ plan, uint64_t* vin = nullptr,
+                             uint64_t* vout = nullptr, uint64_t* vtmp = nullptr) {
   const int cs = plan->copy_src;
   if (cs < 0) return;
   const uint64_t* s = pick(cs, in, out, tmp);
+  const uint64_t* vs = vin ? pick(cs, vin, vout, vtmp) : nullptr;
   const bool fin = plan->copy_in_f64, fout = plan->copy_out_f64;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (uint64_t)gridDim.x * blockDim.x) {
     uint64_t v = s[i];
     if (fin != fout) v = fin ? to_key(v) : from_key(v);
     out[i] = v;
+    if (vs && vs != vout) vout[i] = vs[i];
   }
 }
 
@@ -1135,12 +1139,13 @@ __device__ __forceinline__ uint32_t scan256_excl_c(uint32_t v, uint32_t* s_warp 
   return wpre + x - v;
 }
 
-template <int CT, int ITEMS>
+template <int CT, int ITEMS, bool KV = false>
 struct WsSmem {
   static constexpr int TILE = CT * ITEMS;
   static constexpr int CW = CT / 32;                                          // compute warps
   static constexpr size_t stage_off = 0;                                      // [3][TILE] u64
-  static constexpr size_t whist_off = 3ull * TILE * 8;                        // [CW][257] u32
+  static constexpr size_t vstage_off = 3ull * TILE * 8;                       // [3][TILE] u64 (KV)
+  static constexpr size_t whist_off = (KV ? 6ull : 3ull) * TILE * 8;          // [CW][257] u32
   static constexpr size_t gofs_off = (whist_off + CW * (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [2][256] i32
   static constexpr size_t cnt_off = gofs_off + 2 * kRadix * 4;                // [2][256] u32
   static constexpr size_t bar_off = cnt_off + 2 * kRadix * 4;                 // [12] u64
@@ -1164,6 +1169,10 @@ struct WsSmem {
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
 #endif
+// key/value pass: 18 compute warps x 7 pairs (4032-pair tiles: 3 stages of keys + values = 194 KB)
+constexpr int kKvCT = 576;
+constexpr int kKvItems = 7;
+static_assert(kKvCT * kKvItems == kKvTile, "kKvTile (internal.h) = key/value tile");
 __device__ __forceinline__ void ld_relaxed_v4(const uint32_t* p, uint32_t* v) {
   asm volatile("ld.relaxed.gpu.global.v4.u32 {%0,%1,%2,%3}, [%4];"
                : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
@@ -1259,20 +1268,24 @@ __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64
   for (int q = 0; q < 8; ++q) excl[q] = raw[q] - (n_raw << 30) + msk[q];
 }
 
-template <int CT, int ITEMS, bool IN_F64>
+// KV: key/value pairs (S§8(f) #3): the 64-bit value of each key rides along -- second TMA copy
+// into a value stage, scattered to the key's stage slot, written out to the key's position.
+template <int CT, int ITEMS, bool IN_F64, bool KV = false>
 __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in, uint64_t* out, uint64_t* tmp,
+                                                       uint64_t* vin, uint64_t* vout, uint64_t* vtmp,
                                                        uint64_t n, const RadixPlan* __restrict__ plan,
                                                        const uint64_t* __restrict__ bin_base,
                                                        uint64_t* __restrict__ lookback,
                                                        uint32_t* __restrict__ tile_ctr, int p,
                                                        int out_f64, uint64_t lb_half,
                                                        uint64_t lb_rows) {
-  using L = WsSmem<CT, ITEMS>;
+  using L = WsSmem<CT, ITEMS, KV>;
   constexpr int TILE = L::TILE;
   constexpr int CW = L::CW;
   constexpr int THREADS = CT;  // compute threads
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* stage = (uint64_t*)(smem + L::stage_off);
+  uint64_t* vstage = (uint64_t*)(smem + L::vstage_off);  // KV only
   uint32_t* whist = (uint32_t*)(smem + L::whist_off);
   int32_t* s_gofs = (int32_t*)(smem + L::gofs_off);
   uint32_t* s_cnt = (uint32_t*)(smem + L::cnt_off);
@@ -1290,6 +1303,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   const int shift = 8 * digit;
   const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
   uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const uint64_t* __restrict__ vsrc = KV ? pick(plan->src[p], vin, vout, vtmp) : nullptr;
+  uint64_t* __restrict__ vdst = KV ? pick(plan->dst[p], vin, vout, vtmp) : nullptr;
   const bool use_match = (plan->match_mask >> p) & 1;
   const bool inv = out_f64 && (p == na - 1);
   uint32_t* lb32 = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p) & 1) * lb_half;
@@ -1304,8 +1319,11 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       const uint64_t base = (uint64_t)t * TILE;
       const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
       const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
-      mbar_arrive_expect_tx(&bar_tma[b], bytes);
-      if (bytes) bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bar_tma[b]);
+      mbar_arrive_expect_tx(&bar_tma[b], KV ? 2 * bytes : bytes);
+      if (bytes) {
+        bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bar_tma[b]);
+        if (KV) bulk_g2s(vstage + (size_t)b * TILE, vsrc + base, bytes, &bar_tma[b]);
+      }
     } else {
       mbar_arrive(&bar_tma[b]);
     }
@@ -1414,6 +1432,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #endif
     const int32_t* gofs = s_gofs + (jj & 1) * kRadix;
     const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
+    const uint64_t* vsb = vstage + (size_t)(jj % 3) * TILE;
     const uint64_t rem = n - tile * (uint64_t)TILE;
     const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
     auto wo_full = [&](auto inv_tag) {
@@ -1421,11 +1440,13 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
       for (int q = 0; q < ITEMS; ++q) {
         const uint64_t v = sb[tid + q * THREADS];
-        uint64_t* a = dst_t + gofs[(uint32_t)(v >> shift) & 255u];
+        const int32_t g = gofs[(uint32_t)(v >> shift) & 255u];
+        uint64_t* a = dst_t + g;
 #if HSORT_FAKE == 3
         if (v == 0x123456789ull)
 #endif
         st_global_u64((uint64_t)(a + q * THREADS), INV ? from_key(v) : v);
+        if (KV) st_global_u64((uint64_t)(vdst + tid + g + q * THREADS), vsb[tid + q * THREADS]);
       }
     };
     if (tile_n == TILE) {
@@ -1434,7 +1455,9 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     } else {
       for (int i = tid; i < tile_n; i += THREADS) {
         const uint64_t v = sb[i];
-        st_global_u64((uint64_t)(dst + gofs[(uint32_t)(v >> shift) & 255u] + i), inv ? from_key(v) : v);
+        const int32_t g = gofs[(uint32_t)(v >> shift) & 255u];
+        st_global_u64((uint64_t)(dst + g + i), inv ? from_key(v) : v);
+        if (KV) st_global_u64((uint64_t)(vdst + g + i), vsb[i]);
       }
     }
     __syncwarp();
@@ -1442,13 +1465,14 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   };
   // one tile: load from the stage, per-warp digit counts, tile aggregate + scan, warp ranking,
   // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
-  auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, uint64_t* sb) {
+  auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, uint64_t* sb, uint64_t* vsb) {
     constexpr bool FULL = decltype(full_tag)::value;
     const uint64_t tbase = tile * (uint64_t)TILE;
     const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
     const int wofs = warp * 32 * ITEMS + lane;
     uint32_t* wh = whist + warp * (kRadix + 1);  // this warp's row: zero on entry
     uint64_t k[ITEMS];
+    uint64_t vv[KV ? ITEMS : 1];
     uint32_t dd[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -1456,6 +1480,10 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       uint64_t v;
       if (FULL) v = sb[jj];
       else v = jj < bulk_n ? sb[jj] : (jj < tile_n ? src[tbase + jj] : 0);
+      if (KV) {
+        if (FULL) vv[i] = vsb[jj];
+        else vv[i] = jj < bulk_n ? vsb[jj] : (jj < tile_n ? vsrc[tbase + jj] : 0);
+      }
       k[i] = IN_F64 ? to_key(v) : v;
       const bool valid = FULL || jj < tile_n;
       dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
@@ -1497,7 +1525,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       // high-entropy digits: an 8-ballot multisplit (4 instructions per bit: test -> predicate,
       // vote, select, and) for most items; the first NM items use match.any, which runs on another
       // pipe, so both proceed in parallel
-      constexpr int NM = HSORT_WS_NMATCH < ITEMS ? HSORT_WS_NMATCH : ITEMS;
+      constexpr int NM0 = KV ? (ITEMS * HSORT_WS_NMATCH + 7) / 15 : HSORT_WS_NMATCH;
+      constexpr int NM = NM0 < ITEMS ? NM0 : ITEMS;
 #pragma unroll
       for (int i = 0; i < NM; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
 #pragma unroll
@@ -1531,7 +1560,10 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
       const uint32_t r = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
-      if (FULL || dd[i] < kRadix) sb[r] = k[i];
+      if (FULL || dd[i] < kRadix) {
+        sb[r] = k[i];
+        if (KV) vsb[r] = vv[i];
+      }
     }
     // the row is private to this warp from here to the next tile's counts: clear it now
     __syncwarp();
@@ -1560,9 +1592,10 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     const uint64_t rem = n - tile * (uint64_t)TILE;
     const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
     uint64_t* sb = stage + (size_t)cb * TILE;
+    uint64_t* vsb = vstage + (size_t)cb * TILE;
     long long cr0;
-    if (tile_n == TILE) cr0 = rank_tile(std::true_type{}, tile, tile_n, sb);
-    else cr0 = rank_tile(std::false_type{}, tile, tile_n, sb);
+    if (tile_n == TILE) cr0 = rank_tile(std::true_type{}, tile, tile_n, sb, vsb);
+    else cr0 = rank_tile(std::false_type{}, tile, tile_n, sb, vsb);
 #ifdef HSORT_PHASE_TIMING
     t_cnt += cr0 - cc0;
     long long cw1 = clock64();
@@ -1598,15 +1631,16 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       lb32_next[rr * kRadix + tid] = 0;
 }
 
-template <int CT, int ITEMS>
-cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n, RadixScratch& s,
-                           int p, bool first_in_f64, bool out_f64, cudaStream_t st) {
-  using L = WsSmem<CT, ITEMS>;
+template <int CT, int ITEMS, bool KV = false>
+cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t* vin, uint64_t* vout,
+                           uint64_t* vtmp, uint64_t n, RadixScratch& s, int p, bool first_in_f64,
+                           bool out_f64, cudaStream_t st) {
+  using L = WsSmem<CT, ITEMS, KV>;
   static int blocks_per_sm[64] = {0};
   int dev = 0;
   cudaGetDevice(&dev);
-  auto kt = k_onesweep_ws<CT, ITEMS, true>;
-  auto kf = k_onesweep_ws<CT, ITEMS, false>;
+  auto kt = k_onesweep_ws<CT, ITEMS, true, KV>;
+  auto kf = k_onesweep_ws<CT, ITEMS, false, KV>;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   if (!blocks_per_sm[dev]) {
     cudaError_t e;
@@ -1621,13 +1655,13 @@ cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t 
   uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
   if (grid > tiles) grid = tiles ? tiles : 1;
   if (first_in_f64)
-    kt<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
-                                             s.tile_ctr, p, out_f64 ? 1 : 0, s.max_tiles * kRadix,
-                                             s.lb_rows);
+    kt<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, vin, vout, vtmp, n, s.plan, s.bin_base,
+                                             s.lookback, s.tile_ctr, p, out_f64 ? 1 : 0,
+                                             s.max_tiles * kRadix, s.lb_rows);
   else
-    kf<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
-                                             s.tile_ctr, p, out_f64 ? 1 : 0, s.max_tiles * kRadix,
-                                             s.lb_rows);
+    kf<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, vin, vout, vtmp, n, s.plan, s.bin_base,
+                                             s.lookback, s.tile_ctr, p, out_f64 ? 1 : 0,
+                                             s.max_tiles * kRadix, s.lb_rows);
   return cudaGetLastError();
 }
 
@@ -1643,7 +1677,7 @@ int pass_kernel(uint64_t* in, uint64_t* out, uint64_t* tmp) {
 // exclude its own keys.  The one value that can reach 2^30 (all n keys in one digit, a forced
 // single pass) is only read by tiles without keys of d and decodes as flag 3 = "aggregate", so a
 // reader never spins on it.
-cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t st) {
+cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t st, bool kv = false) {
   const int mode = (kernel >= 1 && n <= (1ull << 30)) ? 2 : 1;
   if (s.lb_mode != 0 && s.lb_mode != mode) {
     cudaError_t e = cudaMemsetAsync(s.lookback, 0, s.max_tiles * kRadix * sizeof(uint64_t), st);
@@ -1652,7 +1686,8 @@ cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t
   }
   s.lb_mode = mode;
   if (mode == 2) {
-    const uint64_t tile = kernel == 2 ? (uint64_t)HSORT_WS_CT * HSORT_WS_ITEMS : (uint64_t)kRadixTile;
+    const uint64_t tile = kv ? (uint64_t)kKvTile
+                             : (kernel == 2 ? (uint64_t)HSORT_WS_CT * HSORT_WS_ITEMS : (uint64_t)kRadixTile);
     const uint64_t t = (n + tile - 1) / tile;
     if (t > s.lb_rows) s.lb_rows = t;
   }
@@ -1667,7 +1702,8 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const int v = pass_kernel(in, out, tmp);
   if (v == 2 && s.lb_mode == 2)
-    return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS>(in, out, tmp, n, s, p, first_in_f64, out_f64, st);
+    return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS>(in, out, tmp, nullptr, nullptr, nullptr, n, s, p,
+                                                       first_in_f64, out_f64, st);
   // look-back window 4: measured best of 1..32
   if (v >= 1) {
     if (s.lb_mode == 2)
@@ -1722,7 +1758,8 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
     if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)
       return e;
   }
-  uint64_t tiles = (n + kRadixTile - 1) / kRadixTile;
+  // smallest tile of any pass kernel: the key/value pass (kKvTile keys)
+  uint64_t tiles = (n + kKvTile - 1) / kKvTile;
   if (tiles < 1) tiles = 1;
   if (tiles > s.max_tiles) {
     if (s.lookback) cudaFree(s.lookback);
@@ -1798,6 +1835,47 @@ cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uin
   int dev = 0;
   cudaGetDevice(&dev);
   k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = mark(11)) != cudaSuccess) return e;
+  return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);
+}
+
+// Key/value GPUSort (S§8(f) #3): K1/K2 on the keys as in radix_sort, then every active digit
+// pass with the key/value warp-specialised kernel; the values follow the keys' ping-pong.
+cudaError_t radix_sort_pairs(RadixScratch& s, const uint64_t* in_c, const uint64_t* vin_c,
+                             uint64_t* out, uint64_t* vout, uint64_t* tmp, uint64_t* vtmp, uint64_t n,
+                             bool in_f64, bool out_f64, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  if (n > (1ull << 30)) return cudaErrorNotSupported;  // 32-bit look-back words
+  uint64_t* in = const_cast<uint64_t*>(in_c);
+  uint64_t* vin = const_cast<uint64_t*>(vin_c);
+  if ((((uintptr_t)in | (uintptr_t)out | (uintptr_t)tmp | (uintptr_t)vin | (uintptr_t)vout |
+        (uintptr_t)vtmp) & 15) != 0)
+    return cudaErrorMisalignedAddress;  // TMA bulk copies
+  if ((in == out) != (vin == vout)) return cudaErrorInvalidValue;  // one plan serves both
+  cudaError_t e = radix_scratch_reserve(s, n);
+  if (e != cudaSuccess) return e;
+  auto mark = [&](int i) -> cudaError_t {
+    return s.timing ? cudaEventRecord(s.ev[i], st) : cudaSuccess;
+  };
+  if ((e = cudaMemsetAsync(s.small, 0, s.small_zero_bytes, st)) != cudaSuccess) return e;
+  if ((e = mark(0)) != cudaSuccess) return e;
+  if ((e = launch_hist(s, in, n, in_f64, s.hist, st)) != cudaSuccess) return e;
+  if ((e = mark(1)) != cudaSuccess) return e;
+  if ((e = select_lb_mode(s, 2, n, st, true)) != cudaSuccess) return e;
+  k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
+                                 out_f64 ? 1 : 0, s.lb_state);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = mark(2)) != cudaSuccess) return e;
+  for (int p = 0; p < kDigits; ++p) {
+    if ((e = launch_ws_pass<kKvCT, kKvItems, true>(in, out, tmp, vin, vout, vtmp, n, s, p,
+                                                    p == 0 && in_f64, out_f64, st)) != cudaSuccess)
+      return e;
+    if ((e = mark(3 + p)) != cudaSuccess) return e;
+  }
+  int dev = 0;
+  cudaGetDevice(&dev);
+  k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan, vin, vout, vtmp);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   if ((e = mark(11)) != cudaSuccess) return e;
   return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);

@@ -165,6 +165,30 @@ def stage_rooflines(hs, torch, d_in, d_out, n, peak, hist_ms, pass_ms, stream):
     kv = statistics.median(kv_ms)
     kv_pass_ms = statistics.mean(kv_pass)
 
+    # other key types / orders (S§8(f) #4): float32 (encode -> 4 LSD passes -> decode) and
+    # float64 descending (encode -> 8 passes -> decode), 2^30 keys, whole-sort time
+    def timed(fn):
+        fn()
+        ts = []
+        for _ in range(3):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            fn()
+            e1.record(stream)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        return statistics.median(ts)
+    d32 = d_in.float()
+    o32 = torch.empty_like(d32)
+    f32_ms = timed(lambda: hs.hsort_sort_device_typed(d32, o32, False, stream))
+    f32_passes = hs.hsort_get_kernel_times()["num_active"]
+    assert bool((o32[1:] >= o32[:-1]).all()), "float32 output not sorted"
+    del d32, o32
+    desc_ms = timed(lambda: hs.hsort_sort_device_typed(d_in, d_out, True, stream))
+    assert bool((d_out[1:] <= d_out[:-1]).all()), "descending output not sorted"
+    types = {"f32_asc": {"sort_ms": f32_ms, "keys_per_s": n / (f32_ms / 1e3), "passes": f32_passes},
+             "f64_desc": {"sort_ms": desc_ms, "keys_per_s": n / (desc_ms / 1e3)}}
+
     cuts = [n * j // MERGE_K for j in range(MERGE_K + 1)]
     for j in range(MERGE_K):
         hs.hsort_sort_device_keys(d_in[cuts[j]:cuts[j + 1]], d_out[cuts[j]:cuts[j + 1]], True, False,
@@ -198,6 +222,7 @@ def stage_rooflines(hs, torch, d_in, d_out, n, peak, hist_ms, pass_ms, stream):
         "K3_onesweep": hbm(pass_ms, 16, "k_onesweep_ws (one 8-bit LSD pass)"),
         "K3_kv_pass": dict(hbm(kv_pass_ms, 32, "k_onesweep_ws<KV> (one LSD pass over key/value pairs)"),
                            sort_ms=kv, pairs_per_s=n / (kv / 1e3)),
+        "key_types": types,
         "K5_merge": dict(hbm(k5, 16, f"k_merge_tile (k = {MERGE_K} resident runs, 2^30 keys)"),
                          k4_corank_ms=k4, k4_k5_frac=16 * n / (merge / 1e3) / 1e9 / peak),
     }

@@ -135,6 +135,20 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
                    int n_gpus);
 
 /* ---------------------------------------------------------------------------------------------
+ * Other key types and orders.  key_type HSORT_KEY_F64 (8-byte float64) or
+ * HSORT_KEY_F32 (4-byte float32); descending != 0 sorts by the reverse of IEEE totalOrder (the
+ * exact reverse of the ascending result: every totalOrder class is one bit pattern).  Keys are
+ * sorted as bit patterns (NaN payloads and -0.0 preserved).  float64 ascending is hsort_sort
+ * (every mode); every other combination runs on one GPU as one batch (BLINE): an encode pass to
+ * 64-bit internal keys (float32 keys zero-extended, so the radix plan skips the 4 empty digits),
+ * the GPUSort, a decode pass.  n must fit one GPU (16 B/key + the key array), else
+ * HSORT_ERR_INVALID.  A and B aligned to the key size; B == A allowed; partial overlap -> INVALID.
+ * ------------------------------------------------------------------------------------------- */
+#define HSORT_KEY_F64 0
+#define HSORT_KEY_F32 1
+int hsort_sort_typed(const void* A_host, void* B_host, uint64_t n, int key_type, int descending);
+
+/* ---------------------------------------------------------------------------------------------
  * Key/value sort (the [5] workload of 64-bit keys with 64-bit values,
  * P:743-761).  B/VB = the pairs (A[i], V[i]) ordered by A under IEEE totalOrder, STABLY: pairs
  * with equal keys keep their input order, so the result is unique (V = 0..n-1 gives the stable
@@ -199,6 +213,12 @@ int hsort_sort_device(const double* d_in, double* d_out, uint64_t n, void* strea
  * float64 bits (inverse transform fused into the last pass). */
 int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, int in_f64,
                            int out_f64, void* stream);
+
+/* Typed GPUSort, device -> device (current device, stream-ordered): key_type / descending as for
+ * hsort_sort_typed.  float64 ascending = hsort_sort_device; otherwise encode -> GPUSort -> decode
+ * (16-byte aligned buffers; d_in == d_out allowed; library scratch 16 B/key). */
+int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_type,
+                            int descending, void* stream);
 
 /* Key/value GPUSort, device -> device (current device, stream-ordered): (d_keys_out,
  * d_vals_out) = the pairs stably sorted by key (float64 totalOrder bits in and out if keys_f64,

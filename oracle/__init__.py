@@ -56,6 +56,8 @@ def _load():
                 "oracle_is_sorted_f64": ([_P, _U64], ctypes.c_int),
                 "oracle_multiset_hash": ([_P, _U64, _P], None),
                 "oracle_sort_pairs_f64": ([_P, _P, _P, _P, _U64], None),
+                "oracle_sort_f32": ([_P, _P, _U64, ctypes.c_int], None),
+                "oracle_sort_desc_f64": ([_P, _P, _U64], None),
                 "oracle_sort_pairs_u64": ([_P, _P, _P, _P, _U64], None),
             }
             for name, (args, res) in sig.items():
@@ -132,6 +134,21 @@ def _pack_runs(runs):
         off[j + 1] = off[j] + r.size
     keys = np.concatenate(runs) if runs else np.zeros(0, dtype=np.uint64)
     return _c(keys, np.uint64), off
+
+
+def sort_f32(A, descending: bool = False) -> np.ndarray:
+    """float32 keys sorted by binary32 totalOrder (or its reverse) (oracle.cpp)."""
+    A = np.ascontiguousarray(A, dtype=np.float32)
+    B = np.empty_like(A)
+    _load().oracle_sort_f32(A.ctypes.data, B.ctypes.data, A.size, int(descending))
+    return B
+
+
+def sort_desc_f64(A) -> np.ndarray:
+    A = np.ascontiguousarray(A, dtype=np.float64)
+    B = np.empty_like(A)
+    _load().oracle_sort_desc_f64(A.ctypes.data, B.ctypes.data, A.size)
+    return B
 
 
 def sort_pairs_f64(A, V):

@@ -23,6 +23,10 @@
 //   oracle_corank              pinned: co-rank invariants (sum, boundary) + brute force.
 //   oracle_pipemerge_count     pinned: Fig. 3 worked example (tests/golden/fig3_pipemerge.txt).
 //   oracle_is_sorted_f64 / oracle_multiset_hash: pinned by planted faults.
+//   oracle_sort_f32 / oracle_sort_desc_f64 pinned: brute force (all permutations of small
+//                              inputs over a binary32 special alphabet) vs a Python restatement
+//                              of the IEEE clauses on binary32 bits; numpy.sort on NaN/-0-free
+//                              data; descending = reverse of ascending (unique result).
 //   oracle_sort_pairs_f64/_u64 pinned: keys = oracle_sort; values = numpy stable argsort on
 //                              NaN/-0-free keys; brute force over all permutations of small
 //                              duplicate-heavy inputs vs a Python insertion sort (stable by
@@ -57,6 +61,23 @@ int oracle_total_order_cmp(double a, double b) {
 void oracle_sort_f64(const double* A, double* B, uint64_t n) {
   if (B != A) std::memcpy(B, A, n * sizeof(double));
   std::sort(B, B + n, total_less);
+}
+
+// ---------------------------------------------------------------------------------------------
+// Other key types and orders.  float32 keys under binary32 totalOrder
+// (std::strong_order<float>), and the descending order (reverse totalOrder) for both types:
+// B = A sorted by y precedes x <=> totalOrder(x, y) strictly.
+void oracle_sort_f32(const float* A, float* B, uint64_t n, int descending) {
+  if (B != A) std::memcpy(B, A, n * sizeof(float));
+  if (descending)
+    std::sort(B, B + n, [](float a, float b) { return std::strong_order(a, b) > 0; });
+  else
+    std::sort(B, B + n, [](float a, float b) { return std::strong_order(a, b) < 0; });
+}
+
+void oracle_sort_desc_f64(const double* A, double* B, uint64_t n) {
+  if (B != A) std::memcpy(B, A, n * sizeof(double));
+  std::sort(B, B + n, [](double a, double b) { return std::strong_order(a, b) > 0; });
 }
 
 // ---------------------------------------------------------------------------------------------

@@ -75,6 +75,8 @@ SIGNATURES = {
     "hsort_finalize": ([], _I),
     "hsort_sort": ([_P, _P, _U64, _U64, _I], _I),
     "hsort_sort_u64": ([_P, _P, _U64, _U64, _I], _I),
+    "hsort_sort_typed": ([_P, _P, _U64, _I, _I], _I),
+    "hsort_sort_device_typed": ([_P, _P, _U64, _I, _I, _P], _I),
     "hsort_sort_pairs": ([_P, _P, _P, _P, _U64], _I),
     "hsort_sort_pairs_u64": ([_P, _P, _P, _P, _U64], _I),
     "hsort_sort_device_pairs": ([_P, _P, _P, _P, _U64, _I, _P], _I),
@@ -216,6 +218,23 @@ def hsort_sort_u64(A, B=None, batch_elems: int = 0, n_gpus: int = 0):
     return B
 
 
+KEY_F64, KEY_F32 = 0, 1
+
+
+def hsort_sort_typed(A, B=None, descending: bool = False):
+    """B = A sorted by IEEE totalOrder (descending: its reverse); A float64 or float32 numpy array
+    (host -> host; float64 ascending = hsort_sort, else one GPU, one batch)."""
+    if not isinstance(A, np.ndarray) or A.dtype not in (np.float64, np.float32) or not A.flags.c_contiguous:
+        raise TypeError("expected a C-contiguous float64 or float32 numpy array")
+    if B is None:
+        B = np.empty_like(A)
+    if not isinstance(B, np.ndarray) or B.dtype != A.dtype or B.size != A.size or not B.flags.c_contiguous:
+        raise ValueError("B must be a C-contiguous array of A's dtype and length")
+    kt = KEY_F64 if A.dtype == np.float64 else KEY_F32
+    _check(lib().hsort_sort_typed(A.ctypes.data, B.ctypes.data, A.size, kt, int(descending)))
+    return B
+
+
 def hsort_sort_pairs(A, V, B=None, VB=None):
     """(B, VB) = the pairs (A[i], V[i]) stably sorted by A under IEEE totalOrder (host -> host,
     one GPU, n <= 2^30).  A float64, V uint64 payloads (e.g. np.arange(n): stable argsort)."""
@@ -287,6 +306,16 @@ def hsort_sort_device_keys(d_in, d_out, in_f64: bool, out_f64: bool, stream=None
     n = d_in.numel()
     _check(lib().hsort_sort_device_keys(_dev_ptr(d_in), _dev_ptr(d_out), n, int(in_f64),
                                         int(out_f64), _stream_ptr(stream)))
+
+
+def hsort_sort_device_typed(d_in, d_out, descending: bool = False, stream=None) -> None:
+    """d_out = d_in sorted by IEEE totalOrder (or its reverse); float64 or float32 CUDA tensors."""
+    import torch
+    kt = {torch.float64: KEY_F64, torch.float32: KEY_F32}[d_in.dtype]
+    if d_out.dtype != d_in.dtype or d_out.numel() != d_in.numel():
+        raise ValueError("d_out must match d_in in dtype and length")
+    _check(lib().hsort_sort_device_typed(_dev_ptr(d_in), _dev_ptr(d_out), d_in.numel(), kt,
+                                         int(descending), _stream_ptr(stream)))
 
 
 def hsort_sort_device_pairs(d_keys_in, d_vals_in, d_keys_out, d_vals_out, keys_f64: bool = True,

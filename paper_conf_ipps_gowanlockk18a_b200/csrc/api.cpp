@@ -1209,6 +1209,96 @@ int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint6
   });
 }
 
+// Other key types / orders (S§8(f) #4), host -> host on one GPU (BLINE): HtoD of the raw keys,
+// encode into internal uint64 keys, the GPUSort on those, decode, DtoH.  float64 ascending keeps
+// the fused path (do_sort, every mode).
+int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
+  if (key_type == HSORT_KEY_F64 && !desc) return do_sort(A, B, n, 0, 1, true);
+  int rc = check_ready();
+  if (rc) return rc;
+  if (key_type != HSORT_KEY_F64 && key_type != HSORT_KEY_F32)
+    return g_err = "key_type must be HSORT_KEY_F64 or HSORT_KEY_F32", HSORT_ERR_INVALID;
+  BusyGuard busy;
+  if (!busy.ok) {
+    g_err = "hsort_sort already running";
+    return HSORT_ERR_BUSY;
+  }
+  if (n == 0) {
+    S().last = hsort_stats{};
+    return HSORT_OK;
+  }
+  const uint64_t es = key_type == HSORT_KEY_F64 ? 8 : 4;
+  if (!A || !B) return g_err = "null A or B with n > 0", HSORT_ERR_INVALID;
+  if ((((uintptr_t)A) | ((uintptr_t)B)) & (es - 1))
+    return g_err = "A and B must be aligned to the key size", HSORT_ERR_INVALID;
+  const uint64_t bytes = n * es;
+  const uintptr_t a0 = (uintptr_t)A, b0 = (uintptr_t)B;
+  if (A != B && a0 < b0 + bytes && b0 < a0 + bytes)
+    return g_err = "A and B partially overlap", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    auto t0 = Clock::now();
+    GpuCtx& g = S().gpus[0];
+    CK(cudaSetDevice(g.dev));
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    const uint64_t held = g.runs.cap + g.alt.cap + g.mout.cap;
+    const uint64_t need = n * 8 * 2 + ((bytes + 15) & ~15ull) + n / 2 +
+                          (uint64_t)S().opt.get("device_reserve_mb") * (1ull << 20);
+    if (need > fr + held)
+      throw HsortError(HSORT_ERR_INVALID, "typed sort: n does not fit one GPU (BLINE only)");
+    hsort_stats st{};
+    st.n = n;
+    st.b_s = n;
+    st.n_b = 1;
+    st.n_gpus = 1;
+    st.n_s = 1;
+    st.mode = HSORT_MODE_BLINE;
+    st.merge_k = 1;
+    st.t_init = S().t_init;
+    const bool din = is_pinned(A, bytes), dout = is_pinned(B, bytes);
+    const int mc = (int)S().opt.get("memcpy_threads");
+    st.direct_in = din;
+    st.direct_out = dout;
+    g.runs.reserve(n * 8);
+    g.alt.reserve(n * 8);
+    g.mout.reserve((bytes + 15) & ~15ull);
+    Acc acc;
+    EvPair eh, es_, ed;
+    eh.make();
+    es_.make();
+    ed.make();
+    CK(cudaEventRecord(eh.a, g.s_h2d));
+    upload(g, g.mout.p, A, bytes, g.s_h2d, din, mc, acc);
+    CK(cudaEventRecord(eh.b, g.s_h2d));
+    CK(cudaStreamWaitEvent(g.s_comp, eh.b, 0));
+    CK(cudaEventRecord(es_.a, g.s_comp));
+    CK(key_encode(g.mout.p, g.runs.u64(), n, key_type, desc != 0, g.s_comp));
+    CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), n, false, false, g.s_comp));
+    CK(key_decode(g.runs.u64(), g.mout.p, n, key_type, desc != 0, g.s_comp));
+    CK(cudaEventRecord(es_.b, g.s_comp));
+    CK(cudaStreamWaitEvent(g.s_d2h, es_.b, 0));
+    CK(cudaEventRecord(ed.a, g.s_d2h));
+    download(g, B, g.mout.p, bytes, g.s_d2h, dout, mc, acc);
+    CK(cudaEventRecord(ed.b, g.s_d2h));
+    CK(cudaStreamSynchronize(g.s_d2h));
+    st.t_sort_phase = secs_since(t0);
+    st.t_h2d = eh.ms() / 1e3;
+    st.t_gpu_sort = es_.ms() / 1e3;
+    st.t_d2h = ed.ms() / 1e3;
+    st.t_stage = acc.t_stage;
+    st.bytes_h2d = acc.h2d;
+    st.bytes_d2h = acc.d2h;
+    st.passes_run = g.rs.h_plan->num_active;
+    st.passes_skipped = 8 - g.rs.h_plan->num_active;
+    eh.destroy();
+    es_.destroy();
+    ed.destroy();
+    st.t_total = secs_since(t0);
+    S().last = st;
+    return HSORT_OK;
+  });
+}
+
 }  // namespace
 
 // =============================================================================================
@@ -1280,6 +1370,10 @@ int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_
 int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_t batch_elems,
                    int n_gpus) {
   return do_sort(A_host, B_host, n, batch_elems, n_gpus, false);
+}
+
+int hsort_sort_typed(const void* A_host, void* B_host, uint64_t n, int key_type, int descending) {
+  return do_sort_typed(A_host, B_host, n, key_type, descending);
 }
 
 int hsort_sort_pairs(const double* A_host, const uint64_t* V_host, double* B_host, uint64_t* VB_host,
@@ -1385,6 +1479,29 @@ int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, in
     g.alt.reserve(n * 8);
     CK(radix_sort(g.rs, d_in, d_out, g.alt.u64(), n, in_f64 != 0, out_f64 != 0,
                   (cudaStream_t)stream));
+    return HSORT_OK;
+  });
+}
+
+int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_type,
+                            int descending, void* stream) {
+  int rc = check_ready();
+  if (rc) return rc;
+  if (key_type != HSORT_KEY_F64 && key_type != HSORT_KEY_F32)
+    return g_err = "key_type must be HSORT_KEY_F64 or HSORT_KEY_F32", HSORT_ERR_INVALID;
+  if (n && (!d_in || !d_out)) return g_err = "null device pointer", HSORT_ERR_INVALID;
+  if (key_type == HSORT_KEY_F64 && !descending)
+    return hsort_sort_device_keys((const uint64_t*)d_in, (uint64_t*)d_out, n, 1, 1, stream);
+  if ((((uintptr_t)d_in) | ((uintptr_t)d_out)) & 15)
+    return g_err = "typed sort: device buffers must be 16-byte aligned", HSORT_ERR_INVALID;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    cudaStream_t st = (cudaStream_t)stream;
+    g.runs.reserve(n * 8);
+    g.alt.reserve(n * 8);
+    CK(key_encode(d_in, g.runs.u64(), n, key_type, descending != 0, st));
+    CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), n, false, false, st));
+    CK(key_decode(g.runs.u64(), d_out, n, key_type, descending != 0, st));
     return HSORT_OK;
   });
 }

@@ -92,6 +92,16 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint
                         uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
                         cudaStream_t st);
 
+// ---- key codecs (codec.cu, S§8(f) #4) ---------------------------------------------------------
+constexpr int kKeyF64 = 0;
+constexpr int kKeyF32 = 1;
+// in (n float64 or float32 bits) -> out (n internal uint64 keys, ascending = the requested
+// order); 16-byte aligned buffers.  decode is the inverse.
+cudaError_t key_encode(const void* in, uint64_t* out, uint64_t n, int key_type, bool desc,
+                       cudaStream_t st);
+cudaError_t key_decode(const uint64_t* in, void* out, uint64_t n, int key_type, bool desc,
+                       cudaStream_t st);
+
 // out[i] = #keys <= values[i] in the sorted run keys[0, n) (device pointers).
 cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
                          uint64_t* out, cudaStream_t st);

@@ -90,4 +90,58 @@ def insertion_sort_bits(bits: list[int]) -> list[int]:
     return out
 
 
+# ---- binary32 (S§8(f) #4): the same clauses on 32-bit fields --------------------------------------
+def bits32_to_f(u: int) -> float:
+    return struct.unpack("<f", struct.pack("<I", u & 0xFFFFFFFF))[0]
+
+
+def _is_nan32(u: int) -> bool:
+    return ((u >> 23) & 0xFF) == 0xFF and (u & ((1 << 23) - 1)) != 0
+
+
+def total_order_le32(ux: int, uy: int) -> bool:
+    """totalOrder(x, y) for the binary32 bit patterns ux, uy (clauses as total_order_le)."""
+    sx, sy = ux >> 31, uy >> 31
+    nx, ny = _is_nan32(ux), _is_nan32(uy)
+    if not nx and not ny:
+        x, y = bits32_to_f(ux), bits32_to_f(uy)  # exact (binary32 -> double)
+        if x < y:
+            return True
+        if x > y:
+            return False
+        if x == 0.0 and sx != sy:
+            return sx == 1
+        return True
+    if nx and not ny:
+        return sx == 1
+    if ny and not nx:
+        return sy == 0
+    if sx != sy:
+        return sx == 1
+    neg = sx == 1
+    qx, qy = bool((ux >> 22) & 1), bool((uy >> 22) & 1)
+    if qx != qy:
+        return (not qx) if not neg else qx
+    px, py = ux & ((1 << 22) - 1), uy & ((1 << 22) - 1)
+    return px <= py if not neg else px >= py
+
+
+def insertion_sort_bits32(bits: list[int], descending: bool = False) -> list[int]:
+    out: list[int] = []
+    for u in bits:
+        i = len(out)
+        if descending:  # u moves left past elements it strictly follows in totalOrder
+            while i > 0 and total_order_le32(out[i - 1], u) and not total_order_le32(u, out[i - 1]):
+                i -= 1
+        else:
+            while i > 0 and total_order_le32(u, out[i - 1]) and not total_order_le32(out[i - 1], u):
+                i -= 1
+        out.insert(i, u)
+    return out
+
+
+SPECIAL32 = [0xFFC00000, 0xFF800001, 0xFF800000, 0xFF7FFFFF, 0xBF800000, 0x80000001, 0x80000000,
+             0x00000000, 0x00000001, 0x3F800000, 0x7F7FFFFF, 0x7F800000, 0x7F800001, 0x7FC00000,
+             0x7FFFFFFF]  # -qNaN -sNaN -inf -max -1 -denorm -0 +0 +denorm 1 max inf sNaN qNaN qNaN(max)
+
 assert math.isnan(bits_to_f(0x7FF8000000000000))

@@ -172,10 +172,10 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
 
 // K5.  One CTA per output tile of kMergeTile keys, T threads x IPT = kMergeTile / T keys.
 //   1. slice table: len_j = r1[j] - r0[j], bnd = exclusive prefix of len (tile-local starts);
-//   2. gather: the k slices are copied into buf0 back to back.  Thread tid loads elements
-//      p = q T + tid (q < IPT, coalesced within a slice); the run of p, max{j : bnd[j] <= p}, only
-//      grows with q, so it is found once and then advanced; all IPT loads are issued before any
-//      store, so IPT HBM reads per thread are in flight;
+//   2. gather: the k slices are copied into buf0 back to back.  Warp w loads elements
+//      [32 IPT w, 32 IPT (w + 1)) lane-interleaved (coalesced within a slice); the run of an
+//      element, max{j : bnd[j] <= p}, only grows along a lane's elements, so it is found once and
+//      then advanced; all IPT loads are issued before any store (IPT HBM reads in flight);
 //   3. ceil(log2 k) pairwise merge-path rounds between buf0 and buf1: in round r the sequences are
 //      the groups of 2^r consecutive runs, so sequence m starts at bnd[min(m 2^r, k)] and no
 //      boundary table is rewritten; the pair holding a thread's first output in round r is
@@ -199,7 +199,8 @@ struct MergeCfg {
   static constexpr int IPT = kMergeTile / T;
   static_assert(T * IPT == kMergeTile, "merge tile");
   static constexpr int BUF = kMergeTile + kMergeTile / IPT;
-  static __device__ __forceinline__ int pp(int p) { return p + p / IPT; }
+  // p >= 0: unsigned division is one shift (a signed one costs three instructions)
+  static __device__ __forceinline__ int pp(int p) { return p + (int)((unsigned)p / IPT); }
 };
 
 // largest j >= a with bnd[j] <= p (j < cnt), starting from a valid j = a: two linear steps (the
@@ -287,33 +288,36 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   __syncthreads();
 
   uint64_t* o = out + (o0 - out_origin);
-  const uint64_t xmask = out_f64 ? ~0ull : 0ull;  // from_key applied iff out_f64
 
-  // 2. gather (k == 1: straight copy)
+  // 2. gather (k == 1: straight copy).  Warp w copies tile elements [w C, w C + C), C = 32 IPT,
+  //    lane-interleaved (coalesced); a lane finds the run of its first element by bisection, then
+  //    advances it (usually zero steps: slices are longer than 32 keys).
+  constexpr int C = 32 * IPT;
   uint64_t v[IPT];
   {
-    int a = 0;
+    const int e0 = w * C + lane;
+    int a = (k > 1 && e0 < L) ? advance_run(bnd, 0, k, (uint32_t)e0) : 0;
 #pragma unroll
     for (int q = 0; q < IPT; ++q) {
-      const int p = q * T + tid;
-      if (p < L) {
-        if (k > 1) a = advance_run(bnd, a, k, (uint32_t)p);
-        v[q] = ld_stream_u64(keys + s_src[a] + p);
+      const int e = e0 + 32 * q;
+      if (e < L) {
+        while (a + 1 < k && bnd[a + 1] <= (uint32_t)e) ++a;
+        v[q] = ld_stream_u64(keys + s_src[a] + e);
       }
     }
   }
   if (k == 1) {
 #pragma unroll
     for (int q = 0; q < IPT; ++q) {
-      const int p = q * T + tid;
-      if (p < L) o[p] = out_f64 ? from_key(v[q]) : v[q];
+      const int e = w * C + lane + 32 * q;
+      if (e < L) o[e] = out_f64 ? from_key(v[q]) : v[q];
     }
     return;
   }
 #pragma unroll
   for (int q = 0; q < IPT; ++q) {
-    const int p = q * T + tid;
-    if (p < L) buf0[Cfg::pp(p)] = v[q];
+    const int e = w * C + lane + 32 * q;
+    if (e < L) buf0[Cfg::pp(e)] = v[q];
   }
   const int p0 = tid * IPT;
   const int pend = p0 + IPT < L ? p0 + IPT : L;
@@ -326,7 +330,6 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   for (int sh = 0; (1 << sh) < k; ++sh) {
     const int nseq = (k + (1 << sh) - 1) >> sh;
     const int npair = (nseq + 1) >> 1;
-    const bool last = npair == 1;
     int p = p0;
     int m = j0 >> (sh + 1);
     while (p < pend) {
@@ -352,11 +355,28 @@ __global__ void __launch_bounds__(T) k_merge_tile(
       // heads (indices clamped into the pair; an exhausted side is never taken)
       uint64_t a = src[Cfg::pp(s0 + i < s2 - 1 ? s0 + i : s2 - 1)];
       uint64_t b = src[Cfg::pp(s1 + jb < s2 - 1 ? s1 + jb : s2 - 1)];
+      if (stop - p == IPT) {
+        // whole output range inside one pair (the common case): fully unrolled, output slots at
+        // constant offsets from pp(p0) (p0 = IPT tid: no pad inside a thread's range)
+        uint64_t* d = dst + Cfg::pp(p);
+#pragma unroll
+        for (int q = 0; q < IPT; ++q) {
+          const bool ta = jb >= lenB || (i < lenA && a <= b);
+          d[q] = ta ? a : b;
+          i += ta;
+          jb += !ta;
+          int nx = ta ? s0 + i : s1 + jb;
+          nx = nx < s2 - 1 ? nx : s2 - 1;
+          const uint64_t y = src[Cfg::pp(nx)];
+          a = ta ? y : a;
+          b = ta ? b : y;
+        }
+        p = stop;
+      }
       for (; p < stop; ++p) {
         const bool ta = jb >= lenB || (i < lenA && a <= b);
         const uint64_t x = ta ? a : b;
-        dst[Cfg::pp(p)] =
-            last ? (x ^ (xmask & ((uint64_t)((int64_t)(~x) >> 63) | 0x8000000000000000ull))) : x;
+        dst[Cfg::pp(p)] = x;
         i += ta;
         jb += !ta;
         int nx = ta ? s0 + i : s1 + jb;
@@ -374,10 +394,18 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   }
 
   // 4. coalesced store of the tile (src holds the merged, transformed keys)
+  if (out_f64) {
 #pragma unroll
-  for (int q = 0; q < IPT; ++q) {
-    const int p = q * T + tid;
-    if (p < L) __stcs(o + p, src[Cfg::pp(p)]);
+    for (int q = 0; q < IPT; ++q) {
+      const int p = q * T + tid;
+      if (p < L) __stcs(o + p, from_key(src[Cfg::pp(p)]));
+    }
+  } else {
+#pragma unroll
+    for (int q = 0; q < IPT; ++q) {
+      const int p = q * T + tid;
+      if (p < L) __stcs(o + p, src[Cfg::pp(p)]);
+    }
   }
 }
 

@@ -6,7 +6,7 @@ timeout 600 python -m pytest tests/test_gpu_merge_api.py -x -q > gpurun_out/${ta
 timeout 300 python tools/merge_bench.py 30 2,4,8,12,32,128 > gpurun_out/${tag}_bench.jsonl 2>&1
 timeout 300 python tools/merge_bench.py 30 12 normal >> gpurun_out/${tag}_bench.jsonl 2>&1
 timeout 300 python tools/merge_bench.py 30 12 zipf_dup >> gpurun_out/${tag}_bench.jsonl 2>&1
-for lib in paper_conf_ipps_gowanlockk18a_b200/ab/m_*.so; do
+for lib in $(ls paper_conf_ipps_gowanlockk18a_b200/ab/m_*.so 2>/dev/null); do
   echo "== $lib" >> gpurun_out/${tag}_bench.jsonl
   HSORT_LIB=$lib timeout 300 python tools/merge_bench.py 30 2,8,12,128 >> gpurun_out/${tag}_bench.jsonl 2>&1
 done

@@ -338,6 +338,7 @@ def main():
             step_ms.append(ev0.elapsed_time(ev1))
             kt = hs.hsort_get_kernel_times()
             n_active = kt["num_active"]
+            plan = hs.hsort_get_last_plan()
             pass_ms.extend(kt["passes"][:n_active])
             hist_ms.append(kt["hist"])
             other_ms.append(kt["scan"] + kt["copy"] + sum(kt["passes"][n_active:]))
@@ -423,6 +424,7 @@ def main():
             "launches_per_step": n_active,
             "share_of_step": share,
             "hist_ms": statistics.mean(hist_ms) if hist_ms else None,
+            "dominant_digit_elision": plan,
         },
         "e2e": {
             "value": e2e_value,
@@ -439,7 +441,9 @@ def main():
             "link_frac": link_floor_s / (e2e_total / e2e_steps),
         },
         "stages": stages,
-        "gpu_launches": args.steps * 11,
+        # per step: K1, K2, 8 pass launches (inactive ones return at once), final copy; with the
+        # elision: K1, K2, the active passes, final copy, the outlier sort (11), the placement
+        "gpu_launches": args.steps * ((n_active + 15) if plan["elided"] else 11),
         "clocks": sampler.summary(),
         "init_s": t_init,
     }

@@ -179,7 +179,10 @@ int hsort_sort_pairs_u64(const uint64_t* A_host, const uint64_t* V_host, uint64_
  *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times),
  *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never),
  *         "pin_w" (STREAM-mode W: 1 cached pinned, 0 pageable + staging, -1 auto = pinned up to
- *         "pin_w_max_mb" (16 GiB) or when a large enough pinned W is already cached).
+ *         "pin_w_max_mb" (16 GiB) or when a large enough pinned W is already cached),
+ *         "dde" (1 = dominant-digit elision in the GPUSort: when the top active digit has one
+ *         value held by all but a few keys, its LSD pass is dropped and the outliers are sorted
+ *         separately; output-invisible; 0 = off).
  * ------------------------------------------------------------------------------------------- */
 int hsort_set_option(const char* key, int64_t value);
 int hsort_get_option(const char* key, int64_t* value);
@@ -193,6 +196,11 @@ const char* hsort_version(void);
  * p >= *num_active_passes are empty launches), ms[10] = final copy.  Returns the number of
  * entries written (>= 0) or a negative hsort_status.  Call after synchronising the stream. */
 int hsort_get_kernel_times(float* ms, int max_entries, int* num_active_passes);
+
+/* Plan of the last GPUSort on the current device (after synchronising its stream): active LSD
+ * passes run, whether the dominant-digit elision dropped the top digit's pass (option "dde"), and
+ * how many outlier keys it sorted separately. */
+int hsort_get_last_plan(int* num_active_passes, int* elided, uint64_t* n_outliers);
 
 /* Planner (A1): pure host arithmetic, no GPU needed.  device_bytes = usable HBM per GPU
  * (0 -> query the current device).  Fills *out; HSORT_ERR_INVALID on bad arguments. */

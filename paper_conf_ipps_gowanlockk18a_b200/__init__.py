@@ -99,6 +99,7 @@ SIGNATURES = {
     "hsort_device_count": ([], _I),
     "hsort_get_kernel_times": ([ctypes.POINTER(ctypes.c_float), _I, ctypes.POINTER(_I)], _I),
     "hsort_device_upper_bounds": ([_P, _U64, _P, _U64, _P, _P], _I),
+    "hsort_get_last_plan": ([ctypes.POINTER(_I), ctypes.POINTER(_I), ctypes.POINTER(_U64)], _I),
     "hsort_host_upper_bounds": ([_P, _U64, _P, _U64, _P], _I),
 }
 
@@ -378,6 +379,13 @@ def hsort_host_corank(keys: np.ndarray, off, o: int) -> np.ndarray:
     r = np.zeros(of.size - 1, dtype=np.uint64)
     _check(lib().hsort_host_corank(keys.ctypes.data, of.ctypes.data, of.size - 1, o, r.ctypes.data))
     return r
+
+
+def hsort_get_last_plan() -> dict:
+    """Plan of the last GPUSort on the current device: passes run, elision, outliers."""
+    na, el, no = _I(), _I(), _U64()
+    _check(lib().hsort_get_last_plan(ctypes.byref(na), ctypes.byref(el), ctypes.byref(no)))
+    return {"num_active": na.value, "elided": bool(el.value), "n_outliers": no.value}
 
 
 def hsort_get_kernel_times() -> dict:

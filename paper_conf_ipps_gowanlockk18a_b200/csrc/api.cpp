@@ -114,6 +114,7 @@ struct Options {
       {"merge_chunk", 1ll << 26},    // GPU merge output chunk (keys)
       {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
+      {"dde", 1},                    // 1: dominant-digit elision in the GPUSort
       {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
       {"pin_w", -1},                 // STREAM W: 1 cached pinned, 0 pageable, -1 pinned if <= pin_w_max_mb
       {"pin_w_max_mb", 16384},       // auto pinning limit: pinning runs at ~2.5 GB/s
@@ -1403,6 +1404,7 @@ int hsort_set_option(const char* key, int64_t value) {
     return HSORT_ERR_BUSY;
   }
   S().opt.v[k] = value;
+  if (k == "dde") g_dde_enabled = value != 0;
   if (k == "kernel_timing") {
     return guarded([&]() -> int {
       for (auto& g : S().gpus) {
@@ -1423,6 +1425,19 @@ int hsort_get_kernel_times(float* ms, int max_entries, int* num_active_passes) {
     GpuCtx& g = current_ctx();
     if (num_active_passes) *num_active_passes = g.rs.h_plan ? g.rs.h_plan->num_active : 0;
     return radix_kernel_times(g.rs, ms, max_entries);
+  });
+}
+
+int hsort_get_last_plan(int* num_active_passes, int* elided, uint64_t* n_outliers) {
+  int rc = check_ready();
+  if (rc) return rc;
+  return guarded([&]() -> int {
+    GpuCtx& g = current_ctx();
+    const RadixPlan* P = g.rs.h_plan;
+    if (num_active_passes) *num_active_passes = P ? P->num_active : 0;
+    if (elided) *elided = P ? P->dde : 0;
+    if (n_outliers) *n_outliers = P && P->dde ? P->dde_n_out : 0;
+    return HSORT_OK;
   });
 }
 

@@ -21,6 +21,26 @@ struct RadixPlan {
   int32_t match_mask;   // bit p: pass p ranks with MATCH.ANY (few distinct digits per warp),
                         // else with the 8-ballot multisplit
   int32_t lb_parity;    // 32-bit look-back mode: status array of pass p is (lb_parity + p) & 1
+  // Dominant-digit elision: the top active digit L has one value v held by all but
+  // n_out <= cap keys.  Its pass is dropped; pass dde_pass (the new last pass, digit P) diverts the
+  // n_out outliers to a side buffer and places the others by digit P alone; the outliers are
+  // sorted separately and written to out[0, n_less) and out[n - (n_out - n_less), n).
+  int32_t dde;          // 1: active
+  int32_t dde_digit;    // L
+  uint32_t dde_value;   // v
+  int32_t dde_pass;     // index of the diverting pass (num_active - 1)
+  uint64_t dde_n_out;   // outliers (n - count of v)
+  uint64_t dde_n_less;  // outliers whose digit L is below v
+  int32_t dde_k1;       // 1: K1 already counted the outliers' digit-P histogram (L = 7, P = 6)
+};
+
+// Device state of the dominant-digit elision, zeroed per sort.
+struct DdeState {
+  uint32_t n_out;           // outliers diverted so far (append counter of the side buffer)
+  uint32_t guess;           // K1: top digit of the first key (the dominant value's guess)
+  uint32_t hist_out[256];   // digit-P histogram of the outliers, counted by pass 0
+  uint32_t hist_k1[256];    // K1's count: digit 6 of the keys whose top digit != guess (used when
+                            // the plan's dde_k1 says the guess was v, L = 7 and P = 6)
 };
 
 struct RadixScratch {
@@ -46,12 +66,19 @@ struct RadixScratch {
   // ev[0] before K1, ev[1] after K1, ev[2] after K2, ev[3+p] after pass p, ev[11] after copy
   bool timing = false;
   cudaEvent_t ev[12] = {};
+  // dominant-digit elision: state + side buffer (2 x side_cap keys: outliers and sort scratch)
+  DdeState* dde = nullptr;
+  uint64_t* side = nullptr;
+  uint64_t side_cap = 0;
+  RadixScratch* sub = nullptr;  // scratch of the outlier sort (its own look-back rows and plan)
 };
 constexpr int kNumKernelEvents = 12;
 
 constexpr int kRadixTile = 4096;  // keys per onesweep tile (THREADS x ITEMS), see radix.cu
 constexpr int kKvTile = 4032;     // pairs per key/value onesweep tile (576 x 7), see radix.cu
 
+// dominant-digit elision on/off (option "dde", default on)
+extern bool g_dde_enabled;
 cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n);
 cudaError_t radix_set_timing(RadixScratch& s, bool on);
 // durations (ms) of [K1, K2, pass0..pass7, final copy] of the last timed sort; returns count

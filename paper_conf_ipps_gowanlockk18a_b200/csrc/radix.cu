@@ -173,11 +173,14 @@ __device__ __forceinline__ uint64_t scan256_excl(uint64_t v, uint64_t* s_warp /*
 }
 
 // K2: bin bases + pass plan.  One CTA of 256 threads.
+// dde_cap > 0: the dominant-digit elision may be planned (outliers <= dde_cap).
 __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ hist,
                                                    uint64_t* __restrict__ bin_base,
                                                    RadixPlan* __restrict__ plan, uint64_t n,
                                                    int in_eq_out, int in_f64, int out_f64,
-                                                   uint32_t* __restrict__ lb_state) {
+                                                   uint32_t* __restrict__ lb_state,
+                                                   uint64_t dde_cap = 0,
+                                                   const DdeState* __restrict__ dde = nullptr) {
   __shared__ uint64_t s_warp[8];
   __shared__ int s_nz[kDigits];
   __shared__ float s_dist[kDigits][8];
@@ -204,6 +207,42 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
     for (int p = 0; p < kDigits; ++p)
       if (s_nz[p] > 1) P.digit[na++] = p;
     for (int p = na; p < kDigits; ++p) P.digit[p] = -1;
+    P.dde = 0;
+    P.dde_digit = -1;
+    P.dde_value = 0;
+    P.dde_pass = -1;
+    P.dde_n_out = 0;
+    P.dde_n_less = 0;
+    P.dde_k1 = 0;
+    if (dde_cap && na >= 3) {
+      // top active digit L: dominant value v; elide its pass if the outliers fit the side buffer
+      // and the remaining na - 1 passes still end in out without a final copy
+      const int L = P.digit[na - 1];
+      uint64_t best = 0, below = 0, below_best = 0;
+      uint32_t v = 0;
+      for (int b = 0; b < kRadix; ++b) {
+        const uint64_t c = hist[L * kRadix + b];
+        if (c > best) {
+          best = c;
+          v = (uint32_t)b;
+          below_best = below;
+        }
+        below += c;
+      }
+      const uint64_t n_out = n - best;
+      if (n_out <= dde_cap && (!in_eq_out || ((na - 1) & 1) == 0)) {
+        P.dde = 1;
+        P.dde_digit = L;
+        P.dde_value = v;
+        --na;
+        P.dde_pass = na - 1;
+        P.digit[na] = -1;
+        P.dde_n_out = n_out;
+        P.dde_n_less = below_best;
+        // K1 counted the outliers' digit-6 histogram if the guess (key 0's top digit) was right
+        P.dde_k1 = (dde && L == 7 && P.digit[na - 1] == 6 && v == dde->guess) ? 1 : 0;
+      }
+    }
     P.num_active = na;
     P.copy_src = -1;
     P.copy_in_f64 = 0;
@@ -261,6 +300,12 @@ __global__ void k_force_plan(RadixPlan* plan, int digit, uint32_t* lb_state) {
   P.dst[0] = 1;
   P.copy_src = -1;
   P.copy_in_f64 = P.copy_out_f64 = P.match_mask = 0;
+  P.dde = 0;
+  P.dde_digit = -1;
+  P.dde_value = 0;
+  P.dde_pass = -1;
+  P.dde_n_out = P.dde_n_less = 0;
+  P.dde_k1 = 0;
   *plan = P;
 }
 
@@ -812,11 +857,16 @@ __global__ void __launch_bounds__(THREADS, MINB) k_onesweep_tma(uint64_t* in, ui
 
 // K1 v2: per-warp entropy probe picks, for each digit, either direct shared atomics (spread
 // digits) or the register run-length cache (low-entropy digits, e.g. the exponent byte).
-template <bool IN_F64, uint32_t MASK, int SH = 0>
+// DDE: also count digit 6 of the keys whose top digit differs from `guess` (the top digit of the
+// first key) into hout -- the elision's outlier histogram for its common case L = 7, P = 6
+// (DESIGN.md §6d), so pass 0 does not have to count it.
+template <bool IN_F64, uint32_t MASK, int SH = 0, bool DDE = false>
 __device__ __forceinline__ void hist2_key(uint64_t k, uint32_t* sh, uint32_t* cd, uint32_t* cc,
-                                          uint32_t mask) {
+                                          uint32_t mask, uint32_t guess = 0,
+                                          uint32_t* hout = nullptr) {
   if (IN_F64) k = to_key(k);
   const uint32_t lo = (uint32_t)k, hi = (uint32_t)(k >> 32);
+  if (DDE && (hi >> 24) != guess) atomicAdd(&hout[(hi >> 16) & 255u], 1u);
 #pragma unroll
   for (int p = 0; p < kDigits; ++p) {
     const uint32_t d = ((p < 4 ? lo : hi) >> (8 * (p & 3))) & 255u;
@@ -835,22 +885,23 @@ __device__ __forceinline__ void hist2_key(uint64_t k, uint32_t* sh, uint32_t* cd
   }
 }
 
-template <bool IN_F64, uint32_t MASK, int SH = 0>
+template <bool IN_F64, uint32_t MASK, int SH = 0, bool DDE = false>
 __device__ __forceinline__ void hist2_loop(const uint64_t* base, uint64_t pairs, uint64_t i,
                                            uint64_t stride, uint32_t* sh, uint32_t* cd,
-                                           uint32_t* cc, uint32_t mask) {
+                                           uint32_t* cc, uint32_t mask, uint32_t guess = 0,
+                                           uint32_t* hout = nullptr) {
   for (; i + 3 * stride < pairs; i += 4 * stride) {
     uint64_t a[8];
 #pragma unroll
     for (int u = 0; u < 4; ++u) ld_stream2(base + 2 * (i + u * stride), a[2 * u], a[2 * u + 1]);
 #pragma unroll
-    for (int u = 0; u < 8; ++u) hist2_key<IN_F64, MASK, SH>(a[u], sh, cd, cc, mask);
+    for (int u = 0; u < 8; ++u) hist2_key<IN_F64, MASK, SH, DDE>(a[u], sh, cd, cc, mask, guess, hout);
   }
   for (; i < pairs; i += stride) {
     uint64_t a0, a1;
     ld_stream2(base + 2 * i, a0, a1);
-    hist2_key<IN_F64, MASK, SH>(a0, sh, cd, cc, mask);
-    hist2_key<IN_F64, MASK, SH>(a1, sh, cd, cc, mask);
+    hist2_key<IN_F64, MASK, SH, DDE>(a0, sh, cd, cc, mask, guess, hout);
+    hist2_key<IN_F64, MASK, SH, DDE>(a1, sh, cd, cc, mask, guess, hout);
   }
 }
 
@@ -913,9 +964,10 @@ __global__ void __launch_bounds__(kHistThreads) k_hist2(const uint64_t* __restri
 #endif
 constexpr int kHist3Copies = HSORT_HIST_COPIES;
 constexpr int kHist3Threads = HSORT_HIST_THREADS;
-template <bool IN_F64, int THREADS, int COPIES>
+template <bool IN_F64, int THREADS, int COPIES, bool DDE = false>
 __global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ src, uint64_t n,
-                                                       uint64_t* __restrict__ hist) {
+                                                       uint64_t* __restrict__ hist,
+                                                       DdeState* __restrict__ dde = nullptr) {
   constexpr int SHC = COPIES == 16 ? 4 : 3;
   extern __shared__ uint32_t sh3[];  // [8 * 256][COPIES]
   for (int i = threadIdx.x; i < kDigits * kRadix * COPIES; i += THREADS) sh3[i] = 0;
@@ -944,13 +996,23 @@ __global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ 
       if (__popc(leaders) <= 4) mask |= 1u << p;
     }
   }
-  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist2_key<IN_F64, 0xFFFFFFFFu, SHC>(src[0], sh, cd, cc, 0xFF);
-  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else if (mask == 0u) hist2_loop<IN_F64, 0u, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else hist2_loop<IN_F64, 0xFFFFFFFFu, SHC>(base, pairs, i0, stride, sh, cd, cc, mask);
+  uint32_t guess = 0;
+  uint32_t* hout = nullptr;
+  if (DDE) {
+    uint64_t k0 = n ? src[0] : 0;
+    if (IN_F64) k0 = to_key(k0);
+    guess = (uint32_t)(k0 >> 56);
+    hout = dde->hist_k1;
+    if (blockIdx.x == 0 && threadIdx.x == 0) dde->guess = guess;
+  }
+  if (head && blockIdx.x == 0 && threadIdx.x == 0)
+    hist2_key<IN_F64, 0xFFFFFFFFu, SHC, DDE>(src[0], sh, cd, cc, 0xFF, guess, hout);
+  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u, SHC, DDE>(base, pairs, i0, stride, sh, cd, cc, mask, guess, hout);
+  else if (mask == 0u) hist2_loop<IN_F64, 0u, SHC, DDE>(base, pairs, i0, stride, sh, cd, cc, mask, guess, hout);
+  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u, SHC, DDE>(base, pairs, i0, stride, sh, cd, cc, mask, guess, hout);
+  else hist2_loop<IN_F64, 0xFFFFFFFFu, SHC, DDE>(base, pairs, i0, stride, sh, cd, cc, mask, guess, hout);
   if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == THREADS - 1)
-    hist2_key<IN_F64, 0xFFFFFFFFu, SHC>(base[m - 1], sh, cd, cc, 0xFF);
+    hist2_key<IN_F64, 0xFFFFFFFFu, SHC, DDE>(base[m - 1], sh, cd, cc, 0xFF, guess, hout);
 #pragma unroll
   for (int p = 0; p < kDigits; ++p)
     if (cc[p]) atomicAdd(&sh[(p * kRadix + cd[p]) << SHC], cc[p]);
@@ -982,6 +1044,17 @@ __global__ void k_final_copy(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_
     if (fin != fout) v = fin ? to_key(v) : from_key(v);
     out[i] = v;
     if (vs && vs != vout) vout[i] = vs[i];
+  }
+}
+
+// Dominant-digit elision, last step: the sorted outliers (side[0, n_out), internal keys) go to
+// out[0, n_less) (digit L below the dominant value) and out[n - (n_out - n_less), n) (above).
+__global__ void k_dde_place(const uint64_t* __restrict__ side, uint64_t n_out, uint64_t n_less,
+                            uint64_t* __restrict__ out, uint64_t n, int out_f64) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_out;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t v = side[i];
+    out[i < n_less ? i : n - n_out + i] = out_f64 ? from_key(v) : v;
   }
 }
 
@@ -1026,7 +1099,7 @@ int hist_variant() {
 }
 
 cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
-                        uint64_t* hist, cudaStream_t st) {
+                        uint64_t* hist, cudaStream_t st, DdeState* dde = nullptr) {
   int dev = 0;
   cudaGetDevice(&dev);
   uint64_t want = (n / 2 + kHistThreads * 8 - 1) / (kHistThreads * 8);
@@ -1043,12 +1116,16 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
     constexpr int smem = kDigits * kRadix * kHist3Copies * 4;
     auto kt = k_hist3<true, kHist3Threads, kHist3Copies>;
     auto kf = k_hist3<false, kHist3Threads, kHist3Copies>;
+    auto kdt = k_hist3<true, kHist3Threads, kHist3Copies, true>;
+    auto kdf = k_hist3<false, kHist3Threads, kHist3Copies, true>;
     static int per_sm[64] = {0};  // resident CTAs per SM, per device
     if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
     if (!per_sm[dev]) {
       cudaError_t e;
       if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
       if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(kdt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(kdf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
       int b = 0;
       if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, kHist3Threads, smem)) != cudaSuccess) return e;
       per_sm[dev] = b > 0 ? b : 1;
@@ -1056,8 +1133,13 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
     const uint64_t want3 = (n / 2 + kHist3Threads * 8 - 1) / (kHist3Threads * 8);
     const uint64_t cap3 = (uint64_t)num_sms(dev) * per_sm[dev];
     const int grid3 = (int)(want3 < 1 ? 1 : (want3 > cap3 ? cap3 : want3));
-    if (in_f64) kt<<<grid3, kHist3Threads, smem, st>>>(in, n, hist);
-    else kf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist);
+    if (dde) {
+      if (in_f64) kdt<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, dde);
+      else kdf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, dde);
+    } else {
+      if (in_f64) kt<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, nullptr);
+      else kf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, nullptr);
+    }
   }
   return cudaGetLastError();
 }
@@ -1270,7 +1352,10 @@ __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64
 
 // KV: key/value pairs (S§8(f) #3): the 64-bit value of each key rides along -- second TMA copy
 // into a value stage, scattered to the key's stage slot, written out to the key's position.
-template <int CT, int ITEMS, bool IN_F64, bool KV = false>
+// DM (dominant-digit elision): 0 none; 1 pass 0 of an elided sort (counts the
+// outliers' digit-P histogram); 2 the elided sort's last pass (diverts the outliers).  The host
+// picks DM per launch after reading K2's plan, so the DM = 0 kernel carries no elision code.
+template <int CT, int ITEMS, bool IN_F64, bool KV = false, int DM = 0>
 __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in, uint64_t* out, uint64_t* tmp,
                                                        uint64_t* vin, uint64_t* vout, uint64_t* vtmp,
                                                        uint64_t n, const RadixPlan* __restrict__ plan,
@@ -1278,7 +1363,10 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
                                                        uint64_t* __restrict__ lookback,
                                                        uint32_t* __restrict__ tile_ctr, int p,
                                                        int out_f64, uint64_t lb_half,
-                                                       uint64_t lb_rows) {
+                                                       uint64_t lb_rows,
+                                                       const uint64_t* __restrict__ hist = nullptr,
+                                                       DdeState* __restrict__ dde = nullptr,
+                                                       uint64_t* __restrict__ side = nullptr) {
   using L = WsSmem<CT, ITEMS, KV>;
   constexpr int TILE = L::TILE;
   constexpr int CW = L::CW;
@@ -1307,6 +1395,13 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   uint64_t* __restrict__ vdst = KV ? pick(plan->dst[p], vin, vout, vtmp) : nullptr;
   const bool use_match = (plan->match_mask >> p) & 1;
   const bool inv = out_f64 && (p == na - 1);
+  // dominant-digit elision: pass 0 counts the outliers' digit-P histogram; the last pass diverts
+  // the outliers (digit L != v) to the side buffer and ranks the rest by digit P
+  static_assert(DM == 0 || !KV, "the elision is keys-only");
+  constexpr bool dde_here = DM == 2;
+  const int sh_l = DM ? 8 * plan->dde_digit : 0;
+  const uint32_t v_l = DM ? plan->dde_value : 0u;
+  const int sh_p = DM ? 8 * plan->digit[plan->dde_pass] : 0;
   uint32_t* lb32 = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p) & 1) * lb_half;
   uint32_t* lb32_next = (uint32_t*)lookback + (uint64_t)((plan->lb_parity + p + 1) & 1) * lb_half;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -1349,8 +1444,31 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     // offsets to the compute warps; then claim tile j+2 and issue its TMA into the stage that
     // tile j-1 used, once every compute warp has written tile j-1 out.
     uint64_t base[8];
+    if (dde_here) {
+      // bases of the dominant keys: n_less + exclusive scan over digits of hist[P] - hist_out
+      uint64_t c[8], tot = 0;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) base[q] = bin_base[digit * kRadix + lane * 8 + q];
+      for (int q = 0; q < 8; ++q) {
+        const uint32_t* ho = plan->dde_k1 ? dde->hist_k1 : dde->hist_out;
+        c[q] = hist[digit * kRadix + lane * 8 + q] - ho[lane * 8 + q];
+        tot += c[q];
+      }
+      uint64_t incl = tot;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += y;
+      }
+      uint64_t run = plan->dde_n_less + incl - tot;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        base[q] = run;
+        run += c[q];
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < 8; ++q) base[q] = bin_base[digit * kRadix + lane * 8 + q];
+    }
 #ifdef HSORT_PHASE_TIMING
     unsigned long long t_wait = 0, t_lb = 0, n_lb = 0;
 #endif
@@ -1434,7 +1552,11 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
     const uint64_t* vsb = vstage + (size_t)(jj % 3) * TILE;
     const uint64_t rem = n - tile * (uint64_t)TILE;
-    const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+    int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
+    if (dde_here) {  // diverted outliers leave the tile: its keys fill stage[0, sum of counts)
+      const uint32_t c = s_cnt[(jj & 1) * kRadix + kRadix - 1];
+      tile_n = (int)((c >> 16) + (c & 0xFFFFu));
+    }
     auto wo_full = [&](auto inv_tag) {
       constexpr bool INV = decltype(inv_tag)::value;
 #pragma unroll
@@ -1449,7 +1571,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
         if (KV) st_global_u64((uint64_t)(vdst + tid + g + q * THREADS), vsb[tid + q * THREADS]);
       }
     };
-    if (tile_n == TILE) {
+    if (tile_n == TILE) {  // (elision: tile_n is the count of keys left after the diversion)
       if (inv) wo_full(std::true_type{});
       else wo_full(std::false_type{});
     } else {
@@ -1465,6 +1587,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   };
   // one tile: load from the stage, per-warp digit counts, tile aggregate + scan, warp ranking,
   // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
+  // DM (compile-time): 0 no elision work, 1 count the outliers' digit-P histogram (pass 0),
+  // 2 divert the outliers (the elision's last pass; never FULL)
   auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, uint64_t* sb, uint64_t* vsb) {
     constexpr bool FULL = decltype(full_tag)::value;
     const uint64_t tbase = tile * (uint64_t)TILE;
@@ -1474,6 +1598,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     uint64_t k[ITEMS];
     uint64_t vv[KV ? ITEMS : 1];
     uint32_t dd[ITEMS];
+    uint32_t omask = 0;  // elision: items of this lane that are outliers
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int jj = wofs + i * 32;
@@ -1487,6 +1612,23 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       k[i] = IN_F64 ? to_key(v) : v;
       const bool valid = FULL || jj < tile_n;
       dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
+      if (DM != 0) omask |= (uint32_t)(valid && ((uint32_t)(k[i] >> sh_l) & 255u) != v_l) << i;
+    }
+    // outliers of the elision (rare; branch-free above): one vote per warp, then the slow path
+    bool w_out = false;
+    if (DM != 0) {
+      w_out = __any_sync(0xffffffffu, omask != 0);
+      if (w_out) {
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i)
+          if ((omask >> i) & 1u) {
+            if (DM == 1) atomicAdd(&dde->hist_out[(uint32_t)(k[i] >> sh_p) & 255u], 1u);
+            if (DM == 2) {
+              side[atomicAdd(&dde->n_out, 1u)] = k[i];
+              dd[i] = kRadix;
+            }
+          }
+      }
     }
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) atomicAdd(&wh[dd[i]], 1u);
@@ -1536,6 +1678,10 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
         for (int i = NM; i < ITEMS; ++i) peers[i] = peer_bit(peers[i], dd[i], 1u << b);
       }
+      if (FULL && DM == 2 && w_out) {  // diverted items carry digit 256: separate them (bit 8)
+#pragma unroll
+        for (int i = NM; i < ITEMS; ++i) peers[i] = peer_bit(peers[i], dd[i], 1u << 8);
+      }
     }
 #if HSORT_FAKE == 2
 #pragma unroll
@@ -1554,13 +1700,15 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
-      rr[i] = (lane == leader && (FULL || dd[i] < kRadix)) ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i])) : 0u;
+      rr[i] = (lane == leader && ((FULL && DM != 2) || dd[i] < kRadix))
+                  ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i]))
+                  : 0u;
     }
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
       const uint32_t r = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
-      if (FULL || dd[i] < kRadix) {
+      if ((FULL && DM != 2) || dd[i] < kRadix) {
         sb[r] = k[i];
         if (KV) vsb[r] = vv[i];
       }
@@ -1631,7 +1779,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       lb32_next[rr * kRadix + tid] = 0;
 }
 
-template <int CT, int ITEMS, bool KV = false>
+template <int CT, int ITEMS, bool KV = false, int DM = 0>
 cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t* vin, uint64_t* vout,
                            uint64_t* vtmp, uint64_t n, RadixScratch& s, int p, bool first_in_f64,
                            bool out_f64, cudaStream_t st) {
@@ -1639,8 +1787,9 @@ cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t*
   static int blocks_per_sm[64] = {0};
   int dev = 0;
   cudaGetDevice(&dev);
-  auto kt = k_onesweep_ws<CT, ITEMS, true, KV>;
-  auto kf = k_onesweep_ws<CT, ITEMS, false, KV>;
+  constexpr bool dde = DM != 0;
+  auto kt = k_onesweep_ws<CT, ITEMS, true, KV, DM>;
+  auto kf = k_onesweep_ws<CT, ITEMS, false, KV, DM>;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   if (!blocks_per_sm[dev]) {
     cudaError_t e;
@@ -1654,14 +1803,17 @@ cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t*
   if (tiles > s.max_tiles) return cudaErrorInvalidValue;
   uint64_t grid = (uint64_t)num_sms(dev) * blocks_per_sm[dev];
   if (grid > tiles) grid = tiles ? tiles : 1;
+  const uint64_t* h = dde ? s.hist : nullptr;
+  DdeState* ds = dde ? s.dde : nullptr;
+  uint64_t* sd = dde ? s.side : nullptr;
   if (first_in_f64)
     kt<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, vin, vout, vtmp, n, s.plan, s.bin_base,
                                              s.lookback, s.tile_ctr, p, out_f64 ? 1 : 0,
-                                             s.max_tiles * kRadix, s.lb_rows);
+                                             s.max_tiles * kRadix, s.lb_rows, h, ds, sd);
   else
     kf<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, vin, vout, vtmp, n, s.plan, s.bin_base,
                                              s.lookback, s.tile_ctr, p, out_f64 ? 1 : 0,
-                                             s.max_tiles * kRadix, s.lb_rows);
+                                             s.max_tiles * kRadix, s.lb_rows, h, ds, sd);
   return cudaGetLastError();
 }
 
@@ -1695,15 +1847,22 @@ cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t
 }
 
 cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
-                        int p, bool first_in_f64, bool out_f64, cudaStream_t st) {
+                        int p, bool first_in_f64, bool out_f64, cudaStream_t st, int dm = 0) {
   uint32_t ep = 0;
   cudaError_t e = next_epoch(s, st, &ep);
   if (e != cudaSuccess) return e;
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const int v = pass_kernel(in, out, tmp);
-  if (v == 2 && s.lb_mode == 2)
+  if (v == 2 && s.lb_mode == 2) {
+    if (dm == 1)
+      return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS, false, 1>(in, out, tmp, nullptr, nullptr, nullptr,
+                                                                   n, s, p, first_in_f64, out_f64, st);
+    if (dm == 2)
+      return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS, false, 2>(in, out, tmp, nullptr, nullptr, nullptr,
+                                                                   n, s, p, first_in_f64, out_f64, st);
     return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS>(in, out, tmp, nullptr, nullptr, nullptr, n, s, p,
                                                        first_in_f64, out_f64, st);
+  }
   // look-back window 4: measured best of 1..32
   if (v >= 1) {
     if (s.lb_mode == 2)
@@ -1806,11 +1965,30 @@ void radix_scratch_release(RadixScratch& s) {
   if (s.lookback) cudaFree(s.lookback);
   if (s.small) cudaFree(s.small);
   if (s.h_plan) cudaFreeHost(s.h_plan);
+  if (s.dde) cudaFree(s.dde);
+  if (s.side) cudaFree(s.side);
+  if (s.sub) {
+    radix_scratch_release(*s.sub);
+    delete s.sub;
+  }
   s = RadixScratch();
 }
 
-cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
-                       uint64_t n, bool in_f64, bool out_f64, cudaStream_t st) {
+#ifndef HSORT_DDE_MIN_N
+#define HSORT_DDE_MIN_N (1ull << 22)  // below this the outlier sort's fixed cost outweighs a pass
+#endif
+bool g_dde_enabled = true;  // hsort_set_option("dde", 0) turns the elision off (A/B, tests)
+
+// Side buffer capacity for n keys: the outliers a plan may divert (K2 checks n_out <= cap).
+uint64_t dde_cap(uint64_t n) {
+  uint64_t c = n >> 13;  // U[0,1) keeps ~n 2^-15 keys below the top byte's dominant value
+  if (c < (1ull << 12)) c = 1ull << 12;
+  if (c > (1ull << 20)) c = 1ull << 20;
+  return c;
+}
+
+cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
+                            uint64_t n, bool in_f64, bool out_f64, cudaStream_t st, bool allow_dde) {
   if (n == 0) return cudaSuccess;
   cudaError_t e = radix_scratch_reserve(s, n);
   if (e != cudaSuccess) return e;
@@ -1818,26 +1996,79 @@ cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uin
   auto mark = [&](int i) -> cudaError_t {
     return s.timing ? cudaEventRecord(s.ev[i], st) : cudaSuccess;
   };
+  const int kernel = pass_kernel(in, out, tmp);
+  // the elision lives in the warp-specialised pass (32-bit look-back words, n <= 2^30); out of
+  // place only (in place, 7 of 8 passes would end in the scratch buffer and need a copy)
+  const bool dde = allow_dde && g_dde_enabled && kernel == 2 && in != out &&
+                   n >= HSORT_DDE_MIN_N && n <= (1ull << 30);
+  uint64_t cap = 0;
+  if (dde) {
+    cap = dde_cap(n);
+    if (!s.dde && (e = cudaMalloc(&s.dde, sizeof(DdeState))) != cudaSuccess) return e;
+    if (s.side_cap < cap) {
+      if (s.side) cudaFree(s.side);
+      s.side = nullptr;
+      s.side_cap = 0;
+      if ((e = cudaMalloc(&s.side, 2 * cap * sizeof(uint64_t))) != cudaSuccess) return e;
+      s.side_cap = cap;
+    }
+    if (!s.sub) s.sub = new RadixScratch();
+    if ((e = cudaMemsetAsync(s.dde, 0, sizeof(DdeState), st)) != cudaSuccess) return e;
+  }
   if ((e = cudaMemsetAsync(s.small, 0, s.small_zero_bytes, st)) != cudaSuccess) return e;
   if ((e = mark(0)) != cudaSuccess) return e;
-  if ((e = launch_hist(s, in, n, in_f64, s.hist, st)) != cudaSuccess) return e;
+  if ((e = launch_hist(s, in, n, in_f64, s.hist, st, dde ? s.dde : nullptr)) != cudaSuccess) return e;
   if ((e = mark(1)) != cudaSuccess) return e;
-  if ((e = select_lb_mode(s, pass_kernel(in, out, tmp), n, st)) != cudaSuccess) return e;
+  if ((e = select_lb_mode(s, kernel, n, st)) != cudaSuccess) return e;
   k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
-                                 out_f64 ? 1 : 0, s.lb_state);
+                                 out_f64 ? 1 : 0, s.lb_state, cap, dde ? s.dde : nullptr);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   if ((e = mark(2)) != cudaSuccess) return e;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dde) {
+    // the host picks each pass's kernel (elision mode) from K2's plan: one short sync
+    if ((e = cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+      return e;
+    if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return e;
+    const RadixPlan P = *s.h_plan;
+    if (P.dde) {
+      for (int p = 0; p < kDigits; ++p) {
+        if (p < P.num_active) {
+          const int dm = p == P.dde_pass ? 2 : (p == 0 && !P.dde_k1 ? 1 : 0);
+          if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st, dm)) != cudaSuccess)
+            return e;
+        }
+        if ((e = mark(3 + p)) != cudaSuccess) return e;
+      }
+      k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
+      if ((e = cudaGetLastError()) != cudaSuccess) return e;
+      // the outliers (internal keys, unordered) -> sorted on their own scratch -> both ends of out
+      const uint64_t n_out = P.dde_n_out;
+      if ((e = radix_sort_impl(*s.sub, s.side, s.side, s.side + cap, n_out, false, false, st, false)) !=
+          cudaSuccess)
+        return e;
+      if (n_out) {
+        k_dde_place<<<num_sms(dev), 256, 0, st>>>(s.side, n_out, P.dde_n_less, out, n, out_f64 ? 1 : 0);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+      }
+      return mark(11);
+    }
+  }
   for (int p = 0; p < kDigits; ++p) {
     if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st)) != cudaSuccess)
       return e;
     if ((e = mark(3 + p)) != cudaSuccess) return e;
   }
-  int dev = 0;
-  cudaGetDevice(&dev);
   k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   if ((e = mark(11)) != cudaSuccess) return e;
   return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);
+}
+
+cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
+                       uint64_t n, bool in_f64, bool out_f64, cudaStream_t st) {
+  return radix_sort_impl(s, in_c, out, tmp, n, in_f64, out_f64, st, true);
 }
 
 // Key/value GPUSort (S§8(f) #3): K1/K2 on the keys as in radix_sort, then every active digit

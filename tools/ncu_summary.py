@@ -57,20 +57,23 @@ ap.add_argument("--n", type=int, required=True)
 ap.add_argument("--out-md", required=True)
 ap.add_argument("--out-json", default=None)
 ap.add_argument("--steps", type=int, default=0,
-                help="keep only the first S device-sort steps (launches up to the S-th k_final_copy)")
+                help="keep only the first S device-sort steps (a step starts at a K1 launch on the "
+                     "first K1's grid; the elision's outlier sort runs its own smaller K1)")
 a = ap.parse_args()
 rows = launches(a.csv)
 if a.steps:
+    k1 = next((r for r in rows if r[0].startswith("k_hist")), None)
     seen, keep = 0, []
     for r in rows:
+        if k1 and r[0].startswith("k_hist") and r[2] == k1[2]:
+            seen += 1
+            if seen > a.steps:
+                break
         keep.append(r)
-        seen += r[0].startswith("k_final_copy")
-        if seen == a.steps:
-            break
     rows = keep
 agg = OrderedDict()
 for k, ns, g, b in rows:
-    e = agg.setdefault(k, [0, 0.0, g, b])
+    e = agg.setdefault((k, g), [0, 0.0, g, b])
     e[0] += 1
     e[1] += ns
 tot = sum(e[1] for e in agg.values())
@@ -78,7 +81,7 @@ md = ["# ncu launch list summary", "", f"source: `{a.csv}` (gpu__time_duration.s
       "cold-cache, serialised launches: compare shares, not absolutes)"
       + (f"; first {a.steps} device-sort steps of the bench command (warm-up + timed)" if a.steps else ""), "",
       "| kernel | launches | total ms | mean ms | share | grid | block |", "|---|---|---|---|---|---|---|"]
-for k, (c, ns, g, b) in sorted(agg.items(), key=lambda x: -x[1][1]):
+for (k, _), (c, ns, g, b) in sorted(agg.items(), key=lambda x: -x[1][1]):
     md.append(f"| `{k}` | {c} | {ns/1e6:.3f} | {ns/1e6/c:.3f} | {ns/tot:.1%} | {g} | {b} |")
 js = {"n": a.n}
 for rep in a.reports:

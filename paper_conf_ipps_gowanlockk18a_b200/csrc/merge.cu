@@ -60,11 +60,58 @@ __device__ __forceinline__ uint64_t upper_bound(const uint64_t* a, uint64_t lo, 
 }
 
 // K4.  ranks[b*k + j] = co-rank of run j at output position o_b = min(b*step, total).
+// first index i in [0, r] with a[i] >= v, given a[r] >= v (or r = end): gallop back from r
+__device__ __forceinline__ uint64_t lower_bound_back(const uint64_t* a, uint64_t r, uint64_t v) {
+  uint64_t hi = r, step = 1;
+  while (hi > 0 && a[hi - 1] >= v) {  // a[hi - 1] >= v: the bound lies further back
+    const uint64_t lo = hi > step ? hi - step : 0;
+    if (a[lo] < v) {  // bound in (lo, hi - 1]
+      uint64_t l = lo + 1, h = hi - 1;
+      while (l < h) {
+        const uint64_t m = l + ((h - l) >> 1);
+        if (a[m] < v) l = m + 1;
+        else h = m;
+      }
+      return l;
+    }
+    hi = lo;
+    step <<= 1;
+  }
+  return hi;
+}
+// first index i in [r, len] with a[i] > v, given a[r - 1] <= v (or r = 0): gallop forward
+__device__ __forceinline__ uint64_t upper_bound_fwd(const uint64_t* a, uint64_t r, uint64_t len,
+                                                    uint64_t v) {
+  uint64_t lo = r, step = 1;
+  while (lo < len && a[lo] <= v) {
+    const uint64_t hi = lo + step < len ? lo + step : len;
+    if (hi == len || a[hi] > v) {  // bound in (lo, hi]
+      uint64_t l = lo + 1, h = hi;
+      while (l < h) {
+        const uint64_t m = l + ((h - l) >> 1);
+        if (a[m] <= v) l = m + 1;
+        else h = m;
+      }
+      return l;
+    }
+    lo = hi;
+    step <<= 1;
+  }
+  return lo;
+}
+
+// coarse != nullptr: row (c - coarse_b0) of `coarse` holds the co-ranks of output position
+// min(c * coarse_step, total) (coarse_step a multiple of step); a fine boundary starts from the
+// windows between its two coarse neighbours: with v_lo = the key at the lower coarse position and
+// v_hi = the key just before the upper one, #(< v_lo) <= o_lo <= o < o_hi <= #(<= v_hi), so the
+// bisection starts at [v_lo, v_hi] with lo/hi found by galloping from the coarse co-ranks.
 template <int C>
 __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ keys,
                                                 const uint64_t* __restrict__ off, int k,
                                                 uint64_t total, uint64_t step, uint64_t b0,
-                                                uint64_t nb, uint64_t* __restrict__ ranks) {
+                                                uint64_t nb, uint64_t* __restrict__ ranks,
+                                                const uint64_t* __restrict__ coarse,
+                                                uint64_t coarse_step, uint64_t coarse_b0) {
   const uint64_t b = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (b >= nb) return;
@@ -90,11 +137,40 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
       if (c * 32 + lane < k) out[c * 32 + lane] = hi[c];
     return;
   }
+  uint64_t L0 = 0, H0 = ~0ull;
+  if (coarse) {
+    const uint64_t ci = o / coarse_step;
+    const uint64_t* r0 = coarse + (ci - coarse_b0) * (uint64_t)k;
+    if (o == ci * coarse_step) {  // a coarse boundary itself
+#pragma unroll
+      for (int c = 0; c < C; ++c)
+        if (c * 32 + lane < k) out[c * 32 + lane] = r0[c * 32 + lane];
+      return;
+    }
+    const uint64_t* r1 = r0 + k;
+    uint64_t rl[C], rh[C], mn = ~0ull, mx = 0;
+#pragma unroll
+    for (int c = 0; c < C; ++c) {
+      const int j = c * 32 + lane;
+      rl[c] = j < k ? r0[j] : 0;
+      rh[c] = j < k ? r1[j] : 0;
+      if (rl[c] < hi[c]) mn = K[base[c] + rl[c]] < mn ? K[base[c] + rl[c]] : mn;
+      if (rh[c] > 0) mx = K[base[c] + rh[c] - 1] > mx ? K[base[c] + rh[c] - 1] : mx;
+    }
+    L0 = warp_min(mn);  // key at merged position o_lo
+    H0 = warp_max(mx);  // key at merged position o_hi - 1
+#pragma unroll
+    for (int c = 0; c < C; ++c) {
+      const uint64_t len = hi[c];
+      lo[c] = lower_bound_back(K + base[c], rl[c], L0);
+      hi[c] = upper_bound_fwd(K + base[c], rh[c], len, H0);
+    }
+  }
   // Find v = the key at merged position o: smallest v with count(<= v) > o.
   // Invariant: lo[c] = #(< L) in run, hi[c] = #(<= H) in run, count(<= H) > o, count(< L) <= o.
   // (An interpolated two-pivot variant was measured: 1.9x slower at k = 12 -- the float64 key
   // space is not uniform across binades, so the interpolation misses -- and removed.)
-  uint64_t L = 0, H = ~0ull;
+  uint64_t L = L0, H = H0;
   while (true) {
     // tighten [L, H] to the keys still inside the windows
     uint64_t mn = ~0ull, mx = 0;
@@ -430,19 +506,51 @@ size_t merge_smem_bytes(int k) {
 
 }  // namespace
 
+namespace {
+cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
+                          uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
+                          const uint64_t* coarse, uint64_t cstep, uint64_t cb0, cudaStream_t st) {
+  const unsigned grid = (unsigned)((n_bounds * 32 + 127) / 128);
+  const int C = (k + 31) / 32;
+#define HS_CORANK(CC)                                                                              \
+  k_corank<CC><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks,    \
+                                     coarse, cstep, cb0)
+  if (C <= 1) HS_CORANK(1);
+  else if (C <= 2) HS_CORANK(2);
+  else if (C <= 4) HS_CORANK(4);
+  else if (C <= 8) HS_CORANK(8);
+  else HS_CORANK(kMaxC);
+#undef HS_CORANK
+  return cudaGetLastError();
+}
+}  // namespace
+
+// K4 in two levels: co-ranks every kCoarse fine steps first (full-range search), then every
+// fine boundary from the windows between its coarse neighbours (K4).
+constexpr uint64_t kCoarse = 16;
+
 cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
                          uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
                          cudaStream_t st) {
   if (k < 1 || k > kMaxMergeRuns) return cudaErrorInvalidValue;
   if (n_bounds == 0) return cudaSuccess;
-  const unsigned grid = (unsigned)((n_bounds * 32 + 127) / 128);
-  int C = (k + 31) / 32;
-  if (C <= 1) k_corank<1><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
-  else if (C <= 2) k_corank<2><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
-  else if (C <= 4) k_corank<4><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
-  else if (C <= 8) k_corank<8><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
-  else k_corank<kMaxC><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks);
-  return cudaGetLastError();
+  if (n_bounds < 4 * kCoarse || k == 1)
+    return corank_launch(keys, d_off, k, total, step, bound_begin, n_bounds, ranks, nullptr, 1, 0, st);
+  const uint64_t cstep = step * kCoarse;
+  const uint64_t o_first = bound_begin * step < total ? bound_begin * step : total;
+  const uint64_t o_last0 = (bound_begin + n_bounds - 1) * step;
+  const uint64_t o_last = o_last0 < total ? o_last0 : total;
+  const uint64_t c0 = o_first / cstep;
+  const uint64_t c1 = (o_last + cstep - 1) / cstep;  // coarse rows c0..c1 bracket every bound
+  const uint64_t nc = c1 - c0 + 1;
+  uint64_t* coarse = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&coarse, nc * (uint64_t)k * sizeof(uint64_t), st);
+  if (e != cudaSuccess) return e;
+  e = corank_launch(keys, d_off, k, total, cstep, c0, nc, coarse, nullptr, 1, 0, st);
+  if (e == cudaSuccess)
+    e = corank_launch(keys, d_off, k, total, step, bound_begin, n_bounds, ranks, coarse, cstep, c0, st);
+  cudaError_t e2 = cudaFreeAsync(coarse, st);
+  return e != cudaSuccess ? e : e2;
 }
 
 cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,

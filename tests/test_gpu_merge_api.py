@@ -38,6 +38,26 @@ def test_corank_matches_oracle(hs_gpu, oracle_mod, k, hi):
         assert np.array_equal(got[b], oracle_mod.corank(runs, o)), (b, o)
 
 
+@pytest.mark.parametrize("k", [2, 5, 33, 200])
+@pytest.mark.parametrize("hi", [2**64, 7, 3000])
+def test_corank_two_level_matches_oracle(hs_gpu, oracle_mod, k, hi):
+    """>= 64 bounds: coarse co-ranks every 16 steps, fine ones from the coarse windows (ties at
+    the coarse cuts with hi = 7 / 3000 exercise the galloping bounds)."""
+    import torch
+    rng = np.random.default_rng(k * 7 + hi % 991)
+    runs, keys, off = _runs(rng, k, 4000 if k < 50 else 300, hi)
+    total = int(off[-1])
+    step = 64
+    nb = total // step + 2
+    d_keys = torch.from_numpy(keys).cuda()
+    d_r = torch.zeros(nb * k, dtype=torch.uint64, device="cuda")
+    hs_gpu.hsort_device_corank(d_keys, off, step, nb, d_r)
+    got = d_r.cpu().numpy().reshape(nb, k)
+    for b in list(range(0, nb, 7)) + [nb - 2, nb - 1]:
+        o = min(b * step, total)
+        assert np.array_equal(got[b], oracle_mod.corank(runs, o)), (b, o)
+
+
 @pytest.mark.parametrize("k", [1, 2, 5, 16, 120, 1024])
 @pytest.mark.parametrize("hi", [2**64, 7])
 def test_device_merge_matches_oracle(hs_gpu, oracle_mod, k, hi):

@@ -1557,10 +1557,14 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       const uint32_t c = s_cnt[(jj & 1) * kRadix + kRadix - 1];
       tile_n = (int)((c >> 16) + (c & 0xFFFFu));
     }
-    auto wo_full = [&](auto inv_tag) {
+    // BOUNDED: the elision's tiles that lost outliers hold tile_n < TILE keys; the unrolled loop
+    // with a bound beats the strided loop used for the ragged last tile
+    auto wo_full = [&](auto inv_tag, auto bounded_tag) {
       constexpr bool INV = decltype(inv_tag)::value;
+      constexpr bool BOUNDED = decltype(bounded_tag)::value;
 #pragma unroll
       for (int q = 0; q < ITEMS; ++q) {
+        if (BOUNDED && tid + q * THREADS >= tile_n) break;
         const uint64_t v = sb[tid + q * THREADS];
         const int32_t g = gofs[(uint32_t)(v >> shift) & 255u];
         uint64_t* a = dst_t + g;
@@ -1572,8 +1576,11 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       }
     };
     if (tile_n == TILE) {  // (elision: tile_n is the count of keys left after the diversion)
-      if (inv) wo_full(std::true_type{});
-      else wo_full(std::false_type{});
+      if (inv) wo_full(std::true_type{}, std::false_type{});
+      else wo_full(std::false_type{}, std::false_type{});
+    } else if (DM == 2 && !KV && rem >= (uint64_t)TILE) {
+      if (inv) wo_full(std::true_type{}, std::true_type{});
+      else wo_full(std::false_type{}, std::true_type{});
     } else {
       for (int i = tid; i < tile_n; i += THREADS) {
         const uint64_t v = sb[i];
@@ -1700,7 +1707,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
-      rr[i] = (lane == leader && ((FULL && DM != 2) || dd[i] < kRadix))
+      rr[i] = (lane == leader && ((FULL && (DM != 2 || !w_out)) || dd[i] < kRadix))
                   ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i]))
                   : 0u;
     }
@@ -1708,7 +1715,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
       const uint32_t r = __shfl_sync(0xffffffffu, rr[i], leader) + __popc(peers[i] & lt);
-      if ((FULL && DM != 2) || dd[i] < kRadix) {
+      if ((FULL && (DM != 2 || !w_out)) || dd[i] < kRadix) {
         sb[r] = k[i];
         if (KV) vsb[r] = vv[i];
       }

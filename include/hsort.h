@@ -141,7 +141,8 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
  * sorted as bit patterns (NaN payloads and -0.0 preserved).  float64 ascending is hsort_sort
  * (every mode); every other combination runs on one GPU as one batch (BLINE): an encode pass to
  * 64-bit internal keys (float32 keys zero-extended, so the radix plan skips the 4 empty digits),
- * the GPUSort, a decode pass.  n must fit one GPU (16 B/key + the key array), else
+ * the GPUSort (out of place, so the dominant-digit elision applies), a decode pass.  n must fit one
+ * GPU (24 B/key + the key array), else
  * HSORT_ERR_INVALID.  A and B aligned to the key size; B == A allowed; partial overlap -> INVALID.
  * ------------------------------------------------------------------------------------------- */
 #define HSORT_KEY_F64 0
@@ -224,7 +225,7 @@ int hsort_sort_device_keys(const uint64_t* d_in, uint64_t* d_out, uint64_t n, in
 
 /* Typed GPUSort, device -> device (current device, stream-ordered): key_type / descending as for
  * hsort_sort_typed.  float64 ascending = hsort_sort_device; otherwise encode -> GPUSort -> decode
- * (16-byte aligned buffers; d_in == d_out allowed; library scratch 16 B/key). */
+ * (16-byte aligned buffers; d_in == d_out allowed; library scratch 24 B/key). */
 int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_type,
                             int descending, void* stream);
 

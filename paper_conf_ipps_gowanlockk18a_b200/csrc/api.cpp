@@ -128,6 +128,7 @@ struct GpuCtx {
   RadixScratch rs;
   DevBuf runs, alt, mout, min, ranks, off;
   DevBuf vruns, valt;  // key/value sorts: values and their ping-pong scratch
+  DevBuf tmp3;         // typed sorts: third key buffer, so the GPUSort runs out of place (elision)
   std::vector<char*> ring_in, ring_out;
   uint64_t ring_bytes = 0;
   std::vector<cudaEvent_t> ev_in, ev_out;
@@ -1001,6 +1002,7 @@ void ctx_destroy(GpuCtx& g) {
   for (auto e : g.ev_out) cudaEventDestroy(e);
   g.runs.release();
   g.alt.release();
+  g.tmp3.release();
   g.vruns.release();
   g.valt.release();
   g.mout.release();
@@ -1242,8 +1244,8 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     CK(cudaSetDevice(g.dev));
     size_t fr = 0, tot = 0;
     CK(cudaMemGetInfo(&fr, &tot));
-    const uint64_t held = g.runs.cap + g.alt.cap + g.mout.cap;
-    const uint64_t need = n * 8 * 2 + ((bytes + 15) & ~15ull) + n / 2 +
+    const uint64_t held = g.runs.cap + g.alt.cap + g.mout.cap + g.tmp3.cap;
+    const uint64_t need = n * 8 * 3 + ((bytes + 15) & ~15ull) + n / 2 +
                           (uint64_t)S().opt.get("device_reserve_mb") * (1ull << 20);
     if (need > fr + held)
       throw HsortError(HSORT_ERR_INVALID, "typed sort: n does not fit one GPU (BLINE only)");
@@ -1262,6 +1264,7 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     st.direct_out = dout;
     g.runs.reserve(n * 8);
     g.alt.reserve(n * 8);
+    g.tmp3.reserve(n * 8);
     g.mout.reserve((bytes + 15) & ~15ull);
     Acc acc;
     EvPair eh, es_, ed;
@@ -1274,8 +1277,8 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     CK(cudaStreamWaitEvent(g.s_comp, eh.b, 0));
     CK(cudaEventRecord(es_.a, g.s_comp));
     CK(key_encode(g.mout.p, g.runs.u64(), n, key_type, desc != 0, g.s_comp));
-    CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), n, false, false, g.s_comp));
-    CK(key_decode(g.runs.u64(), g.mout.p, n, key_type, desc != 0, g.s_comp));
+    CK(radix_sort(g.rs, g.runs.u64(), g.alt.u64(), g.tmp3.u64(), n, false, false, g.s_comp));
+    CK(key_decode(g.alt.u64(), g.mout.p, n, key_type, desc != 0, g.s_comp));
     CK(cudaEventRecord(es_.b, g.s_comp));
     CK(cudaStreamWaitEvent(g.s_d2h, es_.b, 0));
     CK(cudaEventRecord(ed.a, g.s_d2h));
@@ -1514,9 +1517,10 @@ int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_t
     cudaStream_t st = (cudaStream_t)stream;
     g.runs.reserve(n * 8);
     g.alt.reserve(n * 8);
+    g.tmp3.reserve(n * 8);
     CK(key_encode(d_in, g.runs.u64(), n, key_type, descending != 0, st));
-    CK(radix_sort(g.rs, g.runs.u64(), g.runs.u64(), g.alt.u64(), n, false, false, st));
-    CK(key_decode(g.runs.u64(), d_out, n, key_type, descending != 0, st));
+    CK(radix_sort(g.rs, g.runs.u64(), g.alt.u64(), g.tmp3.u64(), n, false, false, st));
+    CK(key_decode(g.alt.u64(), d_out, n, key_type, descending != 0, st));
     return HSORT_OK;
   });
 }

@@ -137,6 +137,38 @@ def cpu_baseline_oracle(n_sample: int):
     }
 
 
+PAR_SAMPLE = 1 << 27        # parallel-CPU baseline sample (~2-3 s on 16 cores)
+
+
+def cpu_parallel_baseline(n_sample: int):
+    """The paper's reference implementation: GNU parallel-mode sort (multiway
+    mergesort) under the same totalOrder, on all physical host cores, 3 trials."""
+    import hsort_inputs
+    import oracle
+    try:
+        import psutil
+        cores = psutil.cpu_count(logical=False) or os.cpu_count()
+    except Exception:
+        cores = os.cpu_count()
+    A = hsort_inputs.generate("uniform", n_sample, seed=SEED)
+    oracle.par_sort_f64(A[: 1 << 20], cores)  # warm (thread pool, library load)
+    ts = []
+    for _ in range(3):
+        t = time.perf_counter()
+        oracle.par_sort_f64(A, cores)
+        ts.append(time.perf_counter() - t)
+    dt = statistics.median(ts)
+    return {
+        "value": n_sample / dt, "unit": "keys/s", "cores": cores, "kind": "gnu_parallel_sort",
+        "sample": f"first {n_sample} keys of the C2 workload (uniform seed {SEED}), "
+                  f"__gnu_parallel::sort (multiway mergesort, exact splitting) under IEEE totalOrder, "
+                  f"{cores} OpenMP threads, median of 3: {dt:.2f} s",
+        "paper_context": "paper: up to 3.47x end-to-end over a 16-thread GNU parallel sort on "
+                         "2x8-core Xeon E5-2620 v4 + 1x Quadro GP100, PCIe 3, n = 1e9 float64 "
+                         "(P:907-910, P:499-504); context only",
+    }
+
+
 MERGE_K = 12  # runs of the RESIDENT auto plan at n = 2^30 (2^27-key batches + halving tail)
 
 
@@ -461,6 +493,9 @@ def main():
     }
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline_oracle(ORACLE_SAMPLE)
+        par = cpu_parallel_baseline(PAR_SAMPLE)
+        par["e2e_speedup"] = e2e_value / par["value"]  # our host->host rate / parallel CPU rate
+        line["cpu_parallel_baseline"] = par
     if rank == 0:
         print(json.dumps(line), flush=True)
     hs.hsort_finalize()

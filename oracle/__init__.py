@@ -25,6 +25,38 @@ _U64 = ctypes.c_uint64
 _P = ctypes.c_void_p
 
 
+_PAR_SRC = os.path.join(_HERE, "par_baseline.cpp")
+_PAR_SO = os.path.join(_HERE, "libparbaseline.so")
+_par = None
+
+
+def build_par(force: bool = False) -> str:
+    """Compile the parallel-CPU baseline (GNU parallel-mode sort, -fopenmp) into its own library."""
+    if force or not os.path.exists(_PAR_SO) or os.path.getmtime(_PAR_SO) < os.path.getmtime(_PAR_SRC):
+        subprocess.check_call(["g++", "-O2", "-std=c++20", "-fopenmp", "-shared", "-fPIC", _PAR_SRC,
+                               "-o", _PAR_SO + ".tmp"])
+        os.replace(_PAR_SO + ".tmp", _PAR_SO)
+    return _PAR_SO
+
+
+def par_sort_f64(A, threads: int = 0) -> np.ndarray:
+    """The parallel-CPU baseline: __gnu_parallel::sort under totalOrder on `threads` cores."""
+    global _par
+    with _lock:
+        if _par is None:
+            build_par()
+            lib = ctypes.CDLL(_PAR_SO)
+            lib.par_sort_f64.argtypes = [_P, _P, _U64, ctypes.c_int]
+            lib.par_sort_f64.restype = None
+            lib.par_max_threads.argtypes = []
+            lib.par_max_threads.restype = ctypes.c_int
+            _par = lib
+    A = np.ascontiguousarray(A, dtype=np.float64)
+    B = np.empty_like(A)
+    _par.par_sort_f64(A.ctypes.data, B.ctypes.data, A.size, int(threads))
+    return B
+
+
 def build(force: bool = False) -> str:
     """Compile oracle.cpp into liboracle.so (serial, -O2, C++20)."""
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):

@@ -98,3 +98,13 @@ def test_empty_and_single(oracle_mod):
     assert oracle_mod.sort_f64(np.zeros(0)).size == 0
     x = np.array([np.nan])
     assert _bits(oracle_mod.sort_f64(x))[0] == _bits(x)[0]
+
+
+def test_parallel_cpu_baseline_equals_oracle(oracle_mod, inputs_mod):
+    """The parallel-CPU baseline (GNU parallel sort, the paper's reference) is bit-identical to the
+    oracle under totalOrder (the result is unique), incl. ±0 and NaN payloads."""
+    for dist, n in (("special", 100_000), ("salted", 1_000_003), ("uniform", 777)):
+        A = inputs_mod.generate(dist, n, seed=n)
+        want = oracle_mod.sort_f64(A).view(np.uint64)
+        for threads in (1, 4):
+            assert np.array_equal(oracle_mod.par_sort_f64(A, threads).view(np.uint64), want)

@@ -483,6 +483,7 @@ def main():
             "link_gbs": {"h2d": bw["h2d"] / 1e9, "d2h": bw["d2h"] / 1e9},
             "link_floor_ms": 1e3 * link_floor_s,
             "link_frac": link_floor_s / (e2e_total / e2e_steps),
+            "step_ms": [round(1e3 * t, 2) for t in e2e_t],  # this rank's steps (value uses the sum)
         },
         "stages": stages,
         # per step: K1, K2, 8 pass launches (inactive ones return at once), final copy; with the

@@ -974,6 +974,15 @@ void ctx_create(GpuCtx& g, int dev, const Options& opt) {
   CK(cudaStreamCreateWithFlags(&g.s_h2d, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g.s_comp, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g.s_d2h, cudaStreamNonBlocking));
+  {  // K4's coarse co-rank tables come from cudaMallocAsync: keep freed blocks in the device's
+     // default pool instead of trimming it at every synchronisation
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t keep = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+    cudaGetLastError();
+  }
   int R = (int)std::max<int64_t>(2, opt.get("n_ring"));
   g.ring_bytes = (uint64_t)std::max<int64_t>(1 << 20, opt.get("p_s"));
   g.ring_bytes = (g.ring_bytes + 4095) & ~4095ull;

@@ -50,11 +50,24 @@ def par_sort_f64(A, threads: int = 0) -> np.ndarray:
             lib.par_sort_f64.restype = None
             lib.par_max_threads.argtypes = []
             lib.par_max_threads.restype = ctypes.c_int
+            lib.par_multiway_merge_u64.argtypes = [_P, _P, ctypes.c_int, _P, ctypes.c_int]
+            lib.par_multiway_merge_u64.restype = None
             _par = lib
     A = np.ascontiguousarray(A, dtype=np.float64)
     B = np.empty_like(A)
     _par.par_sort_f64(A.ctypes.data, B.ctypes.data, A.size, int(threads))
     return B
+
+
+def par_multiway_merge_u64(keys, off, threads: int = 0) -> np.ndarray:
+    """CPU-merge reference: __gnu_parallel::multiway_merge of the sorted runs keys[off[j]:off[j+1]]."""
+    par_sort_f64(np.zeros(0))  # loads the library
+    keys = np.ascontiguousarray(keys, dtype=np.uint64)
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    out = np.empty(int(off[-1] - off[0]), dtype=np.uint64)
+    _par.par_multiway_merge_u64(keys.ctypes.data, off.ctypes.data, off.size - 1, out.ctypes.data,
+                                int(threads))
+    return out
 
 
 def build(force: bool = False) -> str:

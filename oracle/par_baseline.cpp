@@ -24,3 +24,26 @@ void par_sort_f64(const double* A, double* B, uint64_t n, int threads) {
 int par_max_threads(void) { return omp_get_max_threads(); }
 
 }  // extern "C"
+
+#include <parallel/multiway_merge.h>
+
+#include <utility>
+#include <vector>
+
+extern "C" {
+
+// CPU-merge reference (BASELINE.md plan item 3; the paper's own merge): GNU parallel
+// multiway_merge of k sorted uint64 runs keys[off[j], off[j+1]) into out, `threads` OpenMP threads.
+void par_multiway_merge_u64(const uint64_t* keys, const uint64_t* off, int k, uint64_t* out,
+                            int threads) {
+  if (threads > 0) omp_set_num_threads(threads);
+  // (libstdc++'s multiway_merge needs mutable iterators; the runs are only read)
+  uint64_t* base = const_cast<uint64_t*>(keys);
+  std::vector<std::pair<uint64_t*, uint64_t*>> seqs(k);
+  for (int j = 0; j < k; ++j) seqs[j] = {base + off[j], base + off[j + 1]};
+  const uint64_t total = off[k] - off[0];
+  __gnu_parallel::multiway_merge(seqs.begin(), seqs.end(), out, total, std::less<uint64_t>(),
+                                 __gnu_parallel::parallel_tag());
+}
+
+}  // extern "C"

@@ -129,3 +129,13 @@ def test_pipemerge_parity_rule(oracle_mod):
     # with 2+ GPUs fewer pair-wise merges happen than with one.
     for n_b in range(2, 40):
         assert oracle_mod.pipemerge_count(n_b, 2) <= oracle_mod.pipemerge_count(n_b, 1)
+
+
+def test_gnu_multiway_merge_reference_equals_oracle(oracle_mod):
+    """The CPU-merge reference (GNU parallel multiway_merge, the paper's merge) = oracle merge."""
+    rng = np.random.default_rng(4)
+    runs = [np.sort(rng.integers(0, 1000, size=int(rng.integers(0, 5000)), dtype=np.uint64))
+            for _ in range(9)]
+    off = np.cumsum([0] + [r.size for r in runs]).astype(np.uint64)
+    keys = np.concatenate(runs)
+    assert np.array_equal(oracle_mod.par_multiway_merge_u64(keys, off, 4), oracle_mod.merge_runs(runs))

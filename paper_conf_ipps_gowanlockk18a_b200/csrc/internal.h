@@ -79,6 +79,7 @@ constexpr int kKvTile = 4032;     // pairs per key/value onesweep tile (576 x 7)
 
 // dominant-digit elision on/off (option "dde", default on)
 extern bool g_dde_enabled;
+extern uint64_t g_dde_min_n;
 cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n);
 cudaError_t radix_set_timing(RadixScratch& s, bool on);
 // durations (ms) of [K1, K2, pass0..pass7, final copy] of the last timed sort; returns count

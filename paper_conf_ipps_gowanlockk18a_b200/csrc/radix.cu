@@ -1981,10 +1981,10 @@ void radix_scratch_release(RadixScratch& s) {
   s = RadixScratch();
 }
 
-#ifndef HSORT_DDE_MIN_N
-#define HSORT_DDE_MIN_N (1ull << 22)  // below this the outlier sort's fixed cost outweighs a pass
-#endif
 bool g_dde_enabled = true;  // hsort_set_option("dde", 0) turns the elision off (A/B, tests)
+// below this n the outlier sort's fixed cost outweighs a pass (option "dde_min_n"; lowered only
+// by the sanitizer runs, tools/sanitize_run.py)
+uint64_t g_dde_min_n = 1ull << 22;
 
 // Side buffer capacity for n keys: the outliers a plan may divert (K2 checks n_out <= cap).
 uint64_t dde_cap(uint64_t n) {
@@ -2007,7 +2007,7 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
   // the elision lives in the warp-specialised pass (32-bit look-back words, n <= 2^30); out of
   // place only (in place, 7 of 8 passes would end in the scratch buffer and need a copy)
   const bool dde = allow_dde && g_dde_enabled && kernel == 2 && in != out &&
-                   n >= HSORT_DDE_MIN_N && n <= (1ull << 30);
+                   n >= g_dde_min_n && n <= (1ull << 30);
   uint64_t cap = 0;
   if (dde) {
     cap = dde_cap(n);

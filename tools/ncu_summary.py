@@ -71,6 +71,11 @@ if a.steps:
                 break
         keep.append(r)
     rows = keep
+# the library's own kernels (k_*); torch kernels (bench input copies, the output guard outside
+# the timed steps) are listed separately and excluded from the shares
+ours = [r for r in rows if r[0].startswith("k_")]
+other = [r for r in rows if not r[0].startswith("k_")]
+rows = ours
 agg = OrderedDict()
 for k, ns, g, b in rows:
     e = agg.setdefault((k, g), [0, 0.0, g, b])
@@ -83,6 +88,9 @@ md = ["# ncu launch list summary", "", f"source: `{a.csv}` (gpu__time_duration.s
       "| kernel | launches | total ms | mean ms | share | grid | block |", "|---|---|---|---|---|---|---|"]
 for (k, _), (c, ns, g, b) in sorted(agg.items(), key=lambda x: -x[1][1]):
     md.append(f"| `{k}` | {c} | {ns/1e6:.3f} | {ns/1e6/c:.3f} | {ns/tot:.1%} | {g} | {b} |")
+if other:
+    md += ["", f"Not ours (torch; excluded from the shares): {len(other)} launches, "
+           f"{sum(r[1] for r in other)/1e6:.3f} ms (bench input copies and the output guard)."]
 js = {"n": a.n}
 for rep in a.reports:
     m = full_metrics(rep)

@@ -116,6 +116,7 @@ struct Options {
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
       {"dde", 1},                    // 1: dominant-digit elision in the GPUSort
       {"dde_min_n", 1ll << 22},      // smallest n the elision is tried at
+      {"memcpy_nt", 1},              // PARMEMCPY staging copies with non-temporal stores
       {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
       {"pin_w", -1},                 // STREAM W: 1 cached pinned, 0 pageable, -1 pinned if <= pin_w_max_mb
       {"pin_w_max_mb", 16384},       // auto pinning limit: pinning runs at ~2.5 GB/s
@@ -1419,6 +1420,7 @@ int hsort_set_option(const char* key, int64_t value) {
   S().opt.v[k] = value;
   if (k == "dde") g_dde_enabled = value != 0;
   if (k == "dde_min_n") g_dde_min_n = (uint64_t)(value < 1 ? 1 : value);
+  if (k == "memcpy_nt") g_memcpy_nt = value != 0;
   if (k == "kernel_timing") {
     return guarded([&]() -> int {
       for (auto& g : S().gpus) {

@@ -1,6 +1,7 @@
 // pool.cpp — host worker pool and PARMEMCPY (§III-D2: "if host-to-host MCpy
 // to/from pinned memory in Stage is a bottleneck when using std::memcpy, we can parallelize this
 // step on the host").
+#include <emmintrin.h>
 #include "pool.h"
 
 #include <algorithm>
@@ -84,11 +85,43 @@ ThreadPool& pipe_pool() {
   return pool;
 }
 
+bool g_memcpy_nt = true;  // option "memcpy_nt": streaming stores in PARMEMCPY
+
+// memcpy with non-temporal 16-byte stores (SSE2): the destination is not read for ownership and
+// does not displace the cache -- staging copies are write-once, read by DMA or by the caller later
+static void memcpy_nt(void* dst, const void* src, uint64_t bytes) {
+  char* d = (char*)dst;
+  const char* s = (const char*)src;
+  const uint64_t head = (16 - ((uintptr_t)d & 15)) & 15;
+  if (bytes < head + 64) {
+    std::memcpy(d, s, bytes);
+    return;
+  }
+  std::memcpy(d, s, head);
+  d += head;
+  s += head;
+  bytes -= head;
+  const uint64_t body = bytes & ~63ull;
+  for (uint64_t i = 0; i < body; i += 64) {
+    const __m128i a = _mm_loadu_si128((const __m128i*)(s + i));
+    const __m128i b = _mm_loadu_si128((const __m128i*)(s + i + 16));
+    const __m128i c = _mm_loadu_si128((const __m128i*)(s + i + 32));
+    const __m128i e = _mm_loadu_si128((const __m128i*)(s + i + 48));
+    _mm_stream_si128((__m128i*)(d + i), a);
+    _mm_stream_si128((__m128i*)(d + i + 16), b);
+    _mm_stream_si128((__m128i*)(d + i + 32), c);
+    _mm_stream_si128((__m128i*)(d + i + 48), e);
+  }
+  std::memcpy(d + body, s + body, bytes - body);
+  _mm_sfence();
+}
+
 void par_memcpy(void* dst, const void* src, uint64_t bytes, int threads) {
   if (threads <= 0) threads = host_threads();
   constexpr uint64_t kMinChunk = 2ull << 20;
   if (threads == 1 || bytes < 2 * kMinChunk) {
-    std::memcpy(dst, src, bytes);
+    if (g_memcpy_nt && bytes >= kMinChunk) memcpy_nt(dst, src, bytes);
+    else std::memcpy(dst, src, bytes);
     return;
   }
   int64_t tasks = (int64_t)std::min<uint64_t>((uint64_t)threads * 2, bytes / kMinChunk);
@@ -97,7 +130,8 @@ void par_memcpy(void* dst, const void* src, uint64_t bytes, int threads) {
     uint64_t lo = (uint64_t)t * chunk;
     if (lo >= bytes) return;
     uint64_t len = std::min<uint64_t>(chunk, bytes - lo);
-    std::memcpy((char*)dst + lo, (const char*)src + lo, len);
+    if (g_memcpy_nt) memcpy_nt((char*)dst + lo, (const char*)src + lo, len);
+    else std::memcpy((char*)dst + lo, (const char*)src + lo, len);
   });
 }
 

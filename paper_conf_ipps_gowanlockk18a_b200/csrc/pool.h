@@ -51,6 +51,7 @@ ThreadPool& pipe_pool();
 int host_threads();
 
 // PARMEMCPY: dst <- src (bytes) split over `threads` workers (0 = all host threads).
+extern bool g_memcpy_nt;  // PARMEMCPY streaming stores (option "memcpy_nt", default on)
 void par_memcpy(void* dst, const void* src, uint64_t bytes, int threads);
 
 }  // namespace hsort

@@ -155,3 +155,17 @@ def test_sort_without_init_fails_cleanly(hs):
     with pytest.raises(hs.HsortError) as e:
         hs.hsort_sort(A)
     assert e.value.code == -2
+
+
+def test_par_memcpy_streaming_stores(hs):
+    """PARMEMCPY with non-temporal stores (option memcpy_nt): unaligned heads/tails, all sizes."""
+    rng = np.random.default_rng(0)
+    src = rng.integers(0, 256, size=(9 << 20) + 100, dtype=np.uint8)
+    for nt in (1, 0):
+        hs.hsort_set_option("memcpy_nt", nt)
+        for size, so, do in ((0, 0, 0), (5, 1, 3), ((2 << 20) + 3, 7, 1), ((8 << 20) + 17, 3, 9)):
+            dst = np.zeros(size + 16, dtype=np.uint8)
+            hs.hsort_par_memcpy(dst[do:do + size], src[so:so + size], 4)
+            assert np.array_equal(dst[do:do + size], src[so:so + size]), (nt, size, so, do)
+            assert not dst[:do].any() and not dst[do + size:].any()
+    hs.hsort_set_option("memcpy_nt", 1)

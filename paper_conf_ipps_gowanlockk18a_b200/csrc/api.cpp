@@ -1287,13 +1287,24 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     CK(cudaEventRecord(eh.b, g.s_h2d));
     CK(cudaStreamWaitEvent(g.s_comp, eh.b, 0));
     CK(cudaEventRecord(es_.a, g.s_comp));
-    CK(key_encode(g.mout.p, g.runs.u64(), n, key_type, desc != 0, g.s_comp));
-    CK(radix_sort(g.rs, g.runs.u64(), g.alt.u64(), g.tmp3.u64(), n, false, false, g.s_comp));
-    CK(key_decode(g.alt.u64(), g.mout.p, n, key_type, desc != 0, g.s_comp));
+    // float64 descending: the reverse transform fused into the GPUSort (mout -> runs); else the
+    // codec passes around the ascending GPUSort of internal keys
+    const cudaError_t fe = key_type == HSORT_KEY_F64 && desc
+                               ? radix_sort_desc_f64(g.rs, g.mout.u64(), g.runs.u64(), g.alt.u64(), n, g.s_comp)
+                               : cudaErrorNotSupported;
+    if (fe == cudaErrorNotSupported) {
+      cudaGetLastError();
+      CK(key_encode(g.mout.p, g.runs.u64(), n, key_type, desc != 0, g.s_comp));
+      CK(radix_sort(g.rs, g.runs.u64(), g.alt.u64(), g.tmp3.u64(), n, false, false, g.s_comp));
+      CK(key_decode(g.alt.u64(), g.mout.p, n, key_type, desc != 0, g.s_comp));
+    } else {
+      CK(fe);
+    }
+    const void* result = fe == cudaErrorNotSupported ? g.mout.p : g.runs.p;
     CK(cudaEventRecord(es_.b, g.s_comp));
     CK(cudaStreamWaitEvent(g.s_d2h, es_.b, 0));
     CK(cudaEventRecord(ed.a, g.s_d2h));
-    download(g, B, g.mout.p, bytes, g.s_d2h, dout, mc, acc);
+    download(g, B, result, bytes, g.s_d2h, dout, mc, acc);
     CK(cudaEventRecord(ed.b, g.s_d2h));
     CK(cudaStreamSynchronize(g.s_d2h));
     st.t_sort_phase = secs_since(t0);
@@ -1530,6 +1541,16 @@ int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_t
     cudaStream_t st = (cudaStream_t)stream;
     g.runs.reserve(n * 8);
     g.alt.reserve(n * 8);
+    if (key_type == HSORT_KEY_F64 && descending && d_in != d_out) {
+      // reverse transform fused into the GPUSort's first and last pass
+      const cudaError_t fe = radix_sort_desc_f64(g.rs, (const uint64_t*)d_in, (uint64_t*)d_out,
+                                                 g.alt.u64(), n, st);
+      if (fe != cudaErrorNotSupported) {
+        CK(fe);
+        return HSORT_OK;
+      }
+      cudaGetLastError();
+    }
     g.tmp3.reserve(n * 8);
     CK(key_encode(d_in, g.runs.u64(), n, key_type, descending != 0, st));
     CK(radix_sort(g.rs, g.runs.u64(), g.alt.u64(), g.tmp3.u64(), n, false, false, st));

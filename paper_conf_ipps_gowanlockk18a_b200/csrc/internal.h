@@ -32,6 +32,10 @@ struct RadixPlan {
   uint64_t dde_n_out;   // outliers (n - count of v)
   uint64_t dde_n_less;  // outliers whose digit L is below v
   int32_t dde_k1;       // 1: K1 already counted the outliers' digit-P histogram (L = 7, P = 6)
+  // Descending float64 (S§8(f) #4), fused: the passes sort key(u) ^ key_xor (~0 descending, 0
+  // ascending); the first pass applies it on load, the last pass removes it on the inverse store.
+  // K1 counts ascending digits; K2 reads digit value v at 255 - v when descending.
+  uint64_t key_xor;
 };
 
 // Device state of the dominant-digit elision, zeroed per sort.
@@ -91,6 +95,11 @@ void radix_scratch_release(RadixScratch& s);
 // pass).  out_f64: store float64 bits (inverse transform fused into the last pass).
 cudaError_t radix_sort(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,
                        uint64_t n, bool in_f64, bool out_f64, cudaStream_t st);
+// Descending float64 GPUSort with the reverse transform fused into the first and last pass
+// (warp-specialised pass only: 16-byte aligned buffers, 2^20 <= n <= 2^30; returns
+// cudaErrorNotSupported otherwise, and the caller takes the codec path).
+cudaError_t radix_sort_desc_f64(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,
+                                uint64_t n, cudaStream_t st);
 // Key/value GPUSort (S§8(f) #3): (out, vout) = (in, vin) stably sorted by key; n <= 2^30, every
 // buffer 16-byte aligned, tmp/vtmp n-element scratch; in == out iff vin == vout.  The values are
 // opaque 64-bit payloads (e.g. indices: argsort).

@@ -180,13 +180,16 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
                                                    int in_eq_out, int in_f64, int out_f64,
                                                    uint32_t* __restrict__ lb_state,
                                                    uint64_t dde_cap = 0,
-                                                   const DdeState* __restrict__ dde = nullptr) {
+                                                   const DdeState* __restrict__ dde = nullptr,
+                                                   int desc = 0) {
   __shared__ uint64_t s_warp[8];
   __shared__ int s_nz[kDigits];
   __shared__ float s_dist[kDigits][8];
   const int t = threadIdx.x;
+  // descending: the passes sort complemented keys, whose digit value t is digit 255 - t of K1
+  const int tq = desc ? kRadix - 1 - t : t;
   for (int p = 0; p < kDigits; ++p) {
-    uint64_t v = hist[p * kRadix + t];
+    uint64_t v = hist[p * kRadix + tq];
     uint64_t e = scan256_excl(v, s_warp, nullptr);
     bin_base[p * kRadix + t] = e;
     int nz = __syncthreads_count(v != 0);
@@ -214,6 +217,7 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
     P.dde_n_out = 0;
     P.dde_n_less = 0;
     P.dde_k1 = 0;
+    P.key_xor = desc ? ~0ull : 0ull;
     if (dde_cap && na >= 3) {
       // top active digit L: dominant value v; elide its pass if the outliers fit the side buffer
       // and the remaining na - 1 passes still end in out without a final copy
@@ -221,7 +225,7 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
       uint64_t best = 0, below = 0, below_best = 0;
       uint32_t v = 0;
       for (int b = 0; b < kRadix; ++b) {
-        const uint64_t c = hist[L * kRadix + b];
+        const uint64_t c = hist[L * kRadix + (desc ? kRadix - 1 - b : b)];
         if (c > best) {
           best = c;
           v = (uint32_t)b;
@@ -240,7 +244,7 @@ __global__ void __launch_bounds__(256) k_scan_plan(const uint64_t* __restrict__ 
         P.dde_n_out = n_out;
         P.dde_n_less = below_best;
         // K1 counted the outliers' digit-6 histogram if the guess (key 0's top digit) was right
-        P.dde_k1 = (dde && L == 7 && P.digit[na - 1] == 6 && v == dde->guess) ? 1 : 0;
+        P.dde_k1 = (dde && !desc && L == 7 && P.digit[na - 1] == 6 && v == dde->guess) ? 1 : 0;
       }
     }
     P.num_active = na;
@@ -306,6 +310,7 @@ __global__ void k_force_plan(RadixPlan* plan, int digit, uint32_t* lb_state) {
   P.dde_pass = -1;
   P.dde_n_out = P.dde_n_less = 0;
   P.dde_k1 = 0;
+  P.key_xor = 0;
   *plan = P;
 }
 
@@ -1050,11 +1055,11 @@ __global__ void k_final_copy(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_
 // Dominant-digit elision, last step: the sorted outliers (side[0, n_out), internal keys) go to
 // out[0, n_less) (digit L below the dominant value) and out[n - (n_out - n_less), n) (above).
 __global__ void k_dde_place(const uint64_t* __restrict__ side, uint64_t n_out, uint64_t n_less,
-                            uint64_t* __restrict__ out, uint64_t n, int out_f64) {
+                            uint64_t* __restrict__ out, uint64_t n, int out_f64, uint64_t kx) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_out;
        i += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t v = side[i];
-    out[i < n_less ? i : n - n_out + i] = out_f64 ? from_key(v) : v;
+    out[i < n_less ? i : n - n_out + i] = out_f64 ? from_key(v ^ kx) : v;
   }
 }
 
@@ -1355,7 +1360,8 @@ __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64
 // DM (dominant-digit elision): 0 none; 1 pass 0 of an elided sort (counts the
 // outliers' digit-P histogram); 2 the elided sort's last pass (diverts the outliers).  The host
 // picks DM per launch after reading K2's plan, so the DM = 0 kernel carries no elision code.
-template <int CT, int ITEMS, bool IN_F64, bool KV = false, int DM = 0>
+// DESC: a descending float64 sort (compile-time, so ascending kernels carry no extra work).
+template <int CT, int ITEMS, bool IN_F64, bool KV = false, int DM = 0, bool DESC = false>
 __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in, uint64_t* out, uint64_t* tmp,
                                                        uint64_t* vin, uint64_t* vout, uint64_t* vtmp,
                                                        uint64_t n, const RadixPlan* __restrict__ plan,
@@ -1398,6 +1404,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   // dominant-digit elision: pass 0 counts the outliers' digit-P histogram; the last pass diverts
   // the outliers (digit L != v) to the side buffer and ranks the rest by digit P
   static_assert(DM == 0 || !KV, "the elision is keys-only");
+  const uint64_t kx = DESC ? plan->key_xor : 0ull;  // descending: complement on the first load
+  const uint64_t kx_in = p == 0 ? kx : 0ull;        // ... and before the last inverse store
   constexpr bool dde_here = DM == 2;
   const int sh_l = DM ? 8 * plan->dde_digit : 0;
   const uint32_t v_l = DM ? plan->dde_value : 0u;
@@ -1450,7 +1458,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
         const uint32_t* ho = plan->dde_k1 ? dde->hist_k1 : dde->hist_out;
-        c[q] = hist[digit * kRadix + lane * 8 + q] - ho[lane * 8 + q];
+        const int dq = kx ? kRadix - 1 - (lane * 8 + q) : lane * 8 + q;  // K1 counts ascending digits
+        c[q] = hist[digit * kRadix + dq] - ho[lane * 8 + q];
         tot += c[q];
       }
       uint64_t incl = tot;
@@ -1571,7 +1580,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #if HSORT_FAKE == 3
         if (v == 0x123456789ull)
 #endif
-        st_global_u64((uint64_t)(a + q * THREADS), INV ? from_key(v) : v);
+        st_global_u64((uint64_t)(a + q * THREADS), INV ? from_key(v ^ kx) : v);
         if (KV) st_global_u64((uint64_t)(vdst + tid + g + q * THREADS), vsb[tid + q * THREADS]);
       }
     };
@@ -1585,7 +1594,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       for (int i = tid; i < tile_n; i += THREADS) {
         const uint64_t v = sb[i];
         const int32_t g = gofs[(uint32_t)(v >> shift) & 255u];
-        st_global_u64((uint64_t)(dst + g + i), inv ? from_key(v) : v);
+        st_global_u64((uint64_t)(dst + g + i), inv ? from_key(v ^ kx) : v);
         if (KV) st_global_u64((uint64_t)(vdst + g + i), vsb[i]);
       }
     }
@@ -1616,7 +1625,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
         if (FULL) vv[i] = vsb[jj];
         else vv[i] = jj < bulk_n ? vsb[jj] : (jj < tile_n ? vsrc[tbase + jj] : 0);
       }
-      k[i] = IN_F64 ? to_key(v) : v;
+      k[i] = (IN_F64 ? to_key(v) : v) ^ kx_in;
       const bool valid = FULL || jj < tile_n;
       dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
       if (DM != 0) omask |= (uint32_t)(valid && ((uint32_t)(k[i] >> sh_l) & 255u) != v_l) << i;
@@ -1786,7 +1795,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       lb32_next[rr * kRadix + tid] = 0;
 }
 
-template <int CT, int ITEMS, bool KV = false, int DM = 0>
+template <int CT, int ITEMS, bool KV = false, int DM = 0, bool DESC = false>
 cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t* vin, uint64_t* vout,
                            uint64_t* vtmp, uint64_t n, RadixScratch& s, int p, bool first_in_f64,
                            bool out_f64, cudaStream_t st) {
@@ -1795,8 +1804,8 @@ cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t*
   int dev = 0;
   cudaGetDevice(&dev);
   constexpr bool dde = DM != 0;
-  auto kt = k_onesweep_ws<CT, ITEMS, true, KV, DM>;
-  auto kf = k_onesweep_ws<CT, ITEMS, false, KV, DM>;
+  auto kt = k_onesweep_ws<CT, ITEMS, true, KV, DM, DESC>;
+  auto kf = k_onesweep_ws<CT, ITEMS, false, KV, DM, DESC>;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   if (!blocks_per_sm[dev]) {
     cudaError_t e;
@@ -1854,12 +1863,24 @@ cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t
 }
 
 cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t n,
-                        int p, bool first_in_f64, bool out_f64, cudaStream_t st, int dm = 0) {
+                        int p, bool first_in_f64, bool out_f64, cudaStream_t st, int dm = 0,
+                        bool desc = false) {
   uint32_t ep = 0;
   cudaError_t e = next_epoch(s, st, &ep);
   if (e != cudaSuccess) return e;
   // TMA bulk copies need 16-byte aligned tile sources: every buffer the plan may read
   const int v = pass_kernel(in, out, tmp);
+  if (v == 2 && s.lb_mode == 2 && desc) {
+    constexpr int CT = HSORT_WS_CT, IT = HSORT_WS_ITEMS;
+    if (dm == 1)
+      return launch_ws_pass<CT, IT, false, 1, true>(in, out, tmp, nullptr, nullptr, nullptr, n, s, p,
+                                                    first_in_f64, out_f64, st);
+    if (dm == 2)
+      return launch_ws_pass<CT, IT, false, 2, true>(in, out, tmp, nullptr, nullptr, nullptr, n, s, p,
+                                                    first_in_f64, out_f64, st);
+    return launch_ws_pass<CT, IT, false, 0, true>(in, out, tmp, nullptr, nullptr, nullptr, n, s, p,
+                                                  first_in_f64, out_f64, st);
+  }
   if (v == 2 && s.lb_mode == 2) {
     if (dm == 1)
       return launch_ws_pass<HSORT_WS_CT, HSORT_WS_ITEMS, false, 1>(in, out, tmp, nullptr, nullptr, nullptr,
@@ -1995,7 +2016,8 @@ uint64_t dde_cap(uint64_t n) {
 }
 
 cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
-                            uint64_t n, bool in_f64, bool out_f64, cudaStream_t st, bool allow_dde) {
+                            uint64_t n, bool in_f64, bool out_f64, cudaStream_t st, bool allow_dde,
+                            bool desc = false) {
   if (n == 0) return cudaSuccess;
   cudaError_t e = radix_scratch_reserve(s, n);
   if (e != cudaSuccess) return e;
@@ -2004,6 +2026,7 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
     return s.timing ? cudaEventRecord(s.ev[i], st) : cudaSuccess;
   };
   const int kernel = pass_kernel(in, out, tmp);
+  if (desc && (kernel != 2 || n > (1ull << 30) || !in_f64 || !out_f64)) return cudaErrorNotSupported;
   // the elision lives in the warp-specialised pass (32-bit look-back words, n <= 2^30); out of
   // place only (in place, 7 of 8 passes would end in the scratch buffer and need a copy)
   const bool dde = allow_dde && g_dde_enabled && kernel == 2 && in != out &&
@@ -2028,7 +2051,8 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
   if ((e = mark(1)) != cudaSuccess) return e;
   if ((e = select_lb_mode(s, kernel, n, st)) != cudaSuccess) return e;
   k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
-                                 out_f64 ? 1 : 0, s.lb_state, cap, dde ? s.dde : nullptr);
+                                 out_f64 ? 1 : 0, s.lb_state, cap, dde ? s.dde : nullptr,
+                                 desc ? 1 : 0);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   if ((e = mark(2)) != cudaSuccess) return e;
   int dev = 0;
@@ -2043,7 +2067,8 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
       for (int p = 0; p < kDigits; ++p) {
         if (p < P.num_active) {
           const int dm = p == P.dde_pass ? 2 : (p == 0 && !P.dde_k1 ? 1 : 0);
-          if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st, dm)) != cudaSuccess)
+          if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st, dm, desc)) !=
+              cudaSuccess)
             return e;
         }
         if ((e = mark(3 + p)) != cudaSuccess) return e;
@@ -2056,14 +2081,15 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
           cudaSuccess)
         return e;
       if (n_out) {
-        k_dde_place<<<num_sms(dev), 256, 0, st>>>(s.side, n_out, P.dde_n_less, out, n, out_f64 ? 1 : 0);
+        k_dde_place<<<num_sms(dev), 256, 0, st>>>(s.side, n_out, P.dde_n_less, out, n, out_f64 ? 1 : 0,
+                                                  P.key_xor);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
       }
       return mark(11);
     }
   }
   for (int p = 0; p < kDigits; ++p) {
-    if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st)) != cudaSuccess)
+    if ((e = launch_pass(s, in, out, tmp, n, p, p == 0 && in_f64, out_f64, st, 0, desc)) != cudaSuccess)
       return e;
     if ((e = mark(3 + p)) != cudaSuccess) return e;
   }
@@ -2076,6 +2102,12 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
 cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
                        uint64_t n, bool in_f64, bool out_f64, cudaStream_t st) {
   return radix_sort_impl(s, in_c, out, tmp, n, in_f64, out_f64, st, true);
+}
+
+cudaError_t radix_sort_desc_f64(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,
+                                uint64_t n, cudaStream_t st) {
+  if (n < (1ull << 20)) return cudaErrorNotSupported;  // small: the codec path is as fast
+  return radix_sort_impl(s, in, out, tmp, n, true, true, st, true, true);
 }
 
 // Key/value GPUSort (S§8(f) #3): K1/K2 on the keys as in radix_sort, then every active digit

@@ -67,3 +67,20 @@ def test_host_typed(hs_gpu, oracle_mod, inputs_mod, pinned, case):
     assert np.array_equal(B.view(want.dtype), want)
     hs_gpu.hsort_sort_typed(A, A, descending=case.endswith("desc"))  # in place
     assert np.array_equal(A.view(want.dtype), want)
+
+
+@pytest.mark.parametrize("dist,n", [("salted", (1 << 20) + 7), ("special", (1 << 21) + 1),
+                                    ("uniform", (1 << 22) + 3), ("all_equal", 1 << 20)])
+def test_device_f64_descending_fused(hs_gpu, oracle_mod, inputs_mod, dist, n):
+    """Out of place, n >= 2^20: the reverse transform fused into the GPUSort (U[0,1) at 2^22 also
+    takes the dominant-digit elision in the complemented key space)."""
+    import torch
+    A = inputs_mod.generate(dist, n, seed=n % 89)
+    want = oracle_mod.sort_desc_f64(A).view(np.uint64)
+    d = torch.from_numpy(A).cuda()
+    out = torch.empty_like(d)
+    hs_gpu.hsort_sort_device_typed(d, out, True)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy().view(np.uint64), want)
+    if dist == "uniform":
+        assert hs_gpu.hsort_get_last_plan()["elided"]

@@ -236,7 +236,7 @@ int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_t
  * d_vals_out) = the pairs stably sorted by key (float64 totalOrder bits in and out if keys_f64,
  * else ascending uint64).  n <= 2^30; all four buffers 16-byte aligned (TMA tile loads); keys in
  * place iff values in place.  Same K1/K2 as hsort_sort_device, then the key/value onesweep pass
- * (4032-pair tiles) per active digit: 32 HBM bytes per pair per pass. */
+ * (4160-pair tiles) per active digit: 32 HBM bytes per pair per pass. */
 int hsort_sort_device_pairs(const uint64_t* d_keys_in, const uint64_t* d_vals_in,
                             uint64_t* d_keys_out, uint64_t* d_vals_out, uint64_t n, int keys_f64,
                             void* stream);

@@ -79,7 +79,13 @@ struct RadixScratch {
 constexpr int kNumKernelEvents = 12;
 
 constexpr int kRadixTile = 4096;  // keys per onesweep tile (THREADS x ITEMS), see radix.cu
-constexpr int kKvTile = 4032;     // pairs per key/value onesweep tile (576 x 7), see radix.cu
+#ifndef HSORT_KV_CT
+#define HSORT_KV_CT 320    // key/value pass: compute threads (10 warps) ...
+#endif
+#ifndef HSORT_KV_ITEMS
+#define HSORT_KV_ITEMS 13  // ... x pairs per thread: 4160-pair tiles, 3 stages of keys + values = 200 KB
+#endif                     // (A/B over 10 shapes: 576x7 80.4 ms, 320x13 71.3 ms per 2^30 pairs)
+constexpr int kKvTile = HSORT_KV_CT * HSORT_KV_ITEMS;  // pairs per key/value onesweep tile
 
 // dominant-digit elision on/off (option "dde", default on)
 extern bool g_dde_enabled;

@@ -1256,9 +1256,9 @@ struct WsSmem {
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
 #endif
-// key/value pass: 18 compute warps x 7 pairs (4032-pair tiles: 3 stages of keys + values = 194 KB)
-constexpr int kKvCT = 576;
-constexpr int kKvItems = 7;
+// key/value pass: HSORT_KV_CT compute threads x HSORT_KV_ITEMS pairs (internal.h: 10 warps x 13)
+constexpr int kKvCT = HSORT_KV_CT;
+constexpr int kKvItems = HSORT_KV_ITEMS;
 static_assert(kKvCT * kKvItems == kKvTile, "kKvTile (internal.h) = key/value tile");
 __device__ __forceinline__ void ld_relaxed_v4(const uint32_t* p, uint32_t* v) {
   asm volatile("ld.relaxed.gpu.global.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -1945,8 +1945,9 @@ cudaError_t radix_scratch_reserve(RadixScratch& s, uint64_t n) {
     if ((e = cudaHostAlloc(&s.h_plan, sizeof(RadixPlan), cudaHostAllocDefault)) != cudaSuccess)
       return e;
   }
-  // smallest tile of any pass kernel: the key/value pass (kKvTile keys)
-  uint64_t tiles = (n + kKvTile - 1) / kKvTile;
+  // smallest tile of any pass kernel (the TMA fallback pass, or the key/value pass)
+  constexpr uint64_t kMinTile = kKvTile < kRadixTile ? kKvTile : kRadixTile;
+  uint64_t tiles = (n + kMinTile - 1) / kMinTile;
   if (tiles < 1) tiles = 1;
   if (tiles > s.max_tiles) {
     if (s.lookback) cudaFree(s.lookback);

@@ -1,7 +1,7 @@
 """GPU parity of the key/value sort against the oracle, through the C ABI.
 
 Stable sort by key => unique result => bit-exact comparison of keys AND values.  Sizes span
-several 4032-pair tiles and ragged tails; full size (2^30 pairs) is checked by properties that pin
+several 4160-pair tiles and ragged tails; full size (2^30 pairs) is checked by properties that pin
 the unique answer when V = 0..n-1: keys equal the (oracle-pinned) key sort, pairs are preserved
 (A[VB] == B) and equal keys keep input order (VB increasing inside every run of equal keys).
 """
@@ -10,7 +10,7 @@ import pytest
 
 pytestmark = pytest.mark.gpu
 
-SIZES = [1, 2, 3, 4031, 4032, 4033, 3 * 4032 + 5, 100_003, (1 << 20) + 17]
+SIZES = [1, 2, 3, 4159, 4160, 4161, 3 * 4160 + 5, 100_003, (1 << 20) + 17]
 DISTS = ["uniform", "few_distinct", "special", "salted", "all_equal", "sorted", "reverse", "normal"]
 
 

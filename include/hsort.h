@@ -217,7 +217,8 @@ int hsort_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_byt
  * K3 onesweep passes; trivial digits are skipped on the device.  Requires hsort_init().
  * Stream-ordered, except that an out-of-place sort of n >= 2^22 keys waits once on `stream`
  * after K2 (~10 us) to read the plan: if the top active digit has a dominant value (option
- * "dde"), the host launches one pass fewer plus the outlier sort. */
+ * "dde"), the host launches one pass fewer plus the outlier sort.  That wait
+ * makes such a call not capturable into a CUDA graph: set option "dde" = 0 before capturing. */
 int hsort_sort_device(const double* d_in, double* d_out, uint64_t n, void* stream);
 
 /* Same, keys already uint64 (ascending unsigned); in_f64/out_f64 select whether the input is

@@ -210,6 +210,9 @@ int hsort_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_byt
 
 /* ---------------------------------------------------------------------------------------------
  * Device-resident entry points (current device, library-owned scratch; stream-ordered).
+ * The scratch (histograms, plan, look-back words, ping-pong buffers) is one per device: calls on
+ * one device must be ordered -- issue them from one thread on one stream, or synchronise between
+ * streams.  Concurrent calls on different devices are independent.
  * ------------------------------------------------------------------------------------------- */
 
 /* GPUSort of one batch, device -> device:  d_out = totalOrder-sorted d_in.

@@ -6,8 +6,9 @@
 //
 //   K4 k_corank     exact co-ranks (i_0..i_{k-1}) of each output-tile boundary o: the first o
 //                   keys of the merge in which equal keys are taken in run order.  One warp per
-//                   boundary, lanes own runs; bisection on the key value with per-run index
-//                   windows, the value bracket tightened to keys still inside the windows.
+//                   boundary (k <= 16: a G-lane segment, 32 / G boundaries per warp), lanes
+//                   own runs; bisection on the key value with per-run index windows, the value
+//                   bracket tightened to keys still inside the windows.
 //   K5 k_merge_tile each CTA owns one output tile [o_t, o_t+1): loads its k slices into shared
 //                   memory, merges them by a pairwise merge-path tree in shared memory, and writes
 //                   the tile with coalesced stores (inverse key transform fused).
@@ -26,23 +27,27 @@ __device__ __forceinline__ uint64_t from_key(uint64_t k) {
   return k ^ ((uint64_t)((int64_t)(~k) >> 63) | 0x8000000000000000ull);
 }
 
-__device__ __forceinline__ uint64_t warp_sum(uint64_t v) {
+// reductions over one G-lane segment (sm = the segment's lanes)
+template <int G>
+__device__ __forceinline__ uint64_t seg_sum(unsigned sm, uint64_t v) {
 #pragma unroll
-  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  for (int o = G / 2; o; o >>= 1) v += __shfl_xor_sync(sm, v, o, G);
   return v;
 }
-__device__ __forceinline__ uint64_t warp_min(uint64_t v) {
+template <int G>
+__device__ __forceinline__ uint64_t seg_min(unsigned sm, uint64_t v) {
 #pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    uint64_t w = __shfl_xor_sync(0xffffffffu, v, o);
+  for (int o = G / 2; o; o >>= 1) {
+    const uint64_t w = __shfl_xor_sync(sm, v, o, G);
     v = w < v ? w : v;
   }
   return v;
 }
-__device__ __forceinline__ uint64_t warp_max(uint64_t v) {
+template <int G>
+__device__ __forceinline__ uint64_t seg_max(unsigned sm, uint64_t v) {
 #pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    uint64_t w = __shfl_xor_sync(0xffffffffu, v, o);
+  for (int o = G / 2; o; o >>= 1) {
+    const uint64_t w = __shfl_xor_sync(sm, v, o, G);
     v = w > v ? w : v;
   }
   return v;
@@ -105,21 +110,27 @@ __device__ __forceinline__ uint64_t upper_bound_fwd(const uint64_t* a, uint64_t 
 // windows between its two coarse neighbours: with v_lo = the key at the lower coarse position and
 // v_hi = the key just before the upper one, #(< v_lo) <= o_lo <= o < o_hi <= #(<= v_hi), so the
 // bisection starts at [v_lo, v_hi] with lo/hi found by galloping from the coarse co-ranks.
-template <int C>
+template <int C, int G>
 __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ keys,
                                                 const uint64_t* __restrict__ off, int k,
                                                 uint64_t total, uint64_t step, uint64_t b0,
                                                 uint64_t nb, uint64_t* __restrict__ ranks,
                                                 const uint64_t* __restrict__ coarse,
                                                 uint64_t coarse_step, uint64_t coarse_b0) {
-  const uint64_t b = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
+  // G lanes per boundary: G = 32, or (k <= 16) the next power of two >= k, so 32 / G boundaries
+  // share a warp on their own lane segments and more dependent-load chains are in flight per SM
+  static_assert(G == 32 || C == 1, "a segment holds one chunk of runs");
+  const int seg = (threadIdx.x & 31) / G;
+  const int lane = threadIdx.x & (G - 1);
+  const unsigned sm = G == 32 ? 0xffffffffu : ((1u << G) - 1u) << (seg * G);
+  const uint64_t b =
+      (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (uint64_t)(32 / G) + seg;
   if (b >= nb) return;
   const uint64_t o = (b0 + b) * step < total ? (b0 + b) * step : total;
   uint64_t base[C], lo[C], hi[C];
 #pragma unroll
   for (int c = 0; c < C; ++c) {
-    int j = c * 32 + lane;
+    int j = c * G + lane;
     if (j < k) {
       base[c] = off[j] - off[0];
       lo[c] = 0;
@@ -134,7 +145,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
   if (o == total) {
 #pragma unroll
     for (int c = 0; c < C; ++c)
-      if (c * 32 + lane < k) out[c * 32 + lane] = hi[c];
+      if (c * G + lane < k) out[c * G + lane] = hi[c];
     return;
   }
   uint64_t L0 = 0, H0 = ~0ull;
@@ -144,21 +155,21 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
     if (o == ci * coarse_step) {  // a coarse boundary itself
 #pragma unroll
       for (int c = 0; c < C; ++c)
-        if (c * 32 + lane < k) out[c * 32 + lane] = r0[c * 32 + lane];
+        if (c * G + lane < k) out[c * G + lane] = r0[c * G + lane];
       return;
     }
     const uint64_t* r1 = r0 + k;
     uint64_t rl[C], rh[C], mn = ~0ull, mx = 0;
 #pragma unroll
     for (int c = 0; c < C; ++c) {
-      const int j = c * 32 + lane;
+      const int j = c * G + lane;
       rl[c] = j < k ? r0[j] : 0;
       rh[c] = j < k ? r1[j] : 0;
       if (rl[c] < hi[c]) mn = K[base[c] + rl[c]] < mn ? K[base[c] + rl[c]] : mn;
       if (rh[c] > 0) mx = K[base[c] + rh[c] - 1] > mx ? K[base[c] + rh[c] - 1] : mx;
     }
-    L0 = warp_min(mn);  // key at merged position o_lo
-    H0 = warp_max(mx);  // key at merged position o_hi - 1
+    L0 = seg_min<G>(sm, mn);  // key at merged position o_lo
+    H0 = seg_max<G>(sm, mx);  // key at merged position o_hi - 1
 #pragma unroll
     for (int c = 0; c < C; ++c) {
       const uint64_t len = hi[c];
@@ -182,8 +193,8 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
         mx = z > mx ? z : mx;
       }
     }
-    mn = warp_min(mn);
-    mx = warp_max(mx);
+    mn = seg_min<G>(sm, mn);
+    mx = seg_max<G>(sm, mx);
     if (mn > L) L = mn;
     if (mx < H) H = mx;
     if (L >= H) break;
@@ -196,7 +207,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
       s += ub[c];
     }
     // elements <= mid overall: the window searches count from index 0 (lo/hi are absolute)
-    s = warp_sum(s);
+    s = seg_sum<G>(sm, s);
     if (s > o) {
       H = mid;
 #pragma unroll
@@ -226,7 +237,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
     eq[c] = u - l2;
     lt += l2;
   }
-  lt = warp_sum(lt);
+  lt = seg_sum<G>(sm, lt);
   // take the o - lt keys equal to v in run order (j = c*32 + lane)
   uint64_t rem = o - lt;
 #pragma unroll
@@ -234,14 +245,14 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
     uint64_t e = eq[c];
     uint64_t x = e;  // inclusive scan over lanes
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      uint64_t y = __shfl_up_sync(0xffffffffu, x, d);
+    for (int d = 1; d < G; d <<= 1) {
+      uint64_t y = __shfl_up_sync(sm, x, d, G);
       if (lane >= d) x += y;
     }
     uint64_t excl = x - e;
-    uint64_t tot = __shfl_sync(0xffffffffu, x, 31);
+    uint64_t tot = __shfl_sync(sm, x, G - 1, G);
     uint64_t take = rem > excl ? (rem - excl < e ? rem - excl : e) : 0;
-    if (c * 32 + lane < k) out[c * 32 + lane] = lo[c] + take;
+    if (c * G + lane < k) out[c * G + lane] = lo[c] + take;
     rem = rem > tot ? rem - tot : 0;
   }
 }
@@ -504,21 +515,31 @@ size_t merge_smem_bytes(int k) {
 
 }  // namespace
 
+#ifndef HSORT_CORANK_SEG
+#define HSORT_CORANK_SEG 1  // k <= 16: 32 / G co-rank searches per warp (K4)
+#endif
+constexpr bool kCorankSeg = HSORT_CORANK_SEG != 0;
+
 namespace {
 cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
                           uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
                           const uint64_t* coarse, uint64_t cstep, uint64_t cb0, cudaStream_t st) {
-  const unsigned grid = (unsigned)((n_bounds * 32 + 127) / 128);
   const int C = (k + 31) / 32;
-#define HS_CORANK(CC)                                                                              \
-  k_corank<CC><<<grid, 128, 0, st>>>(keys, d_off, k, total, step, bound_begin, n_bounds, ranks,    \
-                                     coarse, cstep, cb0)
-  if (C <= 1) HS_CORANK(1);
+#define HS_CORANK_G(CC, GG)                                                                        \
+  k_corank<CC, GG><<<(unsigned)((n_bounds * GG + 127) / 128), 128, 0, st>>>(                      \
+      keys, d_off, k, total, step, bound_begin, n_bounds, ranks, coarse, cstep, cb0)
+#define HS_CORANK(CC) HS_CORANK_G(CC, 32)
+  if (kCorankSeg && k <= 2) HS_CORANK_G(1, 2);
+  else if (kCorankSeg && k <= 4) HS_CORANK_G(1, 4);
+  else if (kCorankSeg && k <= 8) HS_CORANK_G(1, 8);
+  else if (kCorankSeg && k <= 16) HS_CORANK_G(1, 16);
+  else if (C <= 1) HS_CORANK(1);
   else if (C <= 2) HS_CORANK(2);
   else if (C <= 4) HS_CORANK(4);
   else if (C <= 8) HS_CORANK(8);
   else HS_CORANK(kMaxC);
 #undef HS_CORANK
+#undef HS_CORANK_G
   return cudaGetLastError();
 }
 }  // namespace

@@ -6,7 +6,7 @@
 //
 //   K4 k_corank     exact co-ranks (i_0..i_{k-1}) of each output-tile boundary o: the first o
 //                   keys of the merge in which equal keys are taken in run order.  One warp per
-//                   boundary (k <= 16: a G-lane segment, 32 / G boundaries per warp), lanes
+//                   boundary (k <= 32: a G-lane segment, 32 / G boundaries per warp), lanes
 //                   own runs; bisection on the key value with per-run index windows, the value
 //                   bracket tightened to keys still inside the windows.
 //   K5 k_merge_tile each CTA owns one output tile [o_t, o_t+1): loads its k slices into shared
@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
                                                 uint64_t coarse_step, uint64_t coarse_b0) {
   // G lanes per boundary: G = 32, or (k <= 16) the next power of two >= k, so 32 / G boundaries
   // share a warp on their own lane segments and more dependent-load chains are in flight per SM
-  static_assert(G == 32 || C == 1, "a segment holds one chunk of runs");
+  // a segment holds C chunks of G runs: run j = c G + lane
   const int seg = (threadIdx.x & 31) / G;
   const int lane = threadIdx.x & (G - 1);
   const unsigned sm = G == 32 ? 0xffffffffu : ((1u << G) - 1u) << (seg * G);
@@ -519,6 +519,10 @@ size_t merge_smem_bytes(int k) {
 #define HSORT_CORANK_SEG 1  // k <= 16: 32 / G co-rank searches per warp (K4)
 #endif
 constexpr bool kCorankSeg = HSORT_CORANK_SEG != 0;
+#ifndef HSORT_CORANK_SEG2
+#define HSORT_CORANK_SEG2 1  // 16 < k <= 32: two 16-lane segments per warp, 2 runs per lane
+#endif
+constexpr bool kCorankSeg2 = HSORT_CORANK_SEG2 != 0;
 
 namespace {
 cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
@@ -533,6 +537,7 @@ cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, ui
   else if (kCorankSeg && k <= 4) HS_CORANK_G(1, 4);
   else if (kCorankSeg && k <= 8) HS_CORANK_G(1, 8);
   else if (kCorankSeg && k <= 16) HS_CORANK_G(1, 16);
+  else if (kCorankSeg2 && k <= 32) HS_CORANK_G(2, 16);
   else if (C <= 1) HS_CORANK(1);
   else if (C <= 2) HS_CORANK(2);
   else if (C <= 4) HS_CORANK(4);

@@ -6,7 +6,7 @@
 //
 //   K4 k_corank     exact co-ranks (i_0..i_{k-1}) of each output-tile boundary o: the first o
 //                   keys of the merge in which equal keys are taken in run order.  One warp per
-//                   boundary (k <= 32: a G-lane segment, 32 / G boundaries per warp), lanes
+//                   boundary (k <= 128: a G-lane segment, 32 / G boundaries per warp), lanes
 //                   own runs; bisection on the key value with per-run index windows, the value
 //                   bracket tightened to keys still inside the windows.
 //   K5 k_merge_tile each CTA owns one output tile [o_t, o_t+1): loads its k slices into shared
@@ -523,6 +523,11 @@ constexpr bool kCorankSeg = HSORT_CORANK_SEG != 0;
 #define HSORT_CORANK_SEG2 1  // 16 < k <= 32: two 16-lane segments per warp, 2 runs per lane
 #endif
 constexpr bool kCorankSeg2 = HSORT_CORANK_SEG2 != 0;
+#ifndef HSORT_CORANK_ILP
+#define HSORT_CORANK_ILP 1  // 32 < k <= 128: 16-lane segments, k / 16 runs per lane (2 runs per
+                            // lane at k <= 16 was measured 18-30% slower)
+#endif
+constexpr bool kCorankIlp = HSORT_CORANK_ILP != 0;
 
 namespace {
 cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
@@ -533,7 +538,9 @@ cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, ui
   k_corank<CC, GG><<<(unsigned)((n_bounds * GG + 127) / 128), 128, 0, st>>>(                      \
       keys, d_off, k, total, step, bound_begin, n_bounds, ranks, coarse, cstep, cb0)
 #define HS_CORANK(CC) HS_CORANK_G(CC, 32)
-  if (kCorankSeg && k <= 2) HS_CORANK_G(1, 2);
+  if (kCorankIlp && k > 32 && k <= 64) HS_CORANK_G(4, 16);
+  else if (kCorankIlp && k > 64 && k <= 128) HS_CORANK_G(8, 16);
+  else if (kCorankSeg && k <= 2) HS_CORANK_G(1, 2);
   else if (kCorankSeg && k <= 4) HS_CORANK_G(1, 4);
   else if (kCorankSeg && k <= 8) HS_CORANK_G(1, 8);
   else if (kCorankSeg && k <= 16) HS_CORANK_G(1, 16);

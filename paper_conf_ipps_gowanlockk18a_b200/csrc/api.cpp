@@ -120,6 +120,11 @@ struct Options {
       {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
       {"pin_w", -1},                 // STREAM W: 1 cached pinned, 0 pageable, -1 pinned if <= pin_w_max_mb
       {"pin_w_max_mb", 16384},       // auto pinning limit: pinning runs at ~2.5 GB/s
+      {"virtual_gpus", 0},           // > 0 (set before hsort_init): that many GPU contexts mapped
+                                     // round-robin onto the visible devices (multi-GPU scheduler,
+                                     // exchange and merge testable on one GPU)
+      {"register_host", 0},          // 1: page-lock pageable A/B for the call (cudaHostRegister) and
+                                     // DMA them directly instead of staging through the ring
   };
   int64_t get(const char* k) const { return v.at(k); }
 };
@@ -129,6 +134,8 @@ struct GpuCtx {
   cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
   RadixScratch rs;
   DevBuf runs, alt, mout, min, ranks, off;
+  DevBuf coarse;       // K4's coarse-level co-rank table (two-level search)
+  DevBuf rptr;         // multi-GPU merge: device table of run pointers (peer HBM)
   DevBuf vruns, valt;  // key/value sorts: values and their ping-pong scratch
   DevBuf tmp3;         // typed sorts: third key buffer, so the GPUSort runs out of place (elision)
   std::vector<char*> ring_in, ring_out;
@@ -151,6 +158,8 @@ struct State {
   void* w_pin = nullptr;
   size_t w_pin_bytes = 0;
   double r_cpu_merge = 0;  // last measured CPU merge rate (keys/s), for the A12 split
+  bool peer_ok = true;     // every pair of devices in use can read each other's HBM
+  int n_physical = 0;      // visible CUDA devices
 };
 State& S() {
   static State s;
@@ -303,42 +312,98 @@ std::vector<uint64_t> batch_offsets(uint64_t n, uint64_t b_s, int schedule) {
   return offs;
 }
 
+// Cut [0, n) into N contiguous parts whose inner bounds are multiples of `align` (shards of A
+// per GPU, output ranges of B per GPU).
+std::vector<uint64_t> shard_bounds(uint64_t n, int N, uint64_t align) {
+  std::vector<uint64_t> b(N + 1, 0);
+  for (int g = 1; g < N; ++g) {
+    const uint64_t x = (uint64_t)((unsigned __int128)n * (unsigned)g / (unsigned)N);
+    b[g] = std::max(b[g - 1], x - x % align);
+  }
+  b[N] = n;
+  return b;
+}
+
+// Batches of a RESIDENT plan over N GPUs: shard g of A (shard_bounds, tile-aligned) is cut by
+// batch_offsets(shard, b_s, schedule); the run count is the sum over the shards.
+uint64_t resident_runs(uint64_t n, int N, uint64_t b_s, int schedule, uint64_t* shard_max) {
+  const std::vector<uint64_t> sh = shard_bounds(n, N, kRadixTile);
+  uint64_t runs = 0, mx = 0;
+  for (int g = 0; g < N; ++g) {
+    const uint64_t m = sh[g + 1] - sh[g];
+    if (schedule == 0 || m / std::max<uint64_t>(b_s, 1) > 4 * (uint64_t)kMaxMergeRuns)
+      runs += (m + b_s - 1) / std::max<uint64_t>(b_s, 1);  // closed form (no schedule vector)
+    else
+      runs += batch_offsets(m, b_s, schedule).size() - 1;
+    mx = std::max(mx, sh[g + 1] - sh[g]);
+  }
+  if (shard_max) *shard_max = mx;
+  return runs;
+}
+
+// A1.  device_bytes = usable HBM per GPU; multi_ok = the GPUs can read each other's HBM (peer
+// access; required by the multi-GPU RESIDENT merge).
 hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t device_bytes,
-                       const Options& opt) {
+                       const Options& opt, bool multi_ok = true) {
   hsort_plan_t p{};
   p.n = n;
   p.n_gpus = n_gpus;
   int n_s = (int)std::max<int64_t>(1, opt.get("n_s"));
   uint64_t reserve = (uint64_t)std::max<int64_t>(0, opt.get("device_reserve_mb")) << 20;
-  uint64_t merge_buf = 2ull * (uint64_t)opt.get("merge_chunk") * 8;
+  const uint64_t mchunk = (uint64_t)opt.get("merge_chunk");
+  uint64_t merge_buf = 2ull * mchunk * 8;
   uint64_t budget = device_bytes > reserve ? device_bytes - reserve : 0;
   // single batch footprint: keys + alt + look-back
   auto bline_bytes = [&](uint64_t b) { return (uint64_t)(b * (16.0 + kLookbackBytesPerKey)); };
-  uint64_t b_s;
   int64_t res = opt.get("resident");
-  // auto plan for an array that fits in HBM: a pipelined RESIDENT schedule (HtoD of batch i+1
-  // overlaps the sort of batch i; the merge overlaps the DtoH) beats BLINE's serial
-  // HtoD -> sort -> DtoH once n is large enough for the overlap to matter.
+  const uint64_t host_ring = 2ull * (uint64_t)opt.get("n_ring") * (uint64_t)opt.get("p_s");
+  // RESIDENT footprint per GPU: its shard's runs + one batch of radix scratch + the merge slots,
+  // co-rank rows and coarse table (k runs)
+  auto resident_bytes = [&](uint64_t shard, uint64_t b, uint64_t k) {
+    return shard * 8 + (uint64_t)(b * (8.0 + kLookbackBytesPerKey)) + merge_buf +
+           4 * (mchunk / kMergeTile + 2) * std::max<uint64_t>(k, 1) * 8 + k * 16;
+  };
+  auto set_resident = [&](uint64_t b, int schedule, int N, uint64_t runs, uint64_t bytes) {
+    p.b_s = b;
+    p.schedule = schedule;
+    p.n_b = runs;
+    const std::vector<uint64_t> sh = shard_bounds(n, N, kRadixTile);
+    const std::vector<uint64_t> offs = batch_offsets(sh[N] - sh[N - 1], b, schedule);
+    p.last_batch = offs.size() > 1 ? offs[offs.size() - 1] - offs[offs.size() - 2] : 0;
+    p.n_s = 1;
+    p.n_gpus = N;
+    p.mode = HSORT_MODE_RESIDENT;
+    p.device_bytes_per_gpu = bytes;
+    p.host_bytes = host_ring * (uint64_t)N;
+    p.batches_per_stream = (double)runs / N;
+    return p;
+  };
+  // Pipelined RESIDENT plan (the auto plan for arrays whose runs fit in HBM, on one or N GPUs):
+  // 2^27-key batches + a halving tail per shard, so HtoD of batch i+1 overlaps the sort of batch i
+  // and the merge overlaps the DtoH.  With an explicit batch_elems the shards are
+  // cut into uniform b_s batches instead (schedule 0).
   const uint64_t auto_min = (uint64_t)std::max<int64_t>(0, opt.get("auto_pipeline_min"));
-  if (batch_elems == 0 && auto_min && n >= auto_min && n_gpus == 1 && res != 0) {
-    uint64_t b0 = std::min<uint64_t>(1ull << 27, std::max<uint64_t>(n / 8, kRadixTile));
-    b0 -= b0 % kRadixTile;
-    const uint64_t rb = n * 8 + (uint64_t)(b0 * (8.0 + kLookbackBytesPerKey)) + merge_buf +
-                        4 * ((uint64_t)opt.get("merge_chunk") / kMergeTile + 1) * 64 * 8;
-    if (rb <= budget) {
-      p.b_s = b0;
-      p.schedule = 1;
-      std::vector<uint64_t> offs = batch_offsets(n, b0, 1);
-      p.n_b = offs.size() - 1;
-      p.last_batch = offs[p.n_b] - offs[p.n_b - 1];
-      p.n_s = 1;
-      p.mode = HSORT_MODE_RESIDENT;
-      p.device_bytes_per_gpu = rb;
-      p.host_bytes = 2ull * (uint64_t)opt.get("n_ring") * (uint64_t)opt.get("p_s");
-      p.batches_per_stream = (double)p.n_b;
-      return p;
+  const int N = std::max(1, n_gpus);
+  const bool multi = N > 1 && multi_ok;
+  if (n > 0 && res != 0 && (N == 1 || multi)) {
+    uint64_t smax = 0;  // largest shard
+    const std::vector<uint64_t> sh = shard_bounds(n, N, kRadixTile);
+    for (int g = 0; g < N; ++g) smax = std::max(smax, sh[g + 1] - sh[g]);
+    if (batch_elems == 0 && auto_min && n >= auto_min) {
+      uint64_t b0 = std::min<uint64_t>(1ull << 27, std::max<uint64_t>(smax / 8, kRadixTile));
+      b0 -= b0 % kRadixTile;
+      const uint64_t runs = resident_runs(n, N, b0, 1, nullptr);
+      const uint64_t rb = resident_bytes(smax, b0, runs);
+      if (runs <= (uint64_t)kMaxMergeRuns && rb <= budget) return set_resident(b0, 1, N, runs, rb);
+    } else if (multi && batch_elems > 0 && batch_elems < n) {
+      const uint64_t b = std::min<uint64_t>(batch_elems, std::max<uint64_t>(smax, 1));
+      const uint64_t runs = resident_runs(n, N, b, 0, nullptr);
+      const uint64_t rb = resident_bytes(smax, b, runs);
+      if (runs <= (uint64_t)kMaxMergeRuns && (res == 1 || rb <= budget))
+        return set_resident(b, 0, N, runs, rb);
     }
   }
+  uint64_t b_s;
   if (batch_elems == 0) {
     if (bline_bytes(n) <= budget) {
       b_s = n;
@@ -348,6 +413,7 @@ hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t de
       b_s = (uint64_t)((double)budget / per);
       b_s -= b_s % kRadixTile;
       if (b_s == 0) b_s = kRadixTile;
+      b_s = std::min<uint64_t>(b_s, 1ull << 30);  // the fast onesweep pass handles n <= 2^30
     }
   } else {
     b_s = std::min<uint64_t>(batch_elems, n ? n : 1);
@@ -357,23 +423,22 @@ hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t de
   p.n_b = n ? (n + b_s - 1) / b_s : 0;
   p.last_batch = n ? n - (p.n_b - 1) * b_s : 0;
   p.n_s = p.n_b <= 1 ? 1 : (int)std::min<uint64_t>((uint64_t)n_s, p.n_b);
-  uint64_t resident_bytes = n * 8 + (uint64_t)(b_s * (8.0 + kLookbackBytesPerKey)) + merge_buf +
-                            ((n / kMergeTile + 2) * std::min<uint64_t>(p.n_b, kMaxMergeRuns) * 8);
+  const uint64_t rb1 = resident_bytes(n, b_s, std::min<uint64_t>(p.n_b, kMaxMergeRuns));
   if (p.n_b <= 1) {
     p.mode = HSORT_MODE_BLINE;
     p.device_bytes_per_gpu = bline_bytes(n);
-    p.n_gpus = std::min(n_gpus, 1);
-    if (n_gpus >= 1) p.n_gpus = 1;
-  } else if (n_gpus == 1 && p.n_b <= (uint64_t)kMaxMergeRuns &&
-             (res == 1 || (res == -1 && resident_bytes <= budget))) {
+    p.n_gpus = 1;
+  } else if (N == 1 && p.n_b <= (uint64_t)kMaxMergeRuns &&
+             (res == 1 || (res == -1 && rb1 <= budget))) {
     p.mode = HSORT_MODE_RESIDENT;
-    p.device_bytes_per_gpu = resident_bytes;
+    p.device_bytes_per_gpu = rb1;
+    p.n_gpus = 1;
   } else {
     p.mode = HSORT_MODE_STREAM;
+    p.n_gpus = (int)std::min<uint64_t>((uint64_t)N, p.n_b);
     p.device_bytes_per_gpu = (uint64_t)(b_s * (8.0 * (p.n_s + 1) + kLookbackBytesPerKey));
   }
-  p.host_bytes = (p.mode == HSORT_MODE_STREAM ? n * 8 : 0) +
-                 2ull * (uint64_t)opt.get("n_ring") * (uint64_t)opt.get("p_s") * (uint64_t)std::max(1, p.n_gpus);
+  p.host_bytes = (p.mode == HSORT_MODE_STREAM ? n * 8 : 0) + host_ring * (uint64_t)std::max(1, p.n_gpus);
   p.batches_per_stream = p.n_b ? (double)p.n_b / ((double)p.n_s * std::max(1, p.n_gpus)) : 0.0;
   return p;
 }
@@ -427,19 +492,79 @@ void sort_bline(GpuCtx& g, CallCtx& c) {
   ed.destroy();
 }
 
-// GPU merge of k resident runs (K4 + K5), chunk by chunk: the co-ranks of chunk c are computed
-// just before its merge, and the DtoH of chunk c overlaps the merge of chunk c+1 (two output
-// slots), so the first bytes leave the GPU one chunk after the last batch is sorted.
-void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std::vector<uint64_t>& h_off,
-                       Acc& acc, double* t_merge_gpu, double* t_d2h) {
-  const int k = (int)h_off.size() - 1;
-  const uint64_t total = h_off[k] - h_off[0];
-  g.off.reserve((k + 1) * 8);
-  CK(cudaMemcpyAsync(g.off.p, h_off.data(), (k + 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
-  const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
+// Per-GPU accumulators of one call (each GPU's host thread owns one; summed into hsort_stats).
+struct PhaseTimes {
+  Acc acc;
+  double t_h2d = 0, t_sort = 0, t_d2h = 0, t_merge = 0;
+  int passes = 0;
+};
+
+// Run fn(i) for i in [0, N) on N host threads (inline when N == 1); the first failure is
+// rethrown after every thread has joined.
+template <class F>
+void run_per_gpu(size_t N, F fn) {
+  if (N == 1) {
+    fn(0);
+    return;
+  }
+  std::mutex m;
+  int code = 0;
+  std::string msg;
+  std::vector<std::thread> th;
+  for (size_t i = 0; i < N; ++i)
+    th.emplace_back([&, i] {
+      auto fail = [&](int c, const std::string& w) {
+        std::lock_guard<std::mutex> g(m);
+        if (!code) {
+          code = c;
+          msg = w;
+        }
+      };
+      try {
+        fn(i);
+      } catch (const HsortError& e) {
+        fail(e.code, e.what());
+      } catch (const std::bad_alloc&) {
+        fail(HSORT_ERR_HOST_OOM, "host allocation failed");
+      } catch (const std::exception& e) {
+        fail(HSORT_ERR_INTERNAL, e.what());
+      } catch (...) {
+        fail(HSORT_ERR_INTERNAL, "unknown exception");
+      }
+    });
+  for (auto& t : th) t.join();
+  if (code) throw HsortError(code, msg);
+}
+
+// K4 on g.s_comp with the library-owned coarse-level scratch of this GPU context.
+void corank_on(GpuCtx& g, const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+               int k, uint64_t total, uint64_t step, uint64_t b0, uint64_t nb, uint64_t* ranks,
+               cudaStream_t st) {
+  const uint64_t need = merge_corank_scratch_elems(k, total, step, b0, nb);
+  if (need * 8 > g.coarse.cap) {
+    CK(cudaStreamSynchronize(st));  // the buffer may still be read by an earlier K4 on st
+    g.coarse.reserve(need * 8);
+  }
+  CK(merge_corank(keys, rp, d_off, k, total, step, b0, nb, ranks, g.coarse.u64(), g.coarse.cap / 8, st));
+}
+
+// GPU merge (K4 + K5) of the k runs (keys | rp, d_off; `total` keys) -- output positions
+// [o_lo, o_hi) into B + o_lo, chunk by chunk: the co-ranks of chunk c are computed just before
+// its merge, and the DtoH of chunk c overlaps the merge of chunk c+1 (two output slots), so the
+// first bytes leave the GPU one chunk after the last batch is sorted.  o_lo is a multiple of
+// kMergeTile (a merge tile boundary); o_hi is one too, or total.  With rp the runs are read where
+// they lie, including other GPUs' HBM over NVLink (peer access): the multi-GPU exchange is fused
+// into K4/K5's loads.
+void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_keys, const uint64_t* const* d_rp,
+                       const uint64_t* d_off, int k, uint64_t total, uint64_t o_lo, uint64_t o_hi,
+                       PhaseTimes& pt) {
+  if (o_hi <= o_lo) return;
+  const uint64_t t_lo = o_lo / kMergeTile;
+  const uint64_t t_hi = (o_hi + kMergeTile - 1) / kMergeTile;
+  const uint64_t tiles = t_hi - t_lo;
   const uint64_t ctiles = std::max<uint64_t>(1, (uint64_t)S().opt.get("merge_chunk") / kMergeTile);
   const uint64_t chunk = ctiles * kMergeTile;
-  const uint64_t nch = (total + chunk - 1) / chunk;
+  const uint64_t nch = (tiles + ctiles - 1) / ctiles;
   const uint64_t slots = nch > 1 ? 2 : 1;
   g.mout.reserve(slots * chunk * 8);
   g.ranks.reserve(slots * (ctiles + 1) * (uint64_t)k * 8);
@@ -457,13 +582,13 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std:
   char* B = (char*)c.B;
   auto enqueue_merge = [&](uint64_t ch) {
     const uint64_t s = ch % slots;
-    const uint64_t tb = ch * ctiles, tc = std::min(ctiles, tiles - tb);
+    const uint64_t tb = t_lo + ch * ctiles, tc = std::min(ctiles, t_hi - tb);
     uint64_t* rk = g.ranks.u64() + s * (ctiles + 1) * (uint64_t)k;
     CK(cudaStreamWaitEvent(g.s_comp, ev_free[s], 0));
     CK(cudaEventRecord(em[ch].a, g.s_comp));
-    CK(merge_corank(d_runs, g.off.u64(), k, total, kMergeTile, tb, tc + 1, rk, g.s_comp));
-    CK(merge_tiles(d_runs, g.off.u64(), k, total, rk, tb, tb, tc, g.mout.u64() + s * chunk,
-                   ch * chunk, c.f64, g.s_comp));
+    corank_on(g, d_keys, d_rp, d_off, k, total, kMergeTile, tb, tc + 1, rk, g.s_comp);
+    CK(merge_tiles(d_keys, d_rp, d_off, k, total, rk, tb, tb, tc, g.mout.u64() + s * chunk,
+                   tb * kMergeTile, c.f64, g.s_comp));
     CK(cudaEventRecord(em[ch].b, g.s_comp));
     CK(cudaEventRecord(ev_done[s], g.s_comp));
   };
@@ -471,18 +596,19 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std:
   for (uint64_t ch = 0; ch < nch; ++ch) {
     if (ch + 1 < nch) enqueue_merge(ch + 1);
     const uint64_t s = ch % slots;
-    const uint64_t o = ch * chunk, len = std::min(chunk, total - o);
+    const uint64_t o = (t_lo + ch * ctiles) * kMergeTile, len = std::min(chunk, o_hi - o);
     CK(cudaStreamWaitEvent(g.s_d2h, ev_done[s], 0));
     CK(cudaEventRecord(ed[ch].a, g.s_d2h));
-    download(g, B + o * 8, g.mout.u64() + s * chunk, len * 8, g.s_d2h, c.direct_out, c.mc_threads, acc);
+    download(g, B + o * 8, g.mout.u64() + s * chunk, len * 8, g.s_d2h, c.direct_out, c.mc_threads,
+             pt.acc);
     CK(cudaEventRecord(ed[ch].b, g.s_d2h));
     CK(cudaEventRecord(ev_free[s], g.s_d2h));
   }
   CK(cudaStreamSynchronize(g.s_d2h));
   CK(cudaStreamSynchronize(g.s_comp));
   for (uint64_t ch = 0; ch < nch; ++ch) {
-    *t_merge_gpu += em[ch].ms() / 1e3;
-    *t_d2h += ed[ch].ms() / 1e3;
+    pt.t_merge += em[ch].ms() / 1e3;
+    pt.t_d2h += ed[ch].ms() / 1e3;
     em[ch].destroy();
     ed[ch].destroy();
   }
@@ -492,23 +618,26 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_runs, const std:
   }
 }
 
-void sort_resident(GpuCtx& g, CallCtx& c) {
+// Sort phase of the RESIDENT mode on one GPU: the batches [h_off[i], h_off[i+1]) of the shard
+// A + a0 are HtoD'd into g.runs at the same offsets and sorted in place (runs stay in HBM, in key
+// form); the HtoD of batch i+1 overlaps the sort of batch i.
+void resident_sort_phase(GpuCtx& g, CallCtx& c, uint64_t a0, const std::vector<uint64_t>& h_off,
+                         PhaseTimes& pt) {
   CK(cudaSetDevice(g.dev));
-  const uint64_t n = c.n, b_s = c.plan.b_s, n_b = c.plan.n_b;
-  const std::vector<uint64_t> h_off = batch_offsets(n, b_s, c.plan.schedule);
-  if (h_off.size() != n_b + 1) throw HsortError(HSORT_ERR_INTERNAL, "batch schedule mismatch");
-  g.runs.reserve(n * 8);
-  g.alt.reserve(b_s * 8);
-  Acc acc;
-  std::vector<EvPair> eh(n_b), es(n_b);
+  const uint64_t nb = h_off.size() - 1, shard = h_off[nb];
+  if (shard == 0) return;
+  uint64_t bmax = 0;
+  for (uint64_t i = 0; i < nb; ++i) bmax = std::max(bmax, h_off[i + 1] - h_off[i]);
+  g.runs.reserve(shard * 8);
+  g.alt.reserve(bmax * 8);
+  std::vector<EvPair> eh(nb), es(nb);
   for (auto& e : eh) e.make();
   for (auto& e : es) e.make();
-  auto t0 = Clock::now();
-  int passes = 0;
-  for (uint64_t i = 0; i < n_b; ++i) {
+  for (uint64_t i = 0; i < nb; ++i) {
     const uint64_t o = h_off[i], len = h_off[i + 1] - h_off[i];
     CK(cudaEventRecord(eh[i].a, g.s_h2d));
-    upload(g, g.runs.u64() + o, (const char*)c.A + o * 8, len * 8, g.s_h2d, c.direct_in, c.mc_threads, acc);
+    upload(g, g.runs.u64() + o, (const char*)c.A + (a0 + o) * 8, len * 8, g.s_h2d, c.direct_in,
+           c.mc_threads, pt.acc);
     CK(cudaEventRecord(eh[i].b, g.s_h2d));
     CK(cudaStreamWaitEvent(g.s_comp, eh[i].b, 0));
     CK(cudaEventRecord(es[i].a, g.s_comp));
@@ -516,26 +645,75 @@ void sort_resident(GpuCtx& g, CallCtx& c) {
     CK(cudaEventRecord(es[i].b, g.s_comp));
   }
   CK(cudaStreamSynchronize(g.s_comp));
-  passes = g.rs.h_plan->num_active;  // plan of the last batch
-  c.st->t_sort_phase = secs_since(t0);
-  auto t1 = Clock::now();
-  double tmg = 0, tdh = 0;
-  gpu_merge_to_host(g, c, g.runs.u64(), h_off, acc, &tmg, &tdh);
-  c.st->t_merge_phase = secs_since(t1);
-  c.st->t_merge_gpu = tmg;
-  c.st->t_d2h = tdh;
-  c.st->merge_gpu_fraction = 1.0;
-  for (uint64_t i = 0; i < n_b; ++i) {
-    c.st->t_h2d += eh[i].ms() / 1e3;
-    c.st->t_gpu_sort += es[i].ms() / 1e3;
+  pt.passes = g.rs.h_plan->num_active;  // plan of the last batch
+  for (uint64_t i = 0; i < nb; ++i) {
+    pt.t_h2d += eh[i].ms() / 1e3;
+    pt.t_sort += es[i].ms() / 1e3;
   }
-  c.st->t_stage = acc.t_stage;
-  c.st->bytes_h2d = acc.h2d;
-  c.st->bytes_d2h = acc.d2h;
-  c.st->passes_run = passes;
-  c.st->passes_skipped = 8 - passes;
   for (auto& e : eh) e.destroy();
   for (auto& e : es) e.destroy();
+}
+
+// RESIDENT mode over N >= 1 GPUs (A1 picks it when the runs fit in N x HBM):
+//  1. A is cut into N contiguous shards; GPU g sorts shard g as batches that stay resident
+//     (n_b/(n_s n_GPU) batches per stream), every GPU on its own host thread;
+//  2. the output B is cut into N ranges at merge-tile boundaries; GPU g merges its range from ALL
+//     runs (K4 co-ranks + K5 tiles reading the other GPUs' runs by peer loads: the splitter
+//     exchange, S§8(a) A13, fused into the merge) and DMAs it straight to B[o_g, o_{g+1}).
+// With N = 1 this is the single-GPU RESIDENT schedule (runs back to back in g.runs, no table).
+void sort_resident(std::vector<GpuCtx*>& gs, CallCtx& c) {
+  const size_t N = gs.size();
+  const uint64_t n = c.n;
+  const std::vector<uint64_t> shard = shard_bounds(n, (int)N, kRadixTile);
+  std::vector<std::vector<uint64_t>> h_off(N);
+  uint64_t n_runs = 0;
+  for (size_t g = 0; g < N; ++g) {
+    h_off[g] = batch_offsets(shard[g + 1] - shard[g], c.plan.b_s, c.plan.schedule);
+    n_runs += h_off[g].size() - 1;
+  }
+  if (n_runs != c.plan.n_b) throw HsortError(HSORT_ERR_INTERNAL, "batch schedule mismatch");
+  std::vector<PhaseTimes> pt(N);
+  auto t0 = Clock::now();
+  run_per_gpu(N, [&](size_t g) { resident_sort_phase(*gs[g], c, shard[g], h_off[g], pt[g]); });
+  c.st->t_sort_phase = secs_since(t0);
+  // the global run table (run order: GPU-major, then batch): device pointers and offsets
+  std::vector<const uint64_t*> rp;
+  std::vector<uint64_t> goff{0};
+  for (size_t g = 0; g < N; ++g)
+    for (size_t i = 0; i + 1 < h_off[g].size(); ++i) {
+      rp.push_back(gs[g]->runs.u64() + h_off[g][i]);
+      goff.push_back(goff.back() + h_off[g][i + 1] - h_off[g][i]);
+    }
+  const int k = (int)rp.size();
+  const std::vector<uint64_t> orng = shard_bounds(n, (int)N, kMergeTile);
+  auto t1 = Clock::now();
+  run_per_gpu(N, [&](size_t gi) {
+    GpuCtx& g = *gs[gi];
+    CK(cudaSetDevice(g.dev));
+    g.off.reserve((k + 1) * 8);
+    CK(cudaMemcpyAsync(g.off.p, goff.data(), (k + 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
+    if (N == 1) {
+      gpu_merge_to_host(g, c, g.runs.u64(), nullptr, g.off.u64(), k, n, 0, n, pt[gi]);
+    } else {
+      g.rptr.reserve(k * sizeof(void*));
+      CK(cudaMemcpyAsync(g.rptr.p, rp.data(), k * sizeof(void*), cudaMemcpyHostToDevice, g.s_comp));
+      gpu_merge_to_host(g, c, nullptr, (const uint64_t* const*)g.rptr.p, g.off.u64(), k, n,
+                        orng[gi], orng[gi + 1], pt[gi]);
+    }
+  });
+  c.st->t_merge_phase = secs_since(t1);
+  c.st->merge_gpu_fraction = 1.0;
+  for (auto& P : pt) {
+    c.st->t_h2d += P.t_h2d;
+    c.st->t_gpu_sort += P.t_sort;
+    c.st->t_merge_gpu += P.t_merge;
+    c.st->t_d2h += P.t_d2h;
+    c.st->t_stage += P.acc.t_stage;
+    c.st->bytes_h2d += P.acc.h2d;
+    c.st->bytes_d2h += P.acc.d2h;
+    c.st->passes_run = std::max(c.st->passes_run, P.passes);
+  }
+  c.st->passes_skipped = 8 - c.st->passes_run;
 }
 
 // GPU share of the STREAM merge: output positions [o_lo, o_hi) of the merge of the k runs in
@@ -596,8 +774,8 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
     uint64_t* dout = g.mout.u64() + (uint64_t)s * C;
     CK(cudaStreamWaitEvent(g.s_comp, in_ready[s], 0));
     CK(cudaStreamWaitEvent(g.s_comp, out_free[s], 0));
-    CK(merge_corank(din, doff, k, total, kMergeTile, 0, tiles + 1, rk, g.s_comp));
-    CK(merge_tiles(din, doff, k, total, rk, 0, 0, tiles, dout, 0, c.f64, g.s_comp));
+    corank_on(g, din, nullptr, doff, k, total, kMergeTile, 0, tiles + 1, rk, g.s_comp);
+    CK(merge_tiles(din, nullptr, doff, k, total, rk, 0, 0, tiles, dout, 0, c.f64, g.s_comp));
     CK(cudaEventRecord(in_free[s], g.s_comp));
     CK(cudaEventRecord(merged[s], g.s_comp));
     CK(cudaStreamWaitEvent(g.s_d2h, merged[s], 0));
@@ -793,8 +971,15 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
             }
           } catch (const HsortError& e) {
             fail(e.code, e.what());
-            cv.notify_all();
+          } catch (const std::exception& e) {
+            fail(HSORT_ERR_INTERNAL, e.what());
+          } catch (...) {
+            fail(HSORT_ERR_INTERNAL, "unknown exception in the downloader");
           }
+          // `failed` is set; take m before notifying so an uploader between its predicate check
+          // and its wait cannot miss the wakeup
+          { std::lock_guard<std::mutex> gd(m); }
+          cv.notify_all();
         });
         uint64_t local = 0;
         try {
@@ -831,6 +1016,10 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
           }
         } catch (const HsortError& e) {
           fail(e.code, e.what());
+        } catch (const std::exception& e) {
+          fail(HSORT_ERR_INTERNAL, e.what());
+        } catch (...) {
+          fail(HSORT_ERR_INTERNAL, "unknown exception in the uploader");
         }
         {
           std::lock_guard<std::mutex> gd(m);
@@ -857,6 +1046,10 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
       }
     } catch (const HsortError& e) {
       fail(e.code, e.what());
+    } catch (const std::exception& e) {
+      fail(HSORT_ERR_INTERNAL, e.what());
+    } catch (...) {
+      fail(HSORT_ERR_INTERNAL, "unknown exception in a GPU worker");
     }
   };
   // PIPEMERGE worker: pair j as soon as batches 2j and 2j+1 are in W, one pair at a time, each
@@ -886,6 +1079,8 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
         }
       } catch (const std::exception& e) {
         fail(HSORT_ERR_INTERNAL, e.what());
+      } catch (...) {
+        fail(HSORT_ERR_INTERNAL, "unknown exception in the PIPEMERGE worker");
       }
     });
   }
@@ -944,18 +1139,34 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
     }
   }
   const uint64_t o_f = std::min<uint64_t>(n, (uint64_t)((double)n * f));
-  double t_cpu = 0, t_gpu = 0;
+  double t_cpu = 0;
+  int cpu_code = 0;
+  std::string cpu_err;
   std::thread cpu_part([&] {
-    auto tc = Clock::now();
-    host_merge_runs_range(run.data(), rlen.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64,
-                          c.merge_threads, nullptr);
-    t_cpu = secs_since(tc);
+    try {
+      auto tc = Clock::now();
+      host_merge_runs_range(run.data(), rlen.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64,
+                            c.merge_threads, nullptr);
+      t_cpu = secs_since(tc);
+    } catch (const std::exception& e) {
+      cpu_code = HSORT_ERR_INTERNAL;
+      cpu_err = e.what();
+    } catch (...) {
+      cpu_code = HSORT_ERR_INTERNAL;
+      cpu_err = "unknown exception in the CPU merge";
+    }
   });
+  // the GPU share [0, o_f) is cut into one range per GPU, each streamed through its own GPU
+  std::vector<double> t_gpu(gs.size(), 0.0);
   std::string gpu_err;
   int gpu_code = 0;
   if (o_f > 0) {
+    const std::vector<uint64_t> gr = shard_bounds(o_f, (int)gs.size(), 1);
     try {
-      gpu_merge_from_host(*gs[0], c, run, rlen, 0, o_f, w_direct, &t_gpu);
+      run_per_gpu(gs.size(), [&](size_t gi) {
+        if (gr[gi + 1] > gr[gi])
+          gpu_merge_from_host(*gs[gi], c, run, rlen, gr[gi], gr[gi + 1], w_direct, &t_gpu[gi]);
+      });
     } catch (const HsortError& e) {
       gpu_code = e.code;
       gpu_err = e.what();
@@ -963,9 +1174,10 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   }
   cpu_part.join();
   if (gpu_code) throw HsortError(gpu_code, gpu_err);
+  if (cpu_code) throw HsortError(cpu_code, cpu_err);
   if (n > o_f + (1u << 20) && t_cpu > 0) S().r_cpu_merge = (double)(n - o_f) / t_cpu;
   c.st->t_merge_cpu = t_cpu;
-  c.st->t_merge_gpu = t_gpu;
+  c.st->t_merge_gpu = *std::max_element(t_gpu.begin(), t_gpu.end());
   c.st->t_merge_phase = secs_since(t1);
   c.st->merge_gpu_fraction = (double)o_f / (double)n;
 }
@@ -976,15 +1188,6 @@ void ctx_create(GpuCtx& g, int dev, const Options& opt) {
   CK(cudaStreamCreateWithFlags(&g.s_h2d, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g.s_comp, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g.s_d2h, cudaStreamNonBlocking));
-  {  // K4's coarse co-rank tables come from cudaMallocAsync: keep freed blocks in the device's
-     // default pool instead of trimming it at every synchronisation
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-      uint64_t keep = ~0ull;
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-    }
-    cudaGetLastError();
-  }
   int R = (int)std::max<int64_t>(2, opt.get("n_ring"));
   g.ring_bytes = (uint64_t)std::max<int64_t>(1 << 20, opt.get("p_s"));
   g.ring_bytes = (g.ring_bytes + 4095) & ~4095ull;
@@ -1020,11 +1223,35 @@ void ctx_destroy(GpuCtx& g) {
   g.min.release();
   g.ranks.release();
   g.off.release();
+  g.coarse.release();
+  g.rptr.release();
   radix_scratch_release(g.rs);
   if (g.s_h2d) cudaStreamDestroy(g.s_h2d);
   if (g.s_comp) cudaStreamDestroy(g.s_comp);
   if (g.s_d2h) cudaStreamDestroy(g.s_d2h);
   g = GpuCtx();
+}
+
+// Usable HBM per GPU context for a call on the first n_gpus contexts: free memory of its device
+// shared by the call's contexts on that device (virtual GPUs, option "virtual_gpus"), plus what
+// the context already holds; the minimum over the contexts.
+uint64_t device_budget(int n_gpus) {
+  uint64_t best = ~0ull;
+  std::map<int, int> per_dev;
+  for (int i = 0; i < n_gpus; ++i) per_dev[S().gpus[i].dev]++;
+  std::map<int, uint64_t> free_of;
+  for (auto& kv : per_dev) {
+    CK(cudaSetDevice(kv.first));
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    free_of[kv.first] = fr;
+  }
+  for (int i = 0; i < n_gpus; ++i) {
+    const GpuCtx& g = S().gpus[i];
+    const uint64_t held = g.runs.cap + g.alt.cap + g.mout.cap + g.ranks.cap + g.min.cap + g.coarse.cap;
+    best = std::min<uint64_t>(best, free_of[g.dev] / per_dev[g.dev] + held);
+  }
+  return best == ~0ull ? 0 : best;
 }
 
 GpuCtx& current_ctx() {
@@ -1081,12 +1308,9 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
   return guarded([&]() -> int {
     auto t0 = Clock::now();
     GpuCtx& g0 = S().gpus[0];
+    const uint64_t budget = device_budget(n_gpus);
     CK(cudaSetDevice(g0.dev));
-    size_t fr = 0, tot = 0;
-    CK(cudaMemGetInfo(&fr, &tot));
-    // budget: free memory plus what this library already holds on the device
-    uint64_t held = g0.runs.cap + g0.alt.cap + g0.mout.cap + g0.ranks.cap;
-    hsort_plan_t plan = make_plan(n, batch_elems, n_gpus, fr + held, S().opt);
+    hsort_plan_t plan = make_plan(n, batch_elems, n_gpus, budget, S().opt, S().peer_ok);
     hsort_stats st{};
     st.n = n;
     st.b_s = plan.b_s;
@@ -1112,7 +1336,9 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
     if (plan.mode == HSORT_MODE_BLINE) {
       sort_bline(g0, c);
     } else if (plan.mode == HSORT_MODE_RESIDENT) {
-      sort_resident(g0, c);
+      std::vector<GpuCtx*> gs;
+      for (int i = 0; i < plan.n_gpus; ++i) gs.push_back(&S().gpus[i]);
+      sort_resident(gs, c);
     } else {
       // in-place (B == A) is safe: W holds the runs, B is written only by the merge
       std::vector<GpuCtx*> gs;
@@ -1356,9 +1582,29 @@ int hsort_init(void) {
       cudaGetLastError();
       throw HsortError(HSORT_ERR_CUDA, std::string("no CUDA device: ") + cudaGetErrorString(e));
     }
-    S().gpus.resize(n);
+    S().n_physical = n;
+    const int nv = (int)S().opt.get("virtual_gpus");
+    const int nctx = nv > 0 ? nv : n;
+    S().gpus.resize(nctx);
     try {
-      for (int d = 0; d < n; ++d) ctx_create(S().gpus[d], d, S().opt);
+      for (int i = 0; i < nctx; ++i) ctx_create(S().gpus[i], i % n, S().opt);
+      // the multi-GPU merge reads the other GPUs' runs by peer loads (NVLink): enable peer access
+      // between every pair of distinct devices
+      S().peer_ok = true;
+      for (int a = 0; a < std::min(n, nctx); ++a)
+        for (int b = 0; b < std::min(n, nctx); ++b) {
+          if (a == b) continue;
+          int can = 0;
+          CK(cudaDeviceCanAccessPeer(&can, a, b));
+          if (!can) {
+            S().peer_ok = false;
+            continue;
+          }
+          CK(cudaSetDevice(a));
+          cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+          if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+          else CK(e);
+        }
     } catch (...) {
       for (auto& g : S().gpus) ctx_destroy(g);
       S().gpus.clear();
@@ -1418,13 +1664,15 @@ int hsort_set_option(const char* key, int64_t value) {
     return HSORT_ERR_INVALID;
   }
   std::string k = key;
+  if (k == "virtual_gpus" && (value < 0 || value > 64))
+    return g_err = "virtual_gpus in [0, 64]", HSORT_ERR_INVALID;
   if ((k == "n_s" || k == "n_ring") && value < 1) return g_err = k + " must be >= 1", HSORT_ERR_INVALID;
   if (k == "p_s" && value < (1 << 20)) return g_err = "p_s must be >= 1 MiB", HSORT_ERR_INVALID;
   if (k == "merge_chunk" && value < kMergeTile) return g_err = "merge_chunk too small", HSORT_ERR_INVALID;
   if (k == "merge_gpu_permille" && (value < -1 || value > 1000)) return g_err = "bad permille", HSORT_ERR_INVALID;
   if (k == "resident" && (value < -1 || value > 1)) return g_err = "resident in {-1,0,1}", HSORT_ERR_INVALID;
   if (k == "pin_w" && (value < -1 || value > 1)) return g_err = "pin_w in {-1,0,1}", HSORT_ERR_INVALID;
-  if (S().inited && (k == "p_s" || k == "n_ring")) {
+  if (S().inited && (k == "p_s" || k == "n_ring" || k == "virtual_gpus")) {
     g_err = k + " must be set before hsort_init";
     return HSORT_ERR_BUSY;
   }
@@ -1619,7 +1867,7 @@ int hsort_device_corank(const uint64_t* d_keys, const uint64_t* h_off, int k, ui
     g.off.reserve((k + 1) * 8);
     cudaStream_t st = (cudaStream_t)stream;
     CK(cudaMemcpyAsync(g.off.p, h_off, (k + 1) * 8, cudaMemcpyHostToDevice, st));
-    CK(merge_corank(d_keys, g.off.u64(), k, h_off[k] - h_off[0], step, 0, n_bounds, d_ranks, st));
+    corank_on(g, d_keys, nullptr, g.off.u64(), k, h_off[k] - h_off[0], step, 0, n_bounds, d_ranks, st);
     CK(cudaStreamSynchronize(st));
     return HSORT_OK;
   });
@@ -1639,8 +1887,9 @@ int hsort_device_merge(const uint64_t* d_keys, const uint64_t* h_off, int k, uin
     CK(cudaMemcpyAsync(g.off.p, h_off, (k + 1) * 8, cudaMemcpyHostToDevice, st));
     const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
     g.ranks.reserve((tiles + 1) * (uint64_t)k * 8);
-    CK(merge_corank(d_keys, g.off.u64(), k, total, kMergeTile, 0, tiles + 1, g.ranks.u64(), st));
-    CK(merge_tiles(d_keys, g.off.u64(), k, total, g.ranks.u64(), 0, 0, tiles, d_out, 0, out_f64 != 0, st));
+    corank_on(g, d_keys, nullptr, g.off.u64(), k, total, kMergeTile, 0, tiles + 1, g.ranks.u64(), st);
+    CK(merge_tiles(d_keys, nullptr, g.off.u64(), k, total, g.ranks.u64(), 0, 0, tiles, d_out, 0,
+                   out_f64 != 0, st));
     CK(cudaStreamSynchronize(st));
     return HSORT_OK;
   });

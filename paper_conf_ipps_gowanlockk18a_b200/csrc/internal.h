@@ -123,17 +123,27 @@ cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, 
 constexpr int kMergeTile = 4096;  // output keys per merge CTA
 constexpr int kMaxMergeRuns = 1024;
 
+// Runs of a merge: run j has len_j = d_off[j + 1] - d_off[j] keys (device offsets) and starts at
+// keys + d_off[j] (runs back to back in one buffer) or, when rp != nullptr, at rp[j] (a device
+// table of run pointers: the runs may live anywhere, including other GPUs' HBM read over
+// NVLink with peer access enabled -- the multi-GPU merge).
+//
 // K4: ranks[b*k + j] for b in [0, n_bounds): co-ranks of o = min((bound_begin + b)*step, total).
-cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                         uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
-                         cudaStream_t st);
+// scratch: merge_corank_scratch_elems(...) uint64 of device scratch for the coarse level of the
+// two-level search (nullptr / too small: single level).
+uint64_t merge_corank_scratch_elems(int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                                    uint64_t n_bounds);
+cudaError_t merge_corank(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                         int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                         uint64_t n_bounds, uint64_t* ranks, uint64_t* scratch,
+                         uint64_t scratch_elems, cudaStream_t st);
 // K5: merge tiles [tile_begin, tile_begin + tile_count) (tile t = output [t*kMergeTile, ...)),
 // given co-ranks of boundaries t = rank_tile0, rank_tile0 + 1, ... (row t - rank_tile0 of
 // `ranks`, step kMergeTile); writes out[o - out_origin].
-cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                        const uint64_t* ranks, uint64_t rank_tile0, uint64_t tile_begin,
-                        uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
-                        cudaStream_t st);
+cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                        int k, uint64_t total, const uint64_t* ranks, uint64_t rank_tile0,
+                        uint64_t tile_begin, uint64_t tile_count, uint64_t* out,
+                        uint64_t out_origin, bool out_f64, cudaStream_t st);
 
 // ---- key codecs (codec.cu, S§8(f) #4) ---------------------------------------------------------
 constexpr int kKeyF64 = 0;

@@ -112,14 +112,17 @@ __device__ __forceinline__ uint64_t upper_bound_fwd(const uint64_t* a, uint64_t 
 // bisection starts at [v_lo, v_hi] with lo/hi found by galloping from the coarse co-ranks.
 template <int C, int G>
 __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ keys,
+                                                const uint64_t* const* __restrict__ rp,
                                                 const uint64_t* __restrict__ off, int k,
                                                 uint64_t total, uint64_t step, uint64_t b0,
                                                 uint64_t nb, uint64_t* __restrict__ ranks,
                                                 const uint64_t* __restrict__ coarse,
                                                 uint64_t coarse_step, uint64_t coarse_b0) {
-  // G lanes per boundary: G = 32, or (k <= 16) the next power of two >= k, so 32 / G boundaries
-  // share a warp on their own lane segments and more dependent-load chains are in flight per SM
-  // a segment holds C chunks of G runs: run j = c G + lane
+  // G lanes per boundary, C runs per lane (run j = c G + lane); 32 / G boundaries share a warp on
+  // their own lane segments, so more dependent-load chains are in flight per SM.  corank_launch
+  // picks (C, G): k <= 16 -> (1, next power of two >= k); 16 < k <= 32 -> (2, 16);
+  // 32 < k <= 64 -> (4, 16); 64 < k <= 128 -> (8, 16); k > 128 -> G = 32, C = 8 / 16 / 32
+  // (k <= 256 / 512 / 1024).
   const int seg = (threadIdx.x & 31) / G;
   const int lane = threadIdx.x & (G - 1);
   const unsigned sm = G == 32 ? 0xffffffffu : ((1u << G) - 1u) << (seg * G);
@@ -127,20 +130,22 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
       (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (uint64_t)(32 / G) + seg;
   if (b >= nb) return;
   const uint64_t o = (b0 + b) * step < total ? (b0 + b) * step : total;
-  uint64_t base[C], lo[C], hi[C];
+  // run j = R[c] (j = c G + lane): back to back in `keys`, or anywhere (rp: a table of run
+  // pointers, possibly into peer GPUs' HBM, read over NVLink)
+  const uint64_t* R[C];
+  uint64_t lo[C], hi[C];
 #pragma unroll
   for (int c = 0; c < C; ++c) {
     int j = c * G + lane;
     if (j < k) {
-      base[c] = off[j] - off[0];
+      R[c] = rp ? rp[j] : keys + off[j];
       lo[c] = 0;
       hi[c] = off[j + 1] - off[j];
     } else {
-      base[c] = 0;
+      R[c] = keys;
       lo[c] = hi[c] = 0;
     }
   }
-  const uint64_t* K = keys + off[0];
   uint64_t* out = ranks + b * (uint64_t)k;
   if (o == total) {
 #pragma unroll
@@ -165,16 +170,16 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
       const int j = c * G + lane;
       rl[c] = j < k ? r0[j] : 0;
       rh[c] = j < k ? r1[j] : 0;
-      if (rl[c] < hi[c]) mn = K[base[c] + rl[c]] < mn ? K[base[c] + rl[c]] : mn;
-      if (rh[c] > 0) mx = K[base[c] + rh[c] - 1] > mx ? K[base[c] + rh[c] - 1] : mx;
+      if (rl[c] < hi[c]) mn = R[c][rl[c]] < mn ? R[c][rl[c]] : mn;
+      if (rh[c] > 0) mx = R[c][rh[c] - 1] > mx ? R[c][rh[c] - 1] : mx;
     }
     L0 = seg_min<G>(sm, mn);  // key at merged position o_lo
     H0 = seg_max<G>(sm, mx);  // key at merged position o_hi - 1
 #pragma unroll
     for (int c = 0; c < C; ++c) {
       const uint64_t len = hi[c];
-      lo[c] = lower_bound_back(K + base[c], rl[c], L0);
-      hi[c] = upper_bound_fwd(K + base[c], rh[c], len, H0);
+      lo[c] = lower_bound_back(R[c], rl[c], L0);
+      hi[c] = upper_bound_fwd(R[c], rh[c], len, H0);
     }
   }
   // Find v = the key at merged position o: smallest v with count(<= v) > o.
@@ -188,7 +193,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
 #pragma unroll
     for (int c = 0; c < C; ++c) {
       if (hi[c] > lo[c]) {
-        uint64_t a = K[base[c] + lo[c]], z = K[base[c] + hi[c] - 1];
+        uint64_t a = R[c][lo[c]], z = R[c][hi[c] - 1];
         mn = a < mn ? a : mn;
         mx = z > mx ? z : mx;
       }
@@ -203,7 +208,7 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
     uint64_t s = 0;
 #pragma unroll
     for (int c = 0; c < C; ++c) {
-      ub[c] = upper_bound(K + base[c], lo[c], hi[c], mid);
+      ub[c] = upper_bound(R[c], lo[c], hi[c], mid);
       s += ub[c];
     }
     // elements <= mid overall: the window searches count from index 0 (lo/hi are absolute)
@@ -229,10 +234,10 @@ __global__ void __launch_bounds__(128) k_corank(const uint64_t* __restrict__ key
     uint64_t l2 = a, h2 = z;
     while (l2 < h2) {  // first index with key >= v
       uint64_t mid = l2 + ((h2 - l2) >> 1);
-      if (K[base[c] + mid] < v) l2 = mid + 1;
+      if (R[c][mid] < v) l2 = mid + 1;
       else h2 = mid;
     }
-    uint64_t u = upper_bound(K + base[c], l2, z, v);
+    uint64_t u = upper_bound(R[c], l2, z, v);
     lo[c] = l2;
     eq[c] = u - l2;
     lt += l2;
@@ -309,7 +314,8 @@ __device__ __forceinline__ int advance_run(const uint32_t* bnd, int a, int cnt, 
 
 template <int T>
 __global__ void __launch_bounds__(T) k_merge_tile(
-    const uint64_t* __restrict__ keys, const uint64_t* __restrict__ off, int k, uint64_t total,
+    const uint64_t* __restrict__ keys, const uint64_t* const* __restrict__ rp,
+    const uint64_t* __restrict__ off, int k, uint64_t total,
     const uint64_t* __restrict__ ranks, uint64_t rank_tile0, uint64_t tile_begin,
     uint64_t* __restrict__ out, uint64_t out_origin, int out_f64) {
   using Cfg = MergeCfg<T>;
@@ -317,7 +323,8 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   extern __shared__ __align__(16) unsigned char smem[];
   uint64_t* buf0 = (uint64_t*)smem;
   uint64_t* buf1 = buf0 + Cfg::BUF;
-  uint64_t* s_src = buf1 + Cfg::BUF;            // [k] absolute start of slice j (minus bnd[j])
+  // [k] address of slice j's first key minus bnd[j] keys (slices may sit in peer GPUs' HBM)
+  const uint64_t** s_src = (const uint64_t**)(buf1 + Cfg::BUF);
   uint32_t* bnd = (uint32_t*)(s_src + k);       // [k + 1] tile-local slice starts
   __shared__ uint32_t s_w[T / 32];
 
@@ -330,16 +337,16 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
 
   // 1. slice table (chunks of T runs, block scan); s_src[j] - bnd[j] is stored, so element p of
-  //    slice j is keys[s_src[j] + p]
+  //    slice j is s_src[j][p]
   uint32_t carry = 0;
   for (int c0 = 0; c0 < k; c0 += T) {
     const int j = c0 + tid;
     uint32_t len = 0;
-    uint64_t srcj = 0;
+    const uint64_t* srcj = nullptr;
     if (j < k) {
       const uint64_t a = r0[j];
       len = (uint32_t)(r1[j] - a);
-      srcj = off[j] + a;
+      srcj = (rp ? rp[j] : keys + off[j]) + a;
     }
     uint32_t x = len;
 #pragma unroll
@@ -389,7 +396,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
       const int e = e0 + 32 * q;
       if (e < L) {
         while (a + 1 < k && bnd[a + 1] <= (uint32_t)e) ++a;
-        v[q] = ld_stream_u64(keys + s_src[a] + e);
+        v[q] = ld_stream_u64(s_src[a] + e);
       }
     }
   }
@@ -509,7 +516,7 @@ __global__ void k_upper_bounds(const uint64_t* __restrict__ keys, uint64_t n,
 constexpr int kMergeThreads = HSORT_MERGE_THREADS;
 
 size_t merge_smem_bytes(int k) {
-  return 2 * MergeCfg<kMergeThreads>::BUF * sizeof(uint64_t) + (size_t)k * sizeof(uint64_t) +
+  return 2 * MergeCfg<kMergeThreads>::BUF * sizeof(uint64_t) + (size_t)k * sizeof(void*) +
          ((size_t)k + 1) * sizeof(uint32_t);
 }
 
@@ -530,13 +537,14 @@ constexpr bool kCorankSeg2 = HSORT_CORANK_SEG2 != 0;
 constexpr bool kCorankIlp = HSORT_CORANK_ILP != 0;
 
 namespace {
-cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                          uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
-                          const uint64_t* coarse, uint64_t cstep, uint64_t cb0, cudaStream_t st) {
+cudaError_t corank_launch(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                          int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                          uint64_t n_bounds, uint64_t* ranks, const uint64_t* coarse,
+                          uint64_t cstep, uint64_t cb0, cudaStream_t st) {
   const int C = (k + 31) / 32;
 #define HS_CORANK_G(CC, GG)                                                                        \
   k_corank<CC, GG><<<(unsigned)((n_bounds * GG + 127) / 128), 128, 0, st>>>(                      \
-      keys, d_off, k, total, step, bound_begin, n_bounds, ranks, coarse, cstep, cb0)
+      keys, rp, d_off, k, total, step, bound_begin, n_bounds, ranks, coarse, cstep, cb0)
 #define HS_CORANK(CC) HS_CORANK_G(CC, 32)
   if (kCorankIlp && k > 32 && k <= 64) HS_CORANK_G(4, 16);
   else if (kCorankIlp && k > 64 && k <= 128) HS_CORANK_G(8, 16);
@@ -549,6 +557,7 @@ cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, ui
   else if (C <= 2) HS_CORANK(2);
   else if (C <= 4) HS_CORANK(4);
   else if (C <= 8) HS_CORANK(8);
+  else if (C <= 16) HS_CORANK(16);
   else HS_CORANK(kMaxC);
 #undef HS_CORANK
 #undef HS_CORANK_G
@@ -563,28 +572,44 @@ cudaError_t corank_launch(const uint64_t* keys, const uint64_t* d_off, int k, ui
 #endif
 constexpr uint64_t kCoarse = HSORT_CORANK_COARSE;
 
-cudaError_t merge_corank(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
-                         uint64_t step, uint64_t bound_begin, uint64_t n_bounds, uint64_t* ranks,
-                         cudaStream_t st) {
-  if (k < 1 || k > kMaxMergeRuns) return cudaErrorInvalidValue;
-  if (n_bounds == 0) return cudaSuccess;
-  if (n_bounds < 4 * kCoarse || k == 1)
-    return corank_launch(keys, d_off, k, total, step, bound_begin, n_bounds, ranks, nullptr, 1, 0, st);
+namespace {
+// coarse rows c0 .. c0 + nc - 1 bracketing every requested bound (0 rows: single level)
+void coarse_rows(uint64_t total, uint64_t step, uint64_t bound_begin, uint64_t n_bounds, int k,
+                 uint64_t* c0, uint64_t* nc) {
+  *c0 = *nc = 0;
+  if (n_bounds < 4 * kCoarse || k == 1) return;
   const uint64_t cstep = step * kCoarse;
   const uint64_t o_first = bound_begin * step < total ? bound_begin * step : total;
   const uint64_t o_last0 = (bound_begin + n_bounds - 1) * step;
   const uint64_t o_last = o_last0 < total ? o_last0 : total;
-  const uint64_t c0 = o_first / cstep;
-  const uint64_t c1 = (o_last + cstep - 1) / cstep;  // coarse rows c0..c1 bracket every bound
-  const uint64_t nc = c1 - c0 + 1;
-  uint64_t* coarse = nullptr;
-  cudaError_t e = cudaMallocAsync((void**)&coarse, nc * (uint64_t)k * sizeof(uint64_t), st);
+  *c0 = o_first / cstep;
+  *nc = (o_last + cstep - 1) / cstep - *c0 + 1;
+}
+}  // namespace
+
+uint64_t merge_corank_scratch_elems(int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                                    uint64_t n_bounds) {
+  uint64_t c0, nc;
+  coarse_rows(total, step, bound_begin, n_bounds, k, &c0, &nc);
+  return nc * (uint64_t)k;
+}
+
+cudaError_t merge_corank(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                         int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                         uint64_t n_bounds, uint64_t* ranks, uint64_t* scratch,
+                         uint64_t scratch_elems, cudaStream_t st) {
+  if (k < 1 || k > kMaxMergeRuns) return cudaErrorInvalidValue;
+  if (n_bounds == 0) return cudaSuccess;
+  uint64_t c0, nc;
+  coarse_rows(total, step, bound_begin, n_bounds, k, &c0, &nc);
+  if (nc == 0 || !scratch || scratch_elems < nc * (uint64_t)k)  // single level
+    return corank_launch(keys, rp, d_off, k, total, step, bound_begin, n_bounds, ranks, nullptr, 1,
+                         0, st);
+  const uint64_t cstep = step * kCoarse;
+  cudaError_t e = corank_launch(keys, rp, d_off, k, total, cstep, c0, nc, scratch, nullptr, 1, 0, st);
   if (e != cudaSuccess) return e;
-  e = corank_launch(keys, d_off, k, total, cstep, c0, nc, coarse, nullptr, 1, 0, st);
-  if (e == cudaSuccess)
-    e = corank_launch(keys, d_off, k, total, step, bound_begin, n_bounds, ranks, coarse, cstep, c0, st);
-  cudaError_t e2 = cudaFreeAsync(coarse, st);
-  return e != cudaSuccess ? e : e2;
+  return corank_launch(keys, rp, d_off, k, total, step, bound_begin, n_bounds, ranks, scratch,
+                       cstep, c0, st);
 }
 
 cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
@@ -594,7 +619,8 @@ cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* value
   return cudaGetLastError();
 }
 
-cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint64_t total,
+cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                        int k, uint64_t total,
                         const uint64_t* ranks, uint64_t rank_tile0, uint64_t tile_begin,
                         uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
                         cudaStream_t st) {
@@ -609,7 +635,7 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* d_off, int k, uint
     if (e != cudaSuccess) return e;
     attr_set[dev] = true;
   }
-  k_merge_tile<kMergeThreads><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, d_off, k, total, ranks,
+  k_merge_tile<kMergeThreads><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, rp, d_off, k, total, ranks,
                                                                   rank_tile0, tile_begin, out,
                                                                   out_origin, out_f64 ? 1 : 0);
   return cudaGetLastError();

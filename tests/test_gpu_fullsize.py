@@ -1,0 +1,52 @@
+"""Full-size parity of the exact calls bench.py times (BASELINE.json configs[1], n = 2^30).
+
+The bench's device arm (hsort_sort_device, default options: dominant-digit elision on, 7 passes)
+and its host->host arm (hsort_sort on pinned A/B, batch_elems = 0: the auto RESIDENT plan with
+2^27-key batches + halving tail and the chunked K4/K5 merge) are compared element by element with
+the oracle (oracle.sort_f64: serial std::sort under IEEE totalOrder, ~2.5 min at 2^30) on the
+bench's own input (uniform U[0,1), seed 2).  Problem statement: P:53-63.
+"""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+N_FULL = 1 << 30
+SEED = 2  # bench.py SEED (rank 0)
+
+
+@pytest.fixture(scope="module")
+def full(oracle_mod, inputs_mod):
+    A = inputs_mod.generate("uniform", N_FULL, seed=SEED)
+    want = oracle_mod.sort_f64(A).view(np.uint64)
+    return A, want
+
+
+def _first_diff(a, b):
+    d = np.flatnonzero(a != b)
+    return None if d.size == 0 else (int(d[0]), int(d.size))
+
+
+def test_fullsize_device_sort_matches_oracle(hs_gpu, full):
+    import torch
+    A, want = full
+    d_in = torch.from_numpy(A).cuda()
+    d_out = torch.empty_like(d_in)
+    hs_gpu.hsort_sort_device(d_in, d_out)
+    torch.cuda.synchronize()
+    plan = hs_gpu.hsort_get_last_plan()
+    got = d_out.cpu().numpy().view(np.uint64)
+    assert _first_diff(got, want) is None
+    assert plan["elided"]  # the bench's 7-pass plan is the one checked
+    del d_in, d_out
+
+
+def test_fullsize_host_sort_auto_plan_matches_oracle(hs_gpu, full):
+    import torch
+    A, want = full
+    At = torch.from_numpy(A).pin_memory()
+    Bt = torch.zeros(N_FULL, dtype=torch.float64).pin_memory()
+    hs_gpu.hsort_sort(At, Bt, batch_elems=0, n_gpus=1)
+    st = hs_gpu.hsort_get_stats()
+    assert st["mode_name"] == "RESIDENT" and st["n_b"] == 12 and st["direct_in"] == 1
+    assert _first_diff(Bt.numpy().view(np.uint64), want) is None

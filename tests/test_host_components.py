@@ -92,6 +92,9 @@ def test_planner_table1_identities(hs):
     rows = [l.split() for l in open(os.path.join(GOLDEN, "table1_identities.txt"))
             if l.strip() and not l.startswith("#")]
     old = hs.hsort_get_option("n_s")
+    # the paper's streamed pipeline (runs through W): the multi-GPU RESIDENT plan would keep the
+    # 2-GPU rows resident instead
+    hs.hsort_set_option("resident", 0)
     try:
         for n, b_s, n_s, n_gpu, n_b, per_stream, gpu_bytes in rows:
             hs.hsort_set_option("n_s", int(n_s))
@@ -106,6 +109,7 @@ def test_planner_table1_identities(hs):
                 assert p["device_bytes_per_gpu"] <= int(gpu_bytes) + int(b_s)
     finally:
         hs.hsort_set_option("n_s", old)
+        hs.hsort_set_option("resident", -1)
 
 
 def test_planner_modes_and_ragged_batches(hs):
@@ -132,13 +136,35 @@ def test_planner_modes_and_ragged_batches(hs):
     p = hs.hsort_plan(3 * 10**10, 0, 1, G)  # auto b_s fills HBM with n_s + 1 buffers
     assert p["mode_name"] == "STREAM" and p["b_s"] % 4096 == 0
     assert p["device_bytes_per_gpu"] <= G
-    p = hs.hsort_plan(10**9, 10**8, 4, G)
-    assert p["mode_name"] == "STREAM" and p["n_gpus"] == 4
+    p = hs.hsort_plan(10**9, 10**8, 4, G)  # multi-GPU RESIDENT: 4 tile-aligned shards of 1e8-key batches
+    assert p["mode_name"] == "RESIDENT" and p["n_gpus"] == 4 and p["n_b"] == 12
     hs.hsort_set_option("resident", 0)
     try:
         assert hs.hsort_plan(10**9, 10**8, 1, G)["mode_name"] == "STREAM"
+        p = hs.hsort_plan(10**9, 10**8, 4, G)
+        assert p["mode_name"] == "STREAM" and p["n_gpus"] == 4 and p["n_b"] == 10
     finally:
         hs.hsort_set_option("resident", -1)
+
+
+@pytest.mark.parametrize("N", [2, 4, 8])
+def test_planner_multi_gpu_resident(hs, N):
+    """A1 for n_gpus = N > 1: whenever N shards fit in N x HBM the plan is the
+    multi-GPU RESIDENT one -- every GPU sorts its shard as resident batches and merges one range of
+    B -- and asking for more GPUs never falls back to one GPU."""
+    G = 180 << 30
+    p = hs.hsort_plan(1 << 30, 0, N, G)
+    assert p["mode_name"] == "RESIDENT" and p["n_gpus"] == N and p["schedule"] == 1
+    assert p["n_b"] % N == 0 and p["n_b"] <= 1024  # equal shards, equal schedules
+    assert abs(p["batches_per_stream"] - p["n_b"] / N) < 1e-9
+    assert p["device_bytes_per_gpu"] < (1 << 30) * 8 // N + (3 << 30)
+    p = hs.hsort_plan(3 * 10**10, 0, N, G)  # 240 GB over N x 180 GB
+    if N >= 2 and 3 * 10**10 * 8 / N < G - (6 << 30):
+        assert p["mode_name"] == "RESIDENT" and p["n_gpus"] == N
+    p = hs.hsort_plan(1 << 20, 0, N, G)  # small: one GPU, one batch
+    assert p["mode_name"] == "BLINE" and p["n_gpus"] == 1
+    p = hs.hsort_plan(10**12, 0, N, G)  # 8 TB: streamed through W on all N GPUs
+    assert p["mode_name"] == "STREAM" and p["n_gpus"] == N and p["b_s"] <= 1 << 30
 
 
 def test_options_validation(hs):

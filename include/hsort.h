@@ -299,6 +299,11 @@ int hsort_host_upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* va
  * Pure arithmetic. */
 uint64_t hsort_pipemerge_count(uint64_t n_b, int n_gpus);
 
+/* Kernels the library has launched since it was loaded (all devices; K1, K2, K3 passes, copies,
+ * the elision's kernels, K4, K5, codecs): the difference across a region counts the region's
+ * launches (bench.py gpu_launches). */
+uint64_t hsort_get_launch_count(void);
+
 /* Number of GPUs visible to the library (0 when none; never an error). */
 int hsort_device_count(void);
 

@@ -101,6 +101,7 @@ SIGNATURES = {
     "hsort_device_upper_bounds": ([_P, _U64, _P, _U64, _P, _P], _I),
     "hsort_get_last_plan": ([ctypes.POINTER(_I), ctypes.POINTER(_I), ctypes.POINTER(_U64)], _I),
     "hsort_host_upper_bounds": ([_P, _U64, _P, _U64, _P], _I),
+    "hsort_get_launch_count": ([], _U64),
 }
 
 
@@ -414,6 +415,11 @@ def hsort_host_upper_bounds(keys: np.ndarray, values: np.ndarray) -> np.ndarray:
     _check(lib().hsort_host_upper_bounds(keys.ctypes.data, keys.size, values.ctypes.data,
                                          values.size, out.ctypes.data))
     return out
+
+
+def hsort_get_launch_count() -> int:
+    """Kernels the library has launched since load (differences count a region's launches)."""
+    return lib().hsort_get_launch_count()
 
 
 def hsort_pipemerge_count(n_b: int, n_gpus: int) -> int:

@@ -50,6 +50,8 @@ void host_merge_runs_range(const uint64_t* const* run, const uint64_t* len, int 
 
 using namespace hsort;
 
+std::atomic<unsigned long long> hsort::g_kernel_launches{0};
+
 namespace {
 
 using Clock = std::chrono::steady_clock;
@@ -118,8 +120,10 @@ struct Options {
       {"dde_min_n", 1ll << 22},      // smallest n the elision is tried at
       {"memcpy_nt", 1},              // PARMEMCPY staging copies with non-temporal stores
       {"auto_pipeline_min", 1ll << 24},  // auto plan: pipelined RESIDENT schedule from this n (0 = off)
-      {"pin_w", -1},                 // STREAM W: 1 cached pinned, 0 pageable, -1 pinned if <= pin_w_max_mb
-      {"pin_w_max_mb", 16384},       // auto pinning limit: pinning runs at ~2.5 GB/s
+      {"pin_w", -1},                 // STREAM W: 1 page-locked, 0 pageable, -1 locked if <= pin_w_max_mb
+      {"pin_w_max_mb", 1ll << 20},   // auto page-locking limit of W (MB)
+      {"w_cache", 1},                // keep W (allocated, prefaulted, locked) across calls
+
       {"virtual_gpus", 0},           // > 0 (set before hsort_init): that many GPU contexts mapped
                                      // round-robin onto the visible devices (multi-GPU scheduler,
                                      // exchange and merge testable on one GPU)
@@ -155,8 +159,9 @@ struct State {
   double t_init = 0;
   // pinned working memory W (STREAM mode), allocated once and reused: pinning is expensive
   // so it is cached like the staging ring
-  void* w_pin = nullptr;
-  size_t w_pin_bytes = 0;
+  void* w_base = nullptr;       // mmap'd, prefaulted; page-locked (cudaHostRegister) if w_pinned
+  size_t w_bytes = 0;
+  bool w_pinned = false;
   double r_cpu_merge = 0;  // last measured CPU merge rate (keys/s), for the A12 split
   bool peer_ok = true;     // every pair of devices in use can read each other's HBM
   int n_physical = 0;      // visible CUDA devices
@@ -206,6 +211,61 @@ bool is_pinned(const void* p, uint64_t bytes) {
     return a.type == cudaMemoryTypeHost;
   };
   return one(p) && one((const char*)p + bytes - 1);
+}
+
+// ---- working memory W (STREAM mode) ------------------------------------------------------------
+// W holds the sorted runs between the sort phase and the merge.  Allocating
+// and pinning host memory is expensive (cudaHostAlloc ran at ~2.3 GB/s on the B200
+// box, profiles/r02a_host_probe.jsonl), so W is allocated once and cached like the staging ring:
+// an anonymous mapping (transparent huge pages), prefaulted by all host threads in parallel,
+// then page-locked with cudaHostRegister (~46 GB/s on prefaulted pages) so the runs are DMA'd
+// straight into W and the GPU merge share streams straight out of it.  t_host_alloc reports the
+// cost in the call that paid it.
+void release_w() {
+  if (!S().w_base) return;
+  if (S().w_pinned) {
+    cudaHostUnregister(S().w_base);
+    cudaGetLastError();
+  }
+  munmap(S().w_base, S().w_bytes);
+  S().w_base = nullptr;
+  S().w_bytes = 0;
+  S().w_pinned = false;
+}
+
+uint64_t* acquire_w(uint64_t bytes, bool* direct, double* t_alloc) {
+  const int64_t pin_w = S().opt.get("pin_w");
+  const bool want_pin = pin_w == 1 ||
+                        (pin_w == -1 && bytes <= ((uint64_t)S().opt.get("pin_w_max_mb") << 20));
+  auto ta = Clock::now();
+  if (S().w_base && S().w_bytes < bytes) release_w();
+  if (!S().w_base) {
+    void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+    if (p == MAP_FAILED) throw HsortError(HSORT_ERR_HOST_OOM, "mmap W failed");
+    madvise(p, bytes, MADV_HUGEPAGE);
+    const uint64_t chunk = 64ull << 20;
+    host_pool().parallel_for((int64_t)((bytes + chunk - 1) / chunk), host_threads(), [&](int64_t i) {
+      volatile char* q = (volatile char*)p + (uint64_t)i * chunk;
+      const uint64_t len = std::min(chunk, bytes - (uint64_t)i * chunk);
+      for (uint64_t o = 0; o < len; o += 4096) q[o] = 0;  // first touch: fault the page in
+    });
+    S().w_base = p;
+    S().w_bytes = bytes;
+    S().w_pinned = false;
+  }
+  if (want_pin && !S().w_pinned) {
+    if (cudaHostRegister(S().w_base, S().w_bytes, cudaHostRegisterDefault) == cudaSuccess)
+      S().w_pinned = true;
+    else
+      cudaGetLastError();  // not lockable (limits): W stays pageable and is staged
+  } else if (!want_pin && S().w_pinned) {
+    cudaHostUnregister(S().w_base);
+    cudaGetLastError();
+    S().w_pinned = false;
+  }
+  *t_alloc += secs_since(ta);
+  *direct = S().w_pinned;
+  return (uint64_t*)S().w_base;
 }
 
 // ---- staging ring (A2/A3, A7/A8) -------------------------------------------------------------
@@ -818,46 +878,13 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   // because the pair merges run one after another.
   const uint64_t spare = m_pipe ? 2 * b_s : 0;
   const uint64_t wn = n + spare;
-  uint64_t* W = nullptr;
   bool w_direct = false;
-  void* w_map = nullptr;
-  const int64_t pin_w = S().opt.get("pin_w");
-  const bool want_pin = pin_w == 1 ||
-      (pin_w == -1 && (wn * 8 <= ((uint64_t)S().opt.get("pin_w_max_mb") << 20) || S().w_pin_bytes >= wn * 8));
-  if (want_pin) {
-    if (S().w_pin_bytes < wn * 8) {
-      if (S().w_pin) cudaFreeHost(S().w_pin);
-      S().w_pin = nullptr;
-      S().w_pin_bytes = 0;
-      auto ta = Clock::now();
-      void* p = nullptr;
-      if (cudaHostAlloc(&p, wn * 8, cudaHostAllocDefault) == cudaSuccess) {
-        S().w_pin = p;
-        S().w_pin_bytes = wn * 8;
-      } else {
-        cudaGetLastError();
-      }
-      c.st->t_host_alloc = secs_since(ta);
+  uint64_t* W = acquire_w(wn * 8, &w_direct, &c.st->t_host_alloc);
+  struct WRelease {
+    ~WRelease() {
+      if (S().opt.get("w_cache") == 0) release_w();
     }
-    if (S().w_pin) {
-      W = (uint64_t*)S().w_pin;
-      w_direct = true;
-    }
-  }
-  if (!W) {
-    void* p = mmap(nullptr, wn * 8, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
-    if (p == MAP_FAILED) throw HsortError(HSORT_ERR_HOST_OOM, "mmap W failed");
-    madvise(p, wn * 8, MADV_HUGEPAGE);
-    W = (uint64_t*)p;
-    w_map = p;
-  }
-  struct WFree {
-    void* p;
-    size_t b;
-    ~WFree() {
-      if (p) munmap(p, b);
-    }
-  } wfree{w_map, wn * 8};
+  } w_release;
   uint64_t* const Wb = W + spare;
 
   std::atomic<uint64_t> next_batch{0};
@@ -1328,6 +1355,30 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
     c.plan = plan;
     c.direct_in = is_pinned(A, bytes);
     c.direct_out = is_pinned(B, bytes);
+    // option register_host: page-lock pageable A / B for this call and DMA them directly
+    // (measured ~46 GB/s to lock + ~58 GB/s to unlock prefaulted memory: slower than staging
+    // through the ring unless the caller reuses its buffers -- off by default)
+    struct HostReg {
+      std::vector<void*> p;
+      ~HostReg() {
+        for (void* q : p) cudaHostUnregister(q);
+        if (!p.empty()) cudaGetLastError();
+      }
+    } hreg;
+    if (S().opt.get("register_host") == 1) {
+      auto ta = Clock::now();
+      auto reg = [&](const void* q, unsigned flags) {
+        if (cudaHostRegister(const_cast<void*>(q), bytes, flags) == cudaSuccess) {
+          hreg.p.push_back(const_cast<void*>(q));
+          return true;
+        }
+        cudaGetLastError();
+        return false;
+      };
+      if (!c.direct_in) c.direct_in = reg(A, A == B ? cudaHostRegisterDefault : cudaHostRegisterReadOnly);
+      if (!c.direct_out) c.direct_out = A == B ? c.direct_in : reg(B, cudaHostRegisterDefault);
+      st.t_host_alloc += secs_since(ta);
+    }
     c.mc_threads = (int)S().opt.get("memcpy_threads");
     c.merge_threads = (int)S().opt.get("merge_threads");
     c.st = &st;
@@ -1625,9 +1676,7 @@ int hsort_init(void) {
 
 int hsort_finalize(void) {
   std::lock_guard<std::mutex> lk(S().m);
-  if (S().w_pin) cudaFreeHost(S().w_pin);
-  S().w_pin = nullptr;
-  S().w_pin_bytes = 0;
+  release_w();
   for (auto& g : S().gpus) ctx_destroy(g);
   S().gpus.clear();
   S().inited = false;
@@ -1953,6 +2002,8 @@ int hsort_host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t
     return HSORT_OK;
   });
 }
+
+uint64_t hsort_get_launch_count(void) { return g_kernel_launches.load(); }
 
 uint64_t hsort_pipemerge_count(uint64_t n_b, int n_gpus) {
   // P:430-454 (reading A-9): one GPU -> floor((n_b-1)/2); two or more -> floor(n_b/(2 n_GPU))

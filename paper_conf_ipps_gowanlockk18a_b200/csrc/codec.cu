@@ -126,7 +126,7 @@ cudaError_t key_encode(const void* in, uint64_t* out, uint64_t n, int key_type, 
     k_encode<1><<<codec_grid(n / 4), 256, 0, st>>>(in, out, n, desc ? 1 : 0);
   else
     return cudaErrorInvalidValue;
-  return cudaGetLastError();
+  return launched();
 }
 
 cudaError_t key_decode(const uint64_t* in, void* out, uint64_t n, int key_type, bool desc,
@@ -139,7 +139,7 @@ cudaError_t key_decode(const uint64_t* in, void* out, uint64_t n, int key_type, 
     k_decode<1><<<codec_grid(n / 4), 256, 0, st>>>(in, out, n, desc ? 1 : 0);
   else
     return cudaErrorInvalidValue;
-  return cudaGetLastError();
+  return launched();
 }
 
 }  // namespace hsort

@@ -2,9 +2,18 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdint>
 
 namespace hsort {
+
+// Kernels launched by the library since load (hsort_get_launch_count): every launch site returns
+// launched(k) in place of cudaGetLastError() after its k launches.
+extern std::atomic<unsigned long long> g_kernel_launches;
+inline cudaError_t launched(unsigned k = 1) {
+  g_kernel_launches.fetch_add(k, std::memory_order_relaxed);
+  return cudaGetLastError();
+}
 
 // ---- radix sort (radix.cu) -----------------------------------------------------------------
 // Device pass plan written by K2 (k_scan_plan) and read by every K3 launch, so the whole sort is

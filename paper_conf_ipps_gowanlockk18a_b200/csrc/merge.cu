@@ -561,7 +561,7 @@ cudaError_t corank_launch(const uint64_t* keys, const uint64_t* const* rp, const
   else HS_CORANK(kMaxC);
 #undef HS_CORANK
 #undef HS_CORANK_G
-  return cudaGetLastError();
+  return launched();
 }
 }  // namespace
 
@@ -616,7 +616,7 @@ cudaError_t upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* value
                          uint64_t* out, cudaStream_t st) {
   if (m == 0) return cudaSuccess;
   k_upper_bounds<<<(unsigned)((m + 255) / 256), 256, 0, st>>>(keys, n, values, m, out);
-  return cudaGetLastError();
+  return launched();
 }
 
 cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
@@ -638,7 +638,7 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const u
   k_merge_tile<kMergeThreads><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, rp, d_off, k, total, ranks,
                                                                   rank_tile0, tile_begin, out,
                                                                   out_origin, out_f64 ? 1 : 0);
-  return cudaGetLastError();
+  return launched();
 }
 
 }  // namespace hsort

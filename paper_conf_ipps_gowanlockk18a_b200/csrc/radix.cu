@@ -79,74 +79,6 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 }
 
 // ------------------------------------------------------------------------------------------
-// K1: digit histograms.  Per-CTA shared histograms [8][256]; each thread keeps, per digit, the
-// last digit value and a run count in registers and only issues a shared atomic when the value
-// changes — constant high digits (e.g. the exponent byte of U[0,1)) cost one atomic per run
-// instead of a 32-way conflict per key.
-constexpr int kHistThreads = 512;
-
-template <bool IN_F64>
-__device__ __forceinline__ void hist_key(uint64_t k, uint32_t (*sh)[kRadix], uint32_t* cd,
-                                         uint32_t* cc) {
-  if (IN_F64) k = to_key(k);
-#pragma unroll
-  for (int p = 0; p < kDigits; ++p) {
-    uint32_t d = (uint32_t)(k >> (8 * p)) & 255u;
-    if (d == cd[p]) {
-      ++cc[p];
-    } else {
-      if (cc[p]) atomicAdd(&sh[p][cd[p]], cc[p]);
-      cd[p] = d;
-      cc[p] = 1;
-    }
-  }
-}
-
-template <bool IN_F64>
-__global__ void __launch_bounds__(kHistThreads) k_hist(const uint64_t* __restrict__ src, uint64_t n,
-                                                      uint64_t* __restrict__ hist) {
-  __shared__ uint32_t sh[kDigits][kRadix];
-  for (int i = threadIdx.x; i < kDigits * kRadix; i += kHistThreads) (&sh[0][0])[i] = 0;
-  __syncthreads();
-  uint32_t cd[kDigits], cc[kDigits];
-#pragma unroll
-  for (int p = 0; p < kDigits; ++p) { cd[p] = 0; cc[p] = 0; }
-
-  // head element if src is not 16-byte aligned
-  uint64_t head = ((uintptr_t)src & 15) ? 1 : 0;
-  if (head > n) head = n;
-  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist_key<IN_F64>(src[0], sh, cd, cc);
-  const uint64_t* base = src + head;
-  const uint64_t m = n - head;
-  const uint64_t pairs = m / 2;
-  const uint64_t stride = (uint64_t)gridDim.x * kHistThreads;
-  uint64_t i = (uint64_t)blockIdx.x * kHistThreads + threadIdx.x;
-  // 4 independent 16-byte loads in flight per thread
-  for (; i + 3 * stride < pairs; i += 4 * stride) {
-    uint64_t a[8];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) ld_stream2(base + 2 * (i + u * stride), a[2 * u], a[2 * u + 1]);
-#pragma unroll
-    for (int u = 0; u < 8; ++u) hist_key<IN_F64>(a[u], sh, cd, cc);
-  }
-  for (; i < pairs; i += stride) {
-    uint64_t a0, a1;
-    ld_stream2(base + 2 * i, a0, a1);
-    hist_key<IN_F64>(a0, sh, cd, cc);
-    hist_key<IN_F64>(a1, sh, cd, cc);
-  }
-  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == kHistThreads - 1)
-    hist_key<IN_F64>(base[m - 1], sh, cd, cc);
-#pragma unroll
-  for (int p = 0; p < kDigits; ++p)
-    if (cc[p]) atomicAdd(&sh[p][cd[p]], cc[p]);
-  __syncthreads();
-  for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
-    uint32_t c = (&sh[0][0])[j];
-    if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
-  }
-}
-
 // ------------------------------------------------------------------------------------------
 // Block-wide exclusive scan of one uint64 per thread over the first 256 threads (8 warps).
 __device__ __forceinline__ uint64_t scan256_excl(uint64_t v, uint64_t* s_warp /*[8]*/,
@@ -910,52 +842,6 @@ __device__ __forceinline__ void hist2_loop(const uint64_t* base, uint64_t pairs,
   }
 }
 
-template <bool IN_F64>
-__global__ void __launch_bounds__(kHistThreads) k_hist2(const uint64_t* __restrict__ src, uint64_t n,
-                                                       uint64_t* __restrict__ hist) {
-  __shared__ uint32_t sh[kDigits * kRadix];
-  for (int i = threadIdx.x; i < kDigits * kRadix; i += kHistThreads) sh[i] = 0;
-  __syncthreads();
-  uint32_t cd[kDigits], cc[kDigits];
-#pragma unroll
-  for (int p = 0; p < kDigits; ++p) { cd[p] = 0; cc[p] = 0; }
-  const uint64_t head = (((uintptr_t)src & 15) && n) ? 1 : 0;
-  const uint64_t* base = src + head;
-  const uint64_t m = n - head;
-  const uint64_t pairs = m / 2;
-  const uint64_t stride = (uint64_t)gridDim.x * kHistThreads;
-  const uint64_t i0 = (uint64_t)blockIdx.x * kHistThreads + threadIdx.x;
-  // entropy probe on this warp's first keys: <= 4 distinct values among 32 lanes -> run cache
-  uint32_t mask = 0;
-  {
-    uint64_t k = i0 < pairs ? base[2 * i0] : (m ? base[0] : 0);
-    if (IN_F64) k = to_key(k);
-    const int lane = threadIdx.x & 31;
-#pragma unroll
-    for (int p = 0; p < kDigits; ++p) {
-      const uint32_t d = (uint32_t)(k >> (8 * p)) & 255u;
-      const uint32_t peers = __match_any_sync(0xffffffffu, d);
-      const uint32_t leaders = __ballot_sync(0xffffffffu, lane == 31 - __clz(peers));
-      if (__popc(leaders) <= 4) mask |= 1u << p;
-    }
-  }
-  if (head && blockIdx.x == 0 && threadIdx.x == 0) hist2_key<IN_F64, 0xFFFFFFFFu>(src[0], sh, cd, cc, 0xFF);
-  if (mask == 0x80u) hist2_loop<IN_F64, 0x80u>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else if (mask == 0u) hist2_loop<IN_F64, 0u>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else if (mask == 0xC0u) hist2_loop<IN_F64, 0xC0u>(base, pairs, i0, stride, sh, cd, cc, mask);
-  else hist2_loop<IN_F64, 0xFFFFFFFFu>(base, pairs, i0, stride, sh, cd, cc, mask);
-  if ((m & 1) && blockIdx.x == gridDim.x - 1 && threadIdx.x == kHistThreads - 1)
-    hist2_key<IN_F64, 0xFFFFFFFFu>(base[m - 1], sh, cd, cc, 0xFF);
-#pragma unroll
-  for (int p = 0; p < kDigits; ++p)
-    if (cc[p]) atomicAdd(&sh[p * kRadix + cd[p]], cc[p]);
-  __syncthreads();
-  for (int j = threadIdx.x; j < kDigits * kRadix; j += kHistThreads) {
-    uint32_t c = sh[j];
-    if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
-  }
-}
-
 // K1 v3: as v2, but the shared histograms are replicated 8 times, interleaved so that counter
 // (p, v) of copy c sits at word 8 (256 p + v) + c; lane L uses copy L & 7.  A warp's 32 atomics
 // then spread over 32 banks by (v & 3, L & 7): only the 4 lanes sharing a copy can conflict (v2:
@@ -1098,26 +984,11 @@ int pass_variant() {
   static int v = env_int("HSORT_PASS_VARIANT", HSORT_DEFAULT_PASS_VARIANT);
   return v;
 }
-int hist_variant() {
-  static int v = env_int("HSORT_HIST_VARIANT", 2);
-  return v;
-}
-
 cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in_f64,
                         uint64_t* hist, cudaStream_t st, DdeState* dde = nullptr) {
   int dev = 0;
   cudaGetDevice(&dev);
-  uint64_t want = (n / 2 + kHistThreads * 8 - 1) / (kHistThreads * 8);
-  static const int ctas = env_int("HSORT_HIST_CTAS", 2);  // CTAs per SM (experiments)
-  uint64_t cap = (uint64_t)num_sms(dev) * ctas;
-  int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-  if (hist_variant() == 0) {
-    if (in_f64) k_hist<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
-    else k_hist<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
-  } else if (hist_variant() == 1) {
-    if (in_f64) k_hist2<true><<<grid, kHistThreads, 0, st>>>(in, n, hist);
-    else k_hist2<false><<<grid, kHistThreads, 0, st>>>(in, n, hist);
-  } else {
+  {
     constexpr int smem = kDigits * kRadix * kHist3Copies * 4;
     auto kt = k_hist3<true, kHist3Threads, kHist3Copies>;
     auto kf = k_hist3<false, kHist3Threads, kHist3Copies>;
@@ -1146,7 +1017,7 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
       else kf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, nullptr);
     }
   }
-  return cudaGetLastError();
+  return launched();
 }
 
 template <int THREADS, int ITEMS, int LBW, int MINB, bool S32>
@@ -1180,7 +1051,7 @@ cudaError_t launch_tma_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t
     kf<<<(unsigned)grid, THREADS, L::bytes, st>>>(in, out, tmp, n, s.plan, s.bin_base, s.lookback,
                                                  s.tile_ctr, ep, p, out_f64 ? 1 : 0,
                                                  s.max_tiles * kRadix, s.lb_rows);
-  return cudaGetLastError();
+  return launched();
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1830,7 +1701,7 @@ cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t*
     kf<<<(unsigned)grid, CT + 32, L::bytes, st>>>(in, out, tmp, vin, vout, vtmp, n, s.plan, s.bin_base,
                                              s.lookback, s.tile_ctr, p, out_f64 ? 1 : 0,
                                              s.max_tiles * kRadix, s.lb_rows, h, ds, sd);
-  return cudaGetLastError();
+  return launched();
 }
 
 // Look-back status format of one sort: 2 = 32-bit words (TMA pass, n <= 2^30: an active digit
@@ -1904,7 +1775,7 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
   else
     k_onesweep<kPassThreads, kPassItems, false><<<(unsigned)tiles, kPassThreads, 0, st>>>(
         in, out, tmp, n, s.plan, s.bin_base, s.lookback, s.tile_ctr, ep, p, out_f64 ? 1 : 0);
-  return cudaGetLastError();
+  return launched();
 }
 
 }  // namespace
@@ -2054,7 +1925,7 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
   k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
                                  out_f64 ? 1 : 0, s.lb_state, cap, dde ? s.dde : nullptr,
                                  desc ? 1 : 0);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = launched()) != cudaSuccess) return e;
   if ((e = mark(2)) != cudaSuccess) return e;
   int dev = 0;
   cudaGetDevice(&dev);
@@ -2075,7 +1946,7 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
         if ((e = mark(3 + p)) != cudaSuccess) return e;
       }
       k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
-      if ((e = cudaGetLastError()) != cudaSuccess) return e;
+      if ((e = launched()) != cudaSuccess) return e;
       // the outliers (internal keys, unordered) -> sorted on their own scratch -> both ends of out
       const uint64_t n_out = P.dde_n_out;
       if ((e = radix_sort_impl(*s.sub, s.side, s.side, s.side + cap, n_out, false, false, st, false)) !=
@@ -2084,7 +1955,7 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
       if (n_out) {
         k_dde_place<<<num_sms(dev), 256, 0, st>>>(s.side, n_out, P.dde_n_less, out, n, out_f64 ? 1 : 0,
                                                   P.key_xor);
-        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        if ((e = launched()) != cudaSuccess) return e;
       }
       return mark(11);
     }
@@ -2095,7 +1966,7 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
     if ((e = mark(3 + p)) != cudaSuccess) return e;
   }
   k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = launched()) != cudaSuccess) return e;
   if ((e = mark(11)) != cudaSuccess) return e;
   return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);
 }
@@ -2136,7 +2007,7 @@ cudaError_t radix_sort_pairs(RadixScratch& s, const uint64_t* in_c, const uint64
   if ((e = select_lb_mode(s, 2, n, st, true)) != cudaSuccess) return e;
   k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f64 ? 1 : 0,
                                  out_f64 ? 1 : 0, s.lb_state);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = launched()) != cudaSuccess) return e;
   if ((e = mark(2)) != cudaSuccess) return e;
   for (int p = 0; p < kDigits; ++p) {
     if ((e = launch_ws_pass<kKvCT, kKvItems, true>(in, out, tmp, vin, vout, vtmp, n, s, p,
@@ -2147,7 +2018,7 @@ cudaError_t radix_sort_pairs(RadixScratch& s, const uint64_t* in_c, const uint64
   int dev = 0;
   cudaGetDevice(&dev);
   k_final_copy<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan, vin, vout, vtmp);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = launched()) != cudaSuccess) return e;
   if ((e = mark(11)) != cudaSuccess) return e;
   return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);
 }
@@ -2170,7 +2041,7 @@ cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, 
   if ((e = select_lb_mode(s, pass_kernel(in, dst, nullptr), n, st)) != cudaSuccess) return e;
   k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, 0, 0, 0, nullptr);
   k_force_plan<<<1, 1, 0, st>>>(s.plan, digit, s.lb_state);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  if ((e = launched(2)) != cudaSuccess) return e;
   return launch_pass(s, in, dst, nullptr, n, 0, false, false, st);
 }
 

@@ -88,6 +88,8 @@ typedef struct hsort_stats {
   double t_pipemerge;      /* host: time spent in those pair-wise merges */
   double t_pipemerge_wait; /* host: wait after the sort phase for the last pair merge (P:422-425
                               wants 0: pair merges must not delay the final multiway merge) */
+  int32_t msd_buckets;     /* MSD-first split (option "msd"): key-range buckets R; 0 = merge path */
+  int32_t reserved0;
 } hsort_stats;
 
 /* Planner output (A1).  Pure host arithmetic; see hsort_plan(). */

@@ -127,6 +127,10 @@ struct Options {
       {"virtual_gpus", 0},           // > 0 (set before hsort_init): that many GPU contexts mapped
                                      // round-robin onto the visible devices (multi-GPU scheduler,
                                      // exchange and merge testable on one GPU)
+      {"msd", 0},                    // 1: RESIDENT plans run the MSD-first split (S§8(f) #2):
+                                     // splitter partition per batch, bucket gather (peer loads),
+                                     // one LSD sort per bucket, no merge
+      {"msd_bucket_keys", 1ll << 24},  // target bucket size (keys) of the MSD-first split
       {"register_host", 0},          // 1: page-lock pageable A/B for the call (cudaHostRegister) and
                                      // DMA them directly instead of staging through the ring
   };
@@ -140,6 +144,8 @@ struct GpuCtx {
   DevBuf runs, alt, mout, min, ranks, off;
   DevBuf coarse;       // K4's coarse-level co-rank table (two-level search)
   DevBuf rptr;         // multi-GPU merge: device table of run pointers (peer HBM)
+  DevBuf part, bcnt, btot, bspl, bseg;  // MSD-first split: partitioned batches, tile counts,
+                                        // batch bucket totals, splitters, gather segment table
   DevBuf vruns, valt;  // key/value sorts: values and their ping-pong scratch
   DevBuf tmp3;         // typed sorts: third key buffer, so the GPUSort runs out of place (elision)
   std::vector<char*> ring_in, ring_out;
@@ -419,8 +425,9 @@ hsort_plan_t make_plan(uint64_t n, uint64_t batch_elems, int n_gpus, uint64_t de
   const uint64_t host_ring = 2ull * (uint64_t)opt.get("n_ring") * (uint64_t)opt.get("p_s");
   // RESIDENT footprint per GPU: its shard's runs + one batch of radix scratch + the merge slots,
   // co-rank rows and coarse table (k runs)
+  const uint64_t msd = opt.get("msd") == 1 ? 1 : 0;  // MSD-first split: + the partitioned copy
   auto resident_bytes = [&](uint64_t shard, uint64_t b, uint64_t k) {
-    return shard * 8 + (uint64_t)(b * (8.0 + kLookbackBytesPerKey)) + merge_buf +
+    return shard * 8 * (1 + msd) + (uint64_t)(b * (8.0 + kLookbackBytesPerKey)) + merge_buf +
            4 * (mchunk / kMergeTile + 2) * std::max<uint64_t>(k, 1) * 8 + k * 16;
   };
   auto set_resident = [&](uint64_t b, int schedule, int N, uint64_t runs, uint64_t bytes) {
@@ -763,6 +770,226 @@ void sort_resident(std::vector<GpuCtx*>& gs, CallCtx& c) {
   });
   c.st->t_merge_phase = secs_since(t1);
   c.st->merge_gpu_fraction = 1.0;
+  for (auto& P : pt) {
+    c.st->t_h2d += P.t_h2d;
+    c.st->t_gpu_sort += P.t_sort;
+    c.st->t_merge_gpu += P.t_merge;
+    c.st->t_d2h += P.t_d2h;
+    c.st->t_stage += P.acc.t_stage;
+    c.st->bytes_h2d += P.acc.h2d;
+    c.st->bytes_d2h += P.acc.d2h;
+    c.st->passes_run = std::max(c.st->passes_run, P.passes);
+  }
+  c.st->passes_skipped = 8 - c.st->passes_run;
+}
+
+// ---- N2: MSD-first split (S§8(f) #2, option "msd") --------------------------------------------
+inline uint64_t host_key(uint64_t u) { return u ^ ((uint64_t)((int64_t)u >> 63) | (1ull << 63)); }
+inline uint64_t mix64(uint64_t x) {
+  x += 0x9E3779B97F4A7C15ull;
+  x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+  x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+  return x ^ (x >> 31);
+}
+
+// R - 1 splitters (key space) at the quantiles of S regularly hashed samples of A: bucket r =
+// (s_{r-1}, s_r].  Only the load balance depends on them, never the result.
+std::vector<uint64_t> sample_splitters(const void* A, uint64_t n, bool f64, int R) {
+  const uint64_t S = std::min<uint64_t>(n, std::max<uint64_t>(64ull * R, 1ull << 16));
+  std::vector<uint64_t> smp(S);
+  const uint64_t* a = (const uint64_t*)A;
+  for (uint64_t i = 0; i < S; ++i) {
+    const uint64_t u = a[mix64(i) % n];
+    smp[i] = f64 ? host_key(u) : u;
+  }
+  std::sort(smp.begin(), smp.end());
+  std::vector<uint64_t> spl(std::max(R - 1, 0));
+  for (int r = 0; r + 1 < R; ++r) spl[r] = smp[(uint64_t)(r + 1) * S / R - 1];
+  return spl;
+}
+
+// The MSD-first split over N >= 1 GPUs (replaces the merge of sort_resident):
+//  1. GPU g uploads its shard of A batch by batch; each batch is partitioned into R buckets by
+//     the sampled splitters (K6a-c) while the next one uploads;
+//  2. the host sums the bucket sizes, gives every GPU a contiguous run of buckets (~n/N keys) and
+//     places bucket r at B[sum_{r' < r} T_r'];
+//  3. GPU g gathers its buckets' segments from every GPU's partitioned batches (K6d: peer loads
+//     over NVLink = the exchange), LSD-sorts each bucket in place (inverse transform fused into the
+//     last pass; high digits constant inside a bucket are skipped by K2) and DMAs it to B while
+//     the next bucket sorts.
+void sort_msd(std::vector<GpuCtx*>& gs, CallCtx& c) {
+  const size_t N = gs.size();
+  const uint64_t n = c.n;
+  const std::vector<uint64_t> shard = shard_bounds(n, (int)N, kRadixTile);
+  std::vector<std::vector<uint64_t>> h_off(N);
+  for (size_t g = 0; g < N; ++g) h_off[g] = batch_offsets(shard[g + 1] - shard[g], c.plan.b_s, c.plan.schedule);
+  const uint64_t bk = (uint64_t)std::max<int64_t>(1 << 16, S().opt.get("msd_bucket_keys"));
+  int R = (int)std::min<uint64_t>(kMaxBuckets, std::max<uint64_t>(4 * N, n / bk));
+  R -= R % (int)N;
+  std::vector<uint64_t> spl;
+  std::mutex spl_m;
+  std::condition_variable spl_cv;
+  bool spl_ready = false;
+  std::thread sampler([&] {
+    std::vector<uint64_t> v = sample_splitters(c.A, n, c.f64, R);
+    {
+      std::lock_guard<std::mutex> lk(spl_m);
+      spl = std::move(v);
+      spl_ready = true;
+    }
+    spl_cv.notify_all();
+  });
+  struct SamplerJoin {
+    std::thread& t;
+    ~SamplerJoin() {
+      if (t.joinable()) t.join();
+    }
+  } sj{sampler};
+  std::vector<std::vector<uint32_t>> tot(N);  // [batch][R] bucket sizes per GPU
+  std::vector<PhaseTimes> pt(N);
+  auto t0 = Clock::now();
+  run_per_gpu(N, [&](size_t gi) {
+    GpuCtx& g = *gs[gi];
+    CK(cudaSetDevice(g.dev));
+    const std::vector<uint64_t>& off = h_off[gi];
+    const uint64_t nb = off.size() - 1, sh = off[nb];
+    if (sh == 0) return;
+    uint64_t bmax = 0;
+    for (uint64_t i = 0; i < nb; ++i) bmax = std::max(bmax, off[i + 1] - off[i]);
+    g.runs.reserve(sh * 8);
+    g.part.reserve(sh * 8);
+    g.bcnt.reserve(bucket_count_elems(bmax, R) * 4);
+    g.btot.reserve(nb * R * 4);
+    g.bspl.reserve(R * 8);
+    std::vector<EvPair> eh(nb), es(nb);
+    for (auto& e : eh) e.make();
+    for (auto& e : es) e.make();
+    for (uint64_t i = 0; i < nb; ++i) {
+      const uint64_t o = off[i], len = off[i + 1] - off[i];
+      CK(cudaEventRecord(eh[i].a, g.s_h2d));
+      upload(g, g.runs.u64() + o, (const char*)c.A + (shard[gi] + o) * 8, len * 8, g.s_h2d,
+             c.direct_in, c.mc_threads, pt[gi].acc);
+      CK(cudaEventRecord(eh[i].b, g.s_h2d));
+      if (i == 0) {  // the splitters are sampled while the first batch uploads
+        std::unique_lock<std::mutex> lk(spl_m);
+        spl_cv.wait(lk, [&] { return spl_ready; });
+        if (R > 1)
+          CK(cudaMemcpyAsync(g.bspl.p, spl.data(), (R - 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
+      }
+      CK(cudaStreamWaitEvent(g.s_comp, eh[i].b, 0));
+      CK(cudaEventRecord(es[i].a, g.s_comp));
+      CK(bucket_partition(g.runs.u64() + o, len, c.f64, g.bspl.u64(), R, (uint32_t*)g.bcnt.p,
+                          (uint32_t*)g.btot.p + i * R, g.part.u64() + o, g.s_comp));
+      CK(cudaEventRecord(es[i].b, g.s_comp));
+    }
+    tot[gi].resize(nb * R);
+    CK(cudaMemcpyAsync(tot[gi].data(), g.btot.p, nb * R * 4, cudaMemcpyDeviceToHost, g.s_comp));
+    CK(cudaStreamSynchronize(g.s_comp));
+    for (uint64_t i = 0; i < nb; ++i) {
+      pt[gi].t_h2d += eh[i].ms() / 1e3;
+      pt[gi].t_sort += es[i].ms() / 1e3;
+    }
+    for (auto& e : eh) e.destroy();
+    for (auto& e : es) e.destroy();
+  });
+  c.st->t_sort_phase = secs_since(t0);
+  // bucket sizes, owners (contiguous bucket runs of ~n/N keys), places in B and in the owner's
+  // receive buffer (bucket starts kept 16-byte aligned for the TMA passes)
+  std::vector<uint64_t> T(R, 0), G(R + 1, 0);
+  for (size_t h = 0; h < N; ++h)
+    for (size_t i = 0; i < tot[h].size(); ++i) T[i % R] += tot[h][i];
+  for (int r = 0; r < R; ++r) G[r + 1] = G[r] + T[r];
+  if (G[R] != n) throw HsortError(HSORT_ERR_INTERNAL, "bucket sizes do not add up to n");
+  std::vector<int> first(N + 1, R);
+  first[0] = 0;
+  {
+    size_t g = 1;
+    for (int r = 0; r < R && g < N; ++r)
+      while (g < N && G[r + 1] > (uint64_t)((unsigned __int128)n * g / N)) first[g++] = r + 1;
+    for (; g < N; ++g) first[g] = R;
+    for (size_t q = 1; q < N; ++q) first[q] = std::max(first[q], first[q - 1]);
+  }
+  auto t1 = Clock::now();
+  run_per_gpu(N, [&](size_t gi) {
+    GpuCtx& g = *gs[gi];
+    CK(cudaSetDevice(g.dev));
+    const int r0 = first[gi], r1 = first[gi + 1];
+    if (r1 <= r0) return;
+    std::vector<GatherSeg> segs;
+    std::vector<uint64_t> pstart{0}, roff(r1 - r0 + 1, 0);
+    uint64_t cap = 0, tmax = 0;
+    for (int r = r0; r < r1; ++r) {
+      roff[r - r0] = cap;
+      for (size_t h = 0; h < N; ++h) {
+        const uint64_t nb = h_off[h].size() - 1;
+        for (uint64_t i = 0; i < nb; ++i) {
+          const uint32_t* tb = &tot[h][i * R];
+          const uint64_t len = tb[r];
+          if (!len) continue;
+          uint64_t bb = 0;  // start of bucket r inside batch i of GPU h
+          for (int q = 0; q < r; ++q) bb += tb[q];
+          segs.push_back({gs[h]->part.u64() + h_off[h][i] + bb, len, cap});
+          cap += len;
+          pstart.push_back(pstart.back() + gather_pieces(len));
+        }
+      }
+      tmax = std::max(tmax, T[r]);
+      cap += cap & 1;  // next bucket 16-byte aligned
+    }
+    roff[r1 - r0] = cap;
+    if (segs.empty()) return;
+    pstart.pop_back();
+    const uint64_t pieces = pstart.back() + gather_pieces(segs.back().len);
+    g.runs.reserve(std::max<uint64_t>(cap, 2) * 8);  // this GPU's raw batches are partitioned: free
+    g.alt.reserve(std::max<uint64_t>(tmax, 2) * 8);
+    const size_t tb_bytes = segs.size() * sizeof(GatherSeg);
+    g.bseg.reserve(tb_bytes + pstart.size() * 8);
+    CK(cudaMemcpyAsync(g.bseg.p, segs.data(), tb_bytes, cudaMemcpyHostToDevice, g.s_comp));
+    CK(cudaMemcpyAsync((char*)g.bseg.p + tb_bytes, pstart.data(), pstart.size() * 8,
+                       cudaMemcpyHostToDevice, g.s_comp));
+    EvPair eg;
+    eg.make();
+    CK(cudaEventRecord(eg.a, g.s_comp));
+    CK(gather_segments((const GatherSeg*)g.bseg.p, (const uint64_t*)((char*)g.bseg.p + tb_bytes),
+                       (int)segs.size(), pieces, g.runs.u64(), g.s_comp));
+    CK(cudaEventRecord(eg.b, g.s_comp));
+    const int nr = r1 - r0;
+    std::vector<EvPair> es(nr), ed(nr);
+    for (int q = 0; q < nr; ++q) {
+      es[q].make();
+      ed[q].make();
+    }
+    // every bucket's sort is enqueued first (one compute stream), then the DtoH of bucket q waits
+    // for its sort only, so sorts and DtoH overlap
+    for (int q = 0; q < nr; ++q) {
+      CK(cudaEventRecord(es[q].a, g.s_comp));
+      if (T[r0 + q])
+        CK(radix_sort(g.rs, g.runs.u64() + roff[q], g.runs.u64() + roff[q], g.alt.u64(), T[r0 + q],
+                      false, c.f64, g.s_comp));
+      CK(cudaEventRecord(es[q].b, g.s_comp));
+    }
+    for (int q = 0; q < nr; ++q) {
+      CK(cudaStreamWaitEvent(g.s_d2h, es[q].b, 0));
+      CK(cudaEventRecord(ed[q].a, g.s_d2h));
+      download(g, (char*)c.B + G[r0 + q] * 8, g.runs.u64() + roff[q], T[r0 + q] * 8, g.s_d2h,
+               c.direct_out, c.mc_threads, pt[gi].acc);
+      CK(cudaEventRecord(ed[q].b, g.s_d2h));
+    }
+    CK(cudaStreamSynchronize(g.s_d2h));
+    CK(cudaStreamSynchronize(g.s_comp));
+    pt[gi].t_merge += eg.ms() / 1e3;  // the exchange (gather) takes the merge's place
+    for (int q = 0; q < nr; ++q) {
+      pt[gi].t_sort += es[q].ms() / 1e3;
+      pt[gi].t_d2h += ed[q].ms() / 1e3;
+      es[q].destroy();
+      ed[q].destroy();
+    }
+    eg.destroy();
+    pt[gi].passes = g.rs.h_plan->num_active;
+  });
+  c.st->t_merge_phase = secs_since(t1);
+  c.st->merge_gpu_fraction = 1.0;
+  c.st->msd_buckets = R;
   for (auto& P : pt) {
     c.st->t_h2d += P.t_h2d;
     c.st->t_gpu_sort += P.t_sort;
@@ -1252,6 +1479,11 @@ void ctx_destroy(GpuCtx& g) {
   g.off.release();
   g.coarse.release();
   g.rptr.release();
+  g.part.release();
+  g.bcnt.release();
+  g.btot.release();
+  g.bspl.release();
+  g.bseg.release();
   radix_scratch_release(g.rs);
   if (g.s_h2d) cudaStreamDestroy(g.s_h2d);
   if (g.s_comp) cudaStreamDestroy(g.s_comp);
@@ -1389,7 +1621,8 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
     } else if (plan.mode == HSORT_MODE_RESIDENT) {
       std::vector<GpuCtx*> gs;
       for (int i = 0; i < plan.n_gpus; ++i) gs.push_back(&S().gpus[i]);
-      sort_resident(gs, c);
+      if (S().opt.get("msd") == 1) sort_msd(gs, c);
+      else sort_resident(gs, c);
     } else {
       // in-place (B == A) is safe: W holds the runs, B is written only by the merge
       std::vector<GpuCtx*> gs;

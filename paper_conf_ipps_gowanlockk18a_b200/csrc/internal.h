@@ -154,6 +154,27 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const u
                         uint64_t tile_begin, uint64_t tile_count, uint64_t* out,
                         uint64_t out_origin, bool out_f64, cudaStream_t st);
 
+// ---- MSD-first split (msd.cu, S§8(f) #2) ---------------------------------------------------------
+constexpr int kMaxBuckets = 1024;
+// bucket r of a key k = #{splitters < k} (R - 1 sorted splitters): bucket r = (s_{r-1}, s_r].
+// counts: bucket_count_elems(n, R) uint32 of scratch; totals[R] receives the batch's bucket sizes;
+// out (n keys, transformed if in_f64) holds the batch in bucket order (bucket r at
+// sum_{r' < r} totals[r']).  Stream-ordered.
+uint64_t bucket_count_elems(uint64_t n, int R);
+cudaError_t bucket_partition(const uint64_t* in, uint64_t n, bool in_f64, const uint64_t* d_spl,
+                             int R, uint32_t* counts, uint32_t* totals, uint64_t* out,
+                             cudaStream_t st);
+// dst[seg.dst_off + i] = seg.src[i] for every segment (sources anywhere, incl. peer HBM).
+struct GatherSeg {
+  const uint64_t* src;
+  uint64_t len;
+  uint64_t dst_off;
+};
+uint64_t gather_pieces(uint64_t len);  // CTAs one segment of len keys needs
+// d_piece_start[s] = sum_{s' < s} gather_pieces(len_s'); pieces = the total
+cudaError_t gather_segments(const GatherSeg* d_segs, const uint64_t* d_piece_start, int nseg,
+                            uint64_t pieces, uint64_t* dst, cudaStream_t st);
+
 // ---- key codecs (codec.cu, S§8(f) #4) ---------------------------------------------------------
 constexpr int kKeyF64 = 0;
 constexpr int kKeyF32 = 1;

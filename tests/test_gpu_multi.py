@@ -50,7 +50,7 @@ def _with(hs, opts, fn):
             hs.hsort_set_option(k, v)
 
 
-def _runs_expected(n, N, b, schedule_auto=False):
+def _runs_expected(n, N, b):
     """Run count of the multi-GPU RESIDENT plan: tile-aligned shards, uniform b-key batches."""
     sh = [0] + [(n * g // N) - (n * g // N) % 4096 for g in range(1, N)] + [n]
     for g in range(1, N):
@@ -156,3 +156,46 @@ def test_multi_device_entry_points_still_work(hv, oracle_mod, inputs_mod):
     hv.hsort_sort_device(d, o)
     torch.cuda.synchronize()
     assert np.array_equal(_bits(o.cpu().numpy()), _bits(oracle_mod.sort_f64(A)))
+
+
+# ---- N2: MSD-first split (option "msd", S§8(f) #2) ------------------------------------------------
+MSD_DISTS = ["uniform", "zipf_dup", "special", "all_equal", "normal", "sorted", "few_distinct"]
+
+
+@pytest.mark.parametrize("N", [1, 2, 3, 4])
+@pytest.mark.parametrize("dist", MSD_DISTS)
+def test_msd_split_matches_oracle(hv, oracle_mod, inputs_mod, N, dist):
+    """Sampled splitters -> per-batch bucket partition (K6a-c) -> bucket gather from every GPU
+    (K6d, peer loads) -> one LSD sort per bucket -> DtoH to B[sum of earlier buckets].  No merge.
+    Heavy duplicates / all-equal keys put whole equal-key groups in one bucket."""
+    n = 2_000_003
+    A = inputs_mod.generate(dist, n, seed=N * 100 + len(dist))
+    want = _bits(oracle_mod.sort_f64(A))
+    opts = {"msd": 1, "msd_bucket_keys": 1 << 16, "auto_pipeline_min": 1 << 20}
+    B = _with(hv, opts, lambda: hv.hsort_sort(A, batch_elems=0, n_gpus=N))
+    st = hv.hsort_get_stats()
+    assert st["mode_name"] == "RESIDENT" and st["n_gpus"] == N and st["msd_buckets"] >= 4 * N
+    assert np.array_equal(_bits(B), want), (N, dist)
+
+
+@pytest.mark.parametrize("N", [1, 3])
+def test_msd_split_pinned_explicit_batches_u64(hv, oracle_mod, inputs_mod, N):
+    A = inputs_mod.generate("salted", 1_500_001, seed=N)
+    want = _bits(oracle_mod.sort_f64(A))
+    opts = {"msd": 1, "msd_bucket_keys": 1 << 17}
+    At, Bt = _pinned(A.copy()), _pinned(np.zeros_like(A))
+    _with(hv, opts, lambda: hv.hsort_sort(At, Bt, batch_elems=200_000, n_gpus=N))
+    st = hv.hsort_get_stats()
+    assert st["msd_buckets"] > 0 and st["direct_in"] == 1 and st["direct_out"] == 1
+    assert np.array_equal(_bits(Bt.numpy()), want)
+    K = np.random.default_rng(N).integers(0, 2**64, size=700_001, dtype=np.uint64)
+    got = _with(hv, opts, lambda: hv.hsort_sort_u64(K, batch_elems=100_000, n_gpus=N))
+    assert np.array_equal(got, oracle_mod.sort_u64(K))
+
+
+@pytest.mark.parametrize("n,b", [(5000, 1000), (12_289, 4096), (70_001, 8192)])
+def test_msd_split_tiny(hv, oracle_mod, inputs_mod, n, b):
+    A = inputs_mod.generate("special", n, seed=n)
+    want = _bits(oracle_mod.sort_f64(A))
+    B = _with(hv, {"msd": 1}, lambda: hv.hsort_sort(A, batch_elems=b, n_gpus=4))
+    assert np.array_equal(_bits(B), want)

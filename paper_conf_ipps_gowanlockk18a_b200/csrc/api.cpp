@@ -13,6 +13,7 @@
 // all runs fit in HBM they stay resident and are merged by the GPU (merge.cu) with the merged
 // chunks' DtoH overlapped with the merge.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: no-ops unless a profiler attaches
 #include <sys/mman.h>
 
 #include <algorithm>
@@ -60,6 +61,15 @@ inline double secs_since(Clock::time_point t0) {
 }
 
 thread_local std::string g_err = "";
+
+// NVTX range over a scope (the Fig. 2-style overlap timeline of Stage / HtoD / GPUSort /
+// DtoH / Merge under nsys or ncu --nvtx)
+struct Nvtx {
+  explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+  ~Nvtx() { nvtxRangePop(); }
+  Nvtx(const Nvtx&) = delete;
+  Nvtx& operator=(const Nvtx&) = delete;
+};
 
 struct HsortError : std::runtime_error {
   int code;
@@ -240,6 +250,7 @@ void release_w() {
 }
 
 uint64_t* acquire_w(uint64_t bytes, bool* direct, double* t_alloc) {
+  Nvtx nv("W alloc");
   const int64_t pin_w = S().opt.get("pin_w");
   const bool want_pin = pin_w == 1 ||
                         (pin_w == -1 && bytes <= ((uint64_t)S().opt.get("pin_w_max_mb") << 20));
@@ -283,6 +294,7 @@ struct Acc {  // per-thread stage accumulators
 // Host -> device, through the pinned ring (PIPEDATA Stage + PARMEMCPY) unless direct.
 void upload(GpuCtx& g, void* d_dst, const void* h_src, uint64_t bytes, cudaStream_t st, bool direct,
             int threads, Acc& acc) {
+  Nvtx r(direct ? "HtoD" : "Stage+HtoD");
   acc.h2d += bytes;
   if (bytes == 0) return;
   if (direct) {
@@ -306,6 +318,7 @@ void upload(GpuCtx& g, void* d_dst, const void* h_src, uint64_t bytes, cudaStrea
 // byte is in h_dst (DMA of chunk c overlaps the host copy-out of chunk c-1).
 void download(GpuCtx& g, void* h_dst, const void* d_src, uint64_t bytes, cudaStream_t st,
               bool direct, int threads, Acc& acc) {
+  Nvtx r(direct ? "DtoH" : "DtoH+Stage");
   acc.d2h += bytes;
   if (bytes == 0) return;
   if (direct) {
@@ -626,6 +639,7 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_keys, const uint
                        const uint64_t* d_off, int k, uint64_t total, uint64_t o_lo, uint64_t o_hi,
                        PhaseTimes& pt) {
   if (o_hi <= o_lo) return;
+  Nvtx nv("GPU merge -> B");
   const uint64_t t_lo = o_lo / kMergeTile;
   const uint64_t t_hi = (o_hi + kMergeTile - 1) / kMergeTile;
   const uint64_t tiles = t_hi - t_lo;
@@ -693,6 +707,7 @@ void resident_sort_phase(GpuCtx& g, CallCtx& c, uint64_t a0, const std::vector<u
   CK(cudaSetDevice(g.dev));
   const uint64_t nb = h_off.size() - 1, shard = h_off[nb];
   if (shard == 0) return;
+  Nvtx nv("sort phase (resident)");
   uint64_t bmax = 0;
   for (uint64_t i = 0; i < nb; ++i) bmax = std::max(bmax, h_off[i + 1] - h_off[i]);
   g.runs.reserve(shard * 8);
@@ -1010,6 +1025,7 @@ void sort_msd(std::vector<GpuCtx*>& gs, CallCtx& c) {
 void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t*>& run,
                          const std::vector<uint64_t>& rlen, uint64_t o_lo, uint64_t o_hi,
                          bool w_direct, double* t_gpu) {
+  Nvtx nv("GPU merge share W -> B");
   CK(cudaSetDevice(g.dev));
   const int k = (int)run.size();
   const uint64_t C = std::max<uint64_t>(
@@ -1398,6 +1414,7 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
   std::string cpu_err;
   std::thread cpu_part([&] {
     try {
+      Nvtx nv("CPU merge W -> B");
       auto tc = Clock::now();
       host_merge_runs_range(run.data(), rlen.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64,
                             c.merge_threads, nullptr);
@@ -1565,6 +1582,7 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
   }
   if (n_gpus == 0) n_gpus = vis;
   return guarded([&]() -> int {
+    Nvtx nv("hsort_sort");
     auto t0 = Clock::now();
     GpuCtx& g0 = S().gpus[0];
     const uint64_t budget = device_budget(n_gpus);

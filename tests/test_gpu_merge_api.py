@@ -20,8 +20,8 @@ def _runs(rng, k, maxlen, hi=2**64):
     return runs, np.concatenate(runs), off
 
 
-@pytest.mark.parametrize("k", [1, 2, 3, 8, 33, 100, 300])
-@pytest.mark.parametrize("hi", [2**64, 50])
+@pytest.mark.parametrize("k", [1, 2, 3, 8, 17, 24, 32, 33, 64, 100, 128, 300, 600])
+@pytest.mark.parametrize("hi", [2**64, 50, 7])
 def test_corank_matches_oracle(hs_gpu, oracle_mod, k, hi):
     import torch
     rng = np.random.default_rng(k + hi % 1000)
@@ -38,7 +38,7 @@ def test_corank_matches_oracle(hs_gpu, oracle_mod, k, hi):
         assert np.array_equal(got[b], oracle_mod.corank(runs, o)), (b, o)
 
 
-@pytest.mark.parametrize("k", [2, 5, 33, 200])
+@pytest.mark.parametrize("k", [2, 5, 17, 24, 32, 33, 64, 128, 200])
 @pytest.mark.parametrize("hi", [2**64, 7, 3000])
 def test_corank_two_level_matches_oracle(hs_gpu, oracle_mod, k, hi):
     """>= 64 bounds: coarse co-ranks every 16 steps, fine ones from the coarse windows (ties at

@@ -5,5 +5,5 @@ name=$1
 d=paper_conf_ipps_gowanlockk18a_b200
 mkdir -p $d/ab $d/build/ab
 nvcc -O3 -lineinfo -std=c++17 $EXTRA -gencode arch=compute_100a,code=sm_100a -Xcompiler -fPIC -c $d/csrc/radix.cu -o $d/build/ab/radix_$name.o
-nvcc -shared -gencode arch=compute_100a,code=sm_100a -cudart static -o $d/ab/$name.so $d/build/ab/radix_$name.o $d/build/merge.o $d/build/codec.o $d/build/api.o $d/build/pool.o $d/build/host_merge.o -lpthread
+nvcc -shared -gencode arch=compute_100a,code=sm_100a -cudart static -o $d/ab/$name.so $d/build/ab/radix_$name.o $d/build/merge.o $d/build/codec.o $d/build/msd.o $d/build/api.o $d/build/pool.o $d/build/host_merge.o -lpthread
 echo built $d/ab/$name.so

@@ -531,6 +531,8 @@ def main():
                     help="only the timed host->host and device steps (profiling runs)")
     ap.add_argument("--device-only", action="store_true",
                     help="profiling: skip the host->host arm (ncu captures of the device GPUSort)")
+    ap.add_argument("--no-dde", action="store_true",
+                    help="profiling: dominant-digit elision off (every device pass is a full pass)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -577,6 +579,8 @@ def main():
         n_gpu //= 2
     n = N * n_gpu
     hs.hsort_set_option("kernel_timing", 1)
+    if args.no_dde:
+        hs.hsort_set_option("dde", 0)
     t0 = time.perf_counter()
     hs.hsort_init()
     t_init = time.perf_counter() - t0

@@ -90,6 +90,7 @@ typedef struct hsort_stats {
                               wants 0: pair merges must not delay the final multiway merge) */
   int32_t msd_buckets;     /* MSD-first split (option "msd"): key-range buckets R; 0 = merge path */
   int32_t reserved0;
+  double t_setup;          /* host: planning before the first copy (HBM query, plan, pointer checks) */
 } hsort_stats;
 
 /* Planner output (A1).  Pure host arithmetic; see hsort_plan(). */

@@ -57,7 +57,7 @@ class hsort_stats(ctypes.Structure):
         ("t_init", ctypes.c_double),
         ("bytes_h2d", _U64), ("bytes_d2h", _U64), ("t_host_alloc", ctypes.c_double),
         ("pipe_merges", _U64), ("t_pipemerge", ctypes.c_double), ("t_pipemerge_wait", ctypes.c_double),
-        ("msd_buckets", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+        ("msd_buckets", ctypes.c_int32), ("reserved0", ctypes.c_int32), ("t_setup", ctypes.c_double),
     ]
 
 

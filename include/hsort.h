@@ -42,7 +42,8 @@ typedef enum {
   HSORT_ERR_HOST_OOM = -3,         /* host allocation (W, pinned ring) failed */
   HSORT_ERR_DEVICE_OOM = -4,       /* device allocation failed */
   HSORT_ERR_CUDA = -5,             /* CUDA runtime error (library poisoned until finalize) */
-  HSORT_ERR_NCCL = -6,             /* reserved: NCCL exchange (multi-GPU resident mode) */
+  HSORT_ERR_NCCL = -6,             /* reserved, never returned: the in-library multi-GPU exchange
+                                      uses peer loads over NVLink, not NCCL */
   HSORT_ERR_BUSY = -7,             /* concurrent call, or hsort_init twice */
   HSORT_ERR_INTERNAL = -8          /* invariant violated inside the library */
 } hsort_status;
@@ -296,6 +297,15 @@ int hsort_host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t
 /* Host version of hsort_device_upper_bounds (keys, values, out in host memory). */
 int hsort_host_upper_bounds(const uint64_t* keys, uint64_t n, const uint64_t* values, uint64_t m,
                             uint64_t* out);
+
+/* Splitter arithmetic of the multi-process exchange (A13, paper_conf_ipps_gowanlockk18a_b200/dist.py;
+ * one process per GPU, torch.distributed moves the data).  hsort_sample_positions: the s regular
+ * sample positions of a sorted run of n >= 1 keys, pos[i] = min(n - 1, (i + 1) n / (s + 1)).
+ * hsort_select_splitters: from the m merged (sorted) samples of all ranks, the P - 1 splitters
+ * spl[r - 1] = samples[r m / P] (r = 1..P-1; all 0 when m = 0); rank r then owns the keys k with
+ * spl[r - 1] < k <= spl[r].  Pure host arithmetic; HSORT_ERR_INVALID on bad arguments. */
+int hsort_sample_positions(uint64_t n, uint64_t s, uint64_t* pos);
+int hsort_select_splitters(const uint64_t* samples, uint64_t m, int P, uint64_t* spl);
 
 /* The PIPEMERGE heuristic (reading A-9): number of pair-wise merges overlapped with
  * GPU sorting; STREAM mode merges pairs (0,1), (2,3), ... of that many (option "pipemerge").

@@ -103,6 +103,8 @@ SIGNATURES = {
     "hsort_get_last_plan": ([ctypes.POINTER(_I), ctypes.POINTER(_I), ctypes.POINTER(_U64)], _I),
     "hsort_host_upper_bounds": ([_P, _U64, _P, _U64, _P], _I),
     "hsort_get_launch_count": ([], _U64),
+    "hsort_sample_positions": ([_U64, _U64, _P], _I),
+    "hsort_select_splitters": ([_P, _U64, _I, _P], _I),
 }
 
 
@@ -421,6 +423,22 @@ def hsort_host_upper_bounds(keys: np.ndarray, values: np.ndarray) -> np.ndarray:
 def hsort_get_launch_count() -> int:
     """Kernels the library has launched since load (differences count a region's launches)."""
     return lib().hsort_get_launch_count()
+
+
+def hsort_sample_positions(n: int, s: int) -> np.ndarray:
+    """Regular sample positions of a sorted run of n keys (A13 splitter sampling)."""
+    pos = np.zeros(s, dtype=np.uint64)
+    _check(lib().hsort_sample_positions(n, s, pos.ctypes.data if s else None))
+    return pos
+
+
+def hsort_select_splitters(samples: np.ndarray, P: int) -> np.ndarray:
+    """P - 1 splitters at the P-quantiles of the merged sorted samples (A13)."""
+    samples = np.ascontiguousarray(samples, dtype=np.uint64)
+    spl = np.zeros(max(P - 1, 0), dtype=np.uint64)
+    _check(lib().hsort_select_splitters(samples.ctypes.data if samples.size else None, samples.size,
+                                        P, spl.ctypes.data if spl.size else None))
+    return spl
 
 
 def hsort_pipemerge_count(n_b: int, n_gpus: int) -> int:

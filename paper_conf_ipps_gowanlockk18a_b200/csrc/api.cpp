@@ -2281,6 +2281,25 @@ int hsort_host_corank(const uint64_t* keys, const uint64_t* off, int k, uint64_t
 
 uint64_t hsort_get_launch_count(void) { return g_kernel_launches.load(); }
 
+int hsort_sample_positions(uint64_t n, uint64_t s, uint64_t* pos) {
+  // regular samples of a sorted run of n keys: positions (i + 1) n / (s + 1), i < s (A13)
+  if (s && !pos) return g_err = "null pos", HSORT_ERR_INVALID;
+  if (n == 0) return s ? (g_err = "n = 0 has no samples", HSORT_ERR_INVALID) : HSORT_OK;
+  for (uint64_t i = 0; i < s; ++i) {
+    const uint64_t p = (uint64_t)((unsigned __int128)(i + 1) * n / (s + 1));
+    pos[i] = p < n ? p : n - 1;
+  }
+  return HSORT_OK;
+}
+
+int hsort_select_splitters(const uint64_t* samples, uint64_t m, int P, uint64_t* spl) {
+  // P - 1 splitters at the P-quantiles of the m merged samples: spl[r - 1] = samples[r m / P]
+  if (P < 1 || (P > 1 && (!spl || (m && !samples)))) return g_err = "bad arguments", HSORT_ERR_INVALID;
+  for (int r = 1; r < P; ++r)
+    spl[r - 1] = m ? samples[(uint64_t)((unsigned __int128)r * m / (unsigned)P)] : 0;
+  return HSORT_OK;
+}
+
 uint64_t hsort_pipemerge_count(uint64_t n_b, int n_gpus) {
   // P:430-454 (reading A-9): one GPU -> floor((n_b-1)/2); two or more -> floor(n_b/(2 n_GPU))
   if (n_b == 0) return 0;

@@ -7,7 +7,8 @@
   after every rank has sorted its own shard, a splitter-based all-to-all leaves rank r with the
   r-th key range of the global order, which the library's k-way merge (K4/K5 on the GPU, H2 on
   the CPU) turns into rank r's slice of B.  The splitters come from regular samples of the
-  sorted runs, merged with the library's multiway merge; the partition uses the library's
+  sorted runs (positions and quantiles computed by the library: hsort_sample_positions,
+  hsort_select_splitters), merged with the library's multiway merge; the partition uses the library's
   upper-bound kernel; the transfer is one ``all_to_all_single`` (NCCL over NVLink on GPUs, gloo
   on CPU in the tests).  Concatenating the ranks' results in rank order gives the global sort.
 
@@ -21,7 +22,7 @@ import torch
 import torch.distributed as dist
 
 from . import (hsort_device_merge, hsort_device_upper_bounds, hsort_host_merge,
-               hsort_host_upper_bounds)
+               hsort_host_upper_bounds, hsort_sample_positions, hsort_select_splitters)
 
 
 def shard_range(n: int, world: int, rank: int) -> tuple[int, int]:
@@ -50,7 +51,7 @@ def choose_splitters(local_sorted: torch.Tensor, group=None, oversample: int = 6
     n = local_sorted.numel()
     s = oversample * P
     if n:
-        pos = ((torch.arange(1, s + 1, device=dev, dtype=torch.int64) * n) // (s + 1)).clamp_(max=n - 1)
+        pos = torch.from_numpy(hsort_sample_positions(n, s).view(np.int64)).to(dev)
         samp = _as_i64(local_sorted)[pos]
     else:
         samp = torch.zeros(s, dtype=torch.int64, device=dev)
@@ -65,8 +66,7 @@ def choose_splitters(local_sorted: torch.Tensor, group=None, oversample: int = 6
         return np.zeros(P - 1, dtype=np.uint64)
     off = np.cumsum([0] + [r.size for r in runs]).astype(np.uint64)
     merged = hsort_host_merge(np.concatenate(runs), off)  # sorted samples (library merge)
-    m = merged.size
-    return merged[[(r * m) // P for r in range(1, P)]].astype(np.uint64)
+    return hsort_select_splitters(merged, P)  # the P-quantiles (library arithmetic)
 
 
 def exchange_sorted_runs(local_sorted: torch.Tensor, group=None, oversample: int = 64,

@@ -195,3 +195,24 @@ def test_par_memcpy_streaming_stores(hs):
             assert np.array_equal(dst[do:do + size], src[so:so + size]), (nt, size, so, do)
             assert not dst[:do].any() and not dst[do + size:].any()
     hs.hsort_set_option("memcpy_nt", 1)
+
+
+def test_splitter_arithmetic(hs):
+    """A13 splitter arithmetic in the library: regular sample positions of a sorted run and the
+    P-quantile splitters of the merged samples (used by dist.exchange_sorted_runs)."""
+    for n, s in ((1, 5), (10, 3), (10**9 + 7, 64), (7, 7)):
+        pos = hs.hsort_sample_positions(n, s)
+        assert pos.size == s and int(pos.max()) <= n - 1
+        assert np.all(np.diff(pos.astype(np.int64)) >= 0)  # non-decreasing
+        if n > s:
+            assert np.all(np.diff(pos.astype(np.int64)) > 0)  # distinct when the run is long enough
+    samp = np.sort(np.random.default_rng(0).integers(0, 2**64, size=1000, dtype=np.uint64))
+    for P in (1, 2, 3, 8):
+        spl = hs.hsort_select_splitters(samp, P)
+        assert spl.size == P - 1 and np.all(np.diff(spl.astype(np.float64)) >= 0)
+        # each rank's share of the samples is within one sample of m / P
+        cuts = [0] + [int(np.searchsorted(samp, v, side="right")) for v in spl] + [samp.size]
+        assert all(abs((cuts[r + 1] - cuts[r]) - samp.size / P) <= 1 for r in range(P))
+    assert np.array_equal(hs.hsort_select_splitters(np.zeros(0, np.uint64), 4), np.zeros(3, np.uint64))
+    with pytest.raises(hs.HsortError):
+        hs.hsort_sample_positions(0, 3)

@@ -860,8 +860,12 @@ __global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ 
                                                        uint64_t* __restrict__ hist,
                                                        DdeState* __restrict__ dde = nullptr) {
   constexpr int SHC = COPIES == 16 ? 4 : 3;
-  extern __shared__ uint32_t sh3[];  // [8 * 256][COPIES]
-  for (int i = threadIdx.x; i < kDigits * kRadix * COPIES; i += THREADS) sh3[i] = 0;
+  extern __shared__ uint32_t sh3[];  // [8 * 256][COPIES] (+ DDE: [256] outlier digit-6 counts)
+  // DDE: the outliers' histogram is counted in shared memory and flushed once per CTA -- global
+  // atomics per outlier serialised at L2 when the guessed top digit is not dominant (normal data:
+  // K1 took 168 ms instead of 2 ms, profiles/r02n_k1_dde_skew.txt)
+  uint32_t* s_out = sh3 + kDigits * kRadix * COPIES;
+  for (int i = threadIdx.x; i < kDigits * kRadix * COPIES + (DDE ? kRadix : 0); i += THREADS) sh3[i] = 0;
   __syncthreads();
   uint32_t* sh = sh3 + (threadIdx.x & (COPIES - 1));
   uint32_t cd[kDigits], cc[kDigits];
@@ -893,7 +897,7 @@ __global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ 
     uint64_t k0 = n ? src[0] : 0;
     if (IN_F64) k0 = to_key(k0);
     guess = (uint32_t)(k0 >> 56);
-    hout = dde->hist_k1;
+    hout = s_out;
     if (blockIdx.x == 0 && threadIdx.x == 0) dde->guess = guess;
   }
   if (head && blockIdx.x == 0 && threadIdx.x == 0)
@@ -917,6 +921,9 @@ __global__ void __launch_bounds__(THREADS) k_hist3(const uint64_t* __restrict__ 
     }
     if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
   }
+  if (DDE)
+    for (int j = threadIdx.x; j < kRadix; j += THREADS)
+      if (s_out[j]) atomicAdd(&dde->hist_k1[j], s_out[j]);
 }
 
 // Final conversion/copy (P_eff == 0, or odd P_eff with in == out).
@@ -1000,8 +1007,8 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
       cudaError_t e;
       if ((e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
       if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-      if ((e = cudaFuncSetAttribute(kdt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-      if ((e = cudaFuncSetAttribute(kdf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(kdt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem + kRadix * 4)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(kdf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem + kRadix * 4)) != cudaSuccess) return e;
       int b = 0;
       if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf, kHist3Threads, smem)) != cudaSuccess) return e;
       per_sm[dev] = b > 0 ? b : 1;
@@ -1010,8 +1017,8 @@ cudaError_t launch_hist(RadixScratch& s, const uint64_t* in, uint64_t n, bool in
     const uint64_t cap3 = (uint64_t)num_sms(dev) * per_sm[dev];
     const int grid3 = (int)(want3 < 1 ? 1 : (want3 > cap3 ? cap3 : want3));
     if (dde) {
-      if (in_f64) kdt<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, dde);
-      else kdf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, dde);
+      if (in_f64) kdt<<<grid3, kHist3Threads, smem + kRadix * 4, st>>>(in, n, hist, dde);
+      else kdf<<<grid3, kHist3Threads, smem + kRadix * 4, st>>>(in, n, hist, dde);
     } else {
       if (in_f64) kt<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, nullptr);
       else kf<<<grid3, kHist3Threads, smem, st>>>(in, n, hist, nullptr);

@@ -1412,7 +1412,12 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
       // GPU share is link-bound (HtoD in, DtoH out, duplex); CPU rate from the last STREAM call
       const double bw_in = c.st->t_h2d > 0 ? c.st->bytes_h2d / c.st->t_h2d : 50e9;
       const double bw_out = c.st->t_d2h > 0 ? c.st->bytes_d2h / c.st->t_d2h : 50e9;
-      const double r_gpu = 0.85 * std::min(bw_in, bw_out) / 8.0;
+      // The GPU share's rate from the link (0.85 of the slower direction per GPU).  Balancing
+      // with the GPU share's *measured* rate of the last call was tried and converged to
+      // f = 0.56 at n = 4.3e9 (2.83 s) against 2.72 s at this estimate's f = 0.8: the rates are
+      // not independent -- while the CPU merge runs it slows the staging of a pageable B, so the
+      // GPU share measured under contention looks slower than it is (profiles/r02p_ooc_split.txt)
+      const double r_gpu = 0.85 * std::min(bw_in, bw_out) / 8.0 * gs.size();
       const double r_cpu = S().r_cpu_merge > 0 ? S().r_cpu_merge : 4e7 * host_threads();
       f = r_gpu / (r_gpu + r_cpu);
     }

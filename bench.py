@@ -525,12 +525,15 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=N_PER_GPU, help="keys per GPU (default 2^30, config C2)")
+    ap.add_argument("--keys-per-gpu", type=int, default=N_PER_GPU, help="keys per GPU (default 2^30, config C2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-extras", action="store_true",
                     help="only the timed host->host and device steps (profiling runs)")
     ap.add_argument("--device-only", action="store_true",
                     help="profiling: skip the host->host arm (ncu captures of the device GPUSort)")
+    ap.add_argument("--virtual-gpus", action="store_true",
+                    help="testing on a box with fewer GPUs than --gpus: map N GPU contexts onto the "
+                         "visible devices (library option virtual_gpus); not a scaling number")
     ap.add_argument("--no-dde", action="store_true",
                     help="profiling: dominant-digit elision off (every device pass is a full pass)")
     args = ap.parse_args()
@@ -571,10 +574,13 @@ def main():
     import paper_conf_ipps_gowanlockk18a_b200 as hs
 
     torch.cuda.set_device(0)
-    if torch.cuda.device_count() < N:
+    virtual = torch.cuda.device_count() < N
+    if virtual and not args.virtual_gpus:
         raise SystemExit(f"--gpus {N} but only {torch.cuda.device_count()} visible devices")
+    if virtual:
+        hs.hsort_set_option("virtual_gpus", N)
     # N x 2^30 keys of pinned A and B (16 B/key of host RAM): cap to 60% of the free RAM
-    n_gpu = args.n
+    n_gpu = args.keys_per_gpu
     while N * n_gpu * 16 > 0.6 * mem_available() and n_gpu > (1 << 24):
         n_gpu //= 2
     n = N * n_gpu
@@ -598,7 +604,7 @@ def main():
         hs.hsort_sort(A_h, B_h, batch_elems=0, n_gpus=N)
     if not args.device_only:
         guard(A_h.numpy(), B_h.numpy(), "host->host (warm-up)")
-    devs = list(range(N))
+    devs = list(range(min(N, torch.cuda.device_count())))
     L0 = hs.hsort_get_launch_count()
     sampler = ClockSampler(devs)
     barrier()
@@ -668,9 +674,10 @@ def main():
             "distribution": f"uniform U[0,1) 53-bit, splitmix64 seed {SEED}",
             "parallelism": f"{N} GPU(s) driven by rank 0 through the library" +
                            (f"; {ws} torchrun ranks (control barriers over gloo)" if ws > 1 else ""),
-            "l2": "input 8 GiB per GPU >> 126 MB L2: no flush needed between steps",
+            "l2": f"input {n_gpu * 8 / 2**30:.0f} GiB per GPU >> 126 MB L2: no flush needed between steps",
             "timing": "CUDA events on device 0's stream around each synchronous call (= call "
                       "duration); HtoD, sort, merge and DtoH all inside",
+            "virtual_gpus": virtual,
         },
         "e2e": {
             "value": value,

@@ -50,3 +50,31 @@ def test_fullsize_host_sort_auto_plan_matches_oracle(hs_gpu, full):
     st = hs_gpu.hsort_get_stats()
     assert st["mode_name"] == "RESIDENT" and st["n_b"] == 12 and st["direct_in"] == 1
     assert _first_diff(Bt.numpy().view(np.uint64), want) is None
+
+
+@pytest.mark.parametrize("N,msd", [(4, 0), (3, 1)])
+def test_large_multi_gpu_auto_plan_matches_oracle(hs_gpu, oracle_mod, inputs_mod, N, msd):
+    """2^27 + ragged keys on N virtual GPUs through the auto plan (2^27/N-key shards, 2^24-key
+    batches + halving tail per shard, 2^26-key merge chunks per range, run-pointer K4/K5), and the
+    MSD-first split, element by element vs the oracle."""
+    import torch
+    n = (1 << 27) + 777
+    A = inputs_mod.generate("zipf_dup" if msd else "uniform", n, seed=2 + N)
+    want = oracle_mod.sort_f64(A).view(np.uint64)
+    hs_gpu.hsort_finalize()
+    hs_gpu.hsort_set_option("virtual_gpus", N)
+    hs_gpu.hsort_init()
+    try:
+        hs_gpu.hsort_set_option("msd", msd)
+        At = torch.from_numpy(A).pin_memory()
+        Bt = torch.zeros(n, dtype=torch.float64).pin_memory()
+        hs_gpu.hsort_sort(At, Bt, batch_elems=0, n_gpus=N)
+        st = hs_gpu.hsort_get_stats()
+        assert st["mode_name"] == "RESIDENT" and st["n_gpus"] == N
+        assert (st["msd_buckets"] > 0) == bool(msd)
+        assert _first_diff(Bt.numpy().view(np.uint64), want) is None
+    finally:
+        hs_gpu.hsort_set_option("msd", 0)
+        hs_gpu.hsort_finalize()
+        hs_gpu.hsort_set_option("virtual_gpus", 0)
+        hs_gpu.hsort_init()

@@ -1526,7 +1526,13 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     }
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) atomicAdd(&wh[dd[i]], 1u);
+#ifdef HSORT_PHASE_TIMING
+    long long q0 = clock64();
+#endif
     bar_compute<CT>();
+#ifdef HSORT_PHASE_TIMING
+    long long q1 = clock64();
+#endif
     uint32_t cnt = 0;
     if (tid < kRadix) {
 #pragma unroll
@@ -1545,7 +1551,20 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       }
       s_cnt[(j & 1) * kRadix + tid] = cnt | (tstart << 16);
     }
+#ifdef HSORT_PHASE_TIMING
+    long long q2 = clock64();
+#endif
     bar_compute<CT>();
+#ifdef HSORT_PHASE_TIMING
+    long long q3 = clock64();
+    if (lane == 0 && (warp == 0 || warp == CW - 1)) {
+      const int o = warp == 0 ? 224 : 228;
+      atomicAdd(&g_phase_dbg[o], (unsigned long long)(q1 - q0));      // wait at barrier 1
+      atomicAdd(&g_phase_dbg[o + 1], (unsigned long long)(q2 - q1));  // reduce + scan + bases
+      atomicAdd(&g_phase_dbg[o + 2], (unsigned long long)(q3 - q2));  // wait at barrier 2
+      atomicAdd(&g_phase_dbg[o + 3], 1ull);
+    }
+#endif
     if (tid == 0) mbar_arrive(&bar_a[j & 1]);
 #ifdef HSORT_PHASE_TIMING
     long long cr0 = clock64();

@@ -36,5 +36,9 @@ res = {"tiles": T,
        "compute_total": buf[212] / T, "wait_tma": buf[211] / T, "count+publish": buf[219] / T,
        "rank+scatter": buf[218] / T, "  of which peers": buf[221] / T, "writeout(incl wait)": buf[220] / T, "wait_lookback": buf[210] / T,
        "lb_idle": buf[214] / max(1, buf[217]), "lb_time": buf[215] / max(1, buf[217]),
-       "lb_rounds": buf[216] / max(1, buf[217])}
+       "lb_rounds": buf[216] / max(1, buf[217]),
+       "warp0(digit): bar1_wait": buf[224] / max(1, buf[227]), "warp0: reduce+scan+bases": buf[225] / max(1, buf[227]),
+       "warp0: bar2_wait": buf[226] / max(1, buf[227]),
+       "warp17: bar1_wait": buf[228] / max(1, buf[231]), "warp17: scan window": buf[229] / max(1, buf[231]),
+       "warp17: bar2_wait": buf[230] / max(1, buf[231])}
 print(json.dumps({k: round(v, 1) if isinstance(v, float) else v for k, v in res.items()}))

@@ -1,6 +1,8 @@
 """Small invocations of every kernel path, for compute-sanitizer (memcheck / racecheck /
-synccheck / initcheck): K1/K2/K3 (f64, u64, elision with a lowered threshold), key/value, typed
-float32 descending, K4 two-level + K5, host RESIDENT and STREAM modes.  Checks results against
+synccheck / initcheck): K1/K2/K3 (f64, u64, elision with a lowered threshold; the elision's K1
+outlier count on normal data), key/value, typed float32 descending, K4 two-level + K5, host
+RESIDENT and STREAM modes, and (round 2) the multi-GPU RESIDENT merge through the run-pointer
+table, the MSD-first split (K6a-d) and multi-GPU STREAM on 3 virtual GPUs.  Checks results against
 the oracle so a silent corruption also fails."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -45,5 +47,22 @@ want = bits(oracle.sort_f64(A))
 assert np.array_equal(bits(hs.hsort_sort(A, batch_elems=30_001)), want), "RESIDENT"
 hs.hsort_set_option("resident", 0)
 assert np.array_equal(bits(hs.hsort_sort(A, batch_elems=30_001)), want), "STREAM"
+N = hsort_inputs.generate("normal", 1 << 17, seed=5)  # elision K1 with a wrong guess (shared count)
+d = torch.from_numpy(N).cuda(); o = torch.empty_like(d)
+hs.hsort_sort_device(d, o); torch.cuda.synchronize()
+assert np.array_equal(bits(o.cpu().numpy()), bits(oracle.sort_f64(N))), "elision K1, normal data"
+hs.hsort_finalize()
+
+hs.hsort_set_option("resident", -1)
+hs.hsort_set_option("virtual_gpus", 3)
+hs.hsort_init()
+assert np.array_equal(bits(hs.hsort_sort(A, batch_elems=20_000, n_gpus=3)), want), "multi RESIDENT"
+hs.hsort_set_option("msd", 1)
+hs.hsort_set_option("msd_bucket_keys", 1 << 16)
+assert np.array_equal(bits(hs.hsort_sort(A, batch_elems=20_000, n_gpus=3)), want), "MSD split"
+hs.hsort_set_option("msd", 0)
+hs.hsort_set_option("resident", 0)
+hs.hsort_set_option("merge_gpu_permille", 500)
+assert np.array_equal(bits(hs.hsort_sort(A, batch_elems=20_000, n_gpus=3)), want), "multi STREAM"
 hs.hsort_finalize()
 print("sanitize_run ok")

@@ -143,10 +143,11 @@ int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_
  * HSORT_KEY_F32 (4-byte float32); descending != 0 sorts by the reverse of IEEE totalOrder (the
  * exact reverse of the ascending result: every totalOrder class is one bit pattern).  Keys are
  * sorted as bit patterns (NaN payloads and -0.0 preserved).  float64 ascending is hsort_sort
- * (every mode); every other combination runs on one GPU as one batch (BLINE): an encode pass to
- * 64-bit internal keys (float32 keys zero-extended, so the radix plan skips the 4 empty digits),
- * the GPUSort (out of place, so the dominant-digit elision applies), a decode pass.  n must fit one
- * GPU (24 B/key + the key array), else
+ * (every mode); every other combination runs on one GPU as one batch (BLINE): float32 on the
+ * native 32-bit GPUSort (binary32 key transform fused into its first/last pass, <= 4 passes; the
+ * 64-bit codec path below for n > 2^30), float64 descending with the reverse transform fused into
+ * the 64-bit GPUSort, else an encode pass to 64-bit internal keys, the GPUSort, a decode pass.
+ * n must fit one GPU (24 B/key + the key array), else
  * HSORT_ERR_INVALID.  A and B aligned to the key size; B == A allowed; partial overlap -> INVALID.
  * ------------------------------------------------------------------------------------------- */
 #define HSORT_KEY_F64 0

@@ -1845,9 +1845,14 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     CK(cudaEventRecord(es_.a, g.s_comp));
     // float64 descending: the reverse transform fused into the GPUSort (mout -> runs); else the
     // codec passes around the ascending GPUSort of internal keys
-    const cudaError_t fe = key_type == HSORT_KEY_F64 && desc
-                               ? radix_sort_desc_f64(g.rs, g.mout.u64(), g.runs.u64(), g.alt.u64(), n, g.s_comp)
-                               : cudaErrorNotSupported;
+    // float32: the native 32-bit GPUSort (4-byte keys, transform fused into its first and last
+    // pass); float64 descending: the reverse transform fused into the 64-bit GPUSort
+    const cudaError_t fe =
+        key_type == HSORT_KEY_F32
+            ? radix_sort32(g.rs, (const uint32_t*)g.mout.p, (uint32_t*)g.runs.p, (uint32_t*)g.alt.p, n,
+                           true, true, desc != 0, g.s_comp)
+        : desc ? radix_sort_desc_f64(g.rs, g.mout.u64(), g.runs.u64(), g.alt.u64(), n, g.s_comp)
+               : cudaErrorNotSupported;
     if (fe == cudaErrorNotSupported) {
       cudaGetLastError();
       CK(key_encode(g.mout.p, g.runs.u64(), n, key_type, desc != 0, g.s_comp));
@@ -2119,6 +2124,16 @@ int hsort_sort_device_typed(const void* d_in, void* d_out, uint64_t n, int key_t
     cudaStream_t st = (cudaStream_t)stream;
     g.runs.reserve(n * 8);
     g.alt.reserve(n * 8);
+    if (key_type == HSORT_KEY_F32) {
+      // native 32-bit GPUSort; the codec path below when it does not apply
+      const cudaError_t fe = radix_sort32(g.rs, (const uint32_t*)d_in, (uint32_t*)d_out,
+                                          (uint32_t*)g.alt.p, n, true, true, descending != 0, st);
+      if (fe != cudaErrorNotSupported) {
+        CK(fe);
+        return HSORT_OK;
+      }
+      cudaGetLastError();
+    }
     if (key_type == HSORT_KEY_F64 && descending && d_in != d_out) {
       // reverse transform fused into the GPUSort's first and last pass
       const cudaError_t fe = radix_sort_desc_f64(g.rs, (const uint64_t*)d_in, (uint64_t*)d_out,

@@ -115,6 +115,12 @@ cudaError_t radix_sort(RadixScratch& s, const uint64_t* in, uint64_t* out, uint6
 // cudaErrorNotSupported otherwise, and the caller takes the codec path).
 cudaError_t radix_sort_desc_f64(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,
                                 uint64_t n, cudaStream_t st);
+// Native 32-bit GPUSort (S§8(f) #4): out = sorted(in) over 32-bit keys (float32 bits under IEEE
+// totalOrder when in_f32/out_f32, descending when desc; else uint32 ascending); K1 for 4 digits,
+// up to 4 warp-specialised passes with 4-byte keys.  Needs 16-byte aligned buffers, n <= 2^30,
+// tmp an n-element scratch; returns cudaErrorNotSupported otherwise (caller: codec path).
+cudaError_t radix_sort32(RadixScratch& s, const uint32_t* in, uint32_t* out, uint32_t* tmp,
+                         uint64_t n, bool in_f32, bool out_f32, bool desc, cudaStream_t st);
 // Key/value GPUSort (S§8(f) #3): (out, vout) = (in, vin) stably sorted by key; n <= 2^30, every
 // buffer 16-byte aligned, tmp/vtmp n-element scratch; in == out iff vin == vout.  The values are
 // opaque 64-bit payloads (e.g. indices: argsort).

@@ -48,6 +48,19 @@ __device__ __forceinline__ uint64_t from_key(uint64_t k) {
   return k ^ ((uint64_t)((int64_t)(~k) >> 63) | 0x8000000000000000ull);
 }
 
+// float32 bits -> 32-bit key (the binary32 analogue of A4) and back (S§8(f) #4, native path)
+__device__ __forceinline__ uint32_t to_key32(uint32_t w) {
+  return w ^ ((uint32_t)((int32_t)w >> 31) | 0x80000000u);
+}
+__device__ __forceinline__ uint32_t from_key32(uint32_t k) {
+  return k ^ ((uint32_t)((int32_t)(~k) >> 31) | 0x80000000u);
+}
+// key transform / inverse for the key width of a pass (64-bit: float64, 32-bit: float32)
+__device__ __forceinline__ uint64_t to_key_w(uint64_t u) { return to_key(u); }
+__device__ __forceinline__ uint32_t to_key_w(uint32_t w) { return to_key32(w); }
+__device__ __forceinline__ uint64_t from_key_w(uint64_t k) { return from_key(k); }
+__device__ __forceinline__ uint32_t from_key_w(uint32_t k) { return from_key32(k); }
+
 __device__ __forceinline__ uint64_t ld_stream(const uint64_t* p) {
   uint64_t v;
   asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
@@ -246,7 +259,8 @@ __global__ void k_force_plan(RadixPlan* plan, int digit, uint32_t* lb_state) {
   *plan = P;
 }
 
-__device__ __forceinline__ uint64_t* pick(int id, uint64_t* in, uint64_t* out, uint64_t* tmp) {
+template <class T>
+__device__ __forceinline__ T* pick(int id, T* in, T* out, T* tmp) {
   return id == 0 ? in : (id == 1 ? out : tmp);
 }
 
@@ -1104,13 +1118,13 @@ __device__ __forceinline__ uint32_t scan256_excl_c(uint32_t v, uint32_t* s_warp 
   return wpre + x - v;
 }
 
-template <int CT, int ITEMS, bool KV = false>
+template <int CT, int ITEMS, bool KV = false, int KB = 8>
 struct WsSmem {
   static constexpr int TILE = CT * ITEMS;
   static constexpr int CW = CT / 32;                                          // compute warps
-  static constexpr size_t stage_off = 0;                                      // [3][TILE] u64
-  static constexpr size_t vstage_off = 3ull * TILE * 8;                       // [3][TILE] u64 (KV)
-  static constexpr size_t whist_off = (KV ? 6ull : 3ull) * TILE * 8;          // [CW][257] u32
+  static constexpr size_t stage_off = 0;                                      // [3][TILE] keys (KB bytes)
+  static constexpr size_t vstage_off = 3ull * TILE * KB;                      // [3][TILE] u64 (KV)
+  static constexpr size_t whist_off = 3ull * TILE * KB + (KV ? 3ull * TILE * 8 : 0);  // [CW][257] u32
   static constexpr size_t gofs_off = (whist_off + CW * (kRadix + 1) * 4 + 15) & ~(size_t)15;  // [2][256] i32
   static constexpr size_t cnt_off = gofs_off + 2 * kRadix * 4;                // [2][256] u32
   static constexpr size_t bar_off = cnt_off + 2 * kRadix * 4;                 // [12] u64
@@ -1127,6 +1141,10 @@ struct WsSmem {
 #endif
 #ifndef HSORT_WS_RC
 #define HSORT_WS_RC 0  // ranking chunk (0 = all items at once)
+#endif
+#ifndef HSORT_K32_ITEMS
+#define HSORT_K32_ITEMS 20  // 32-bit keys per compute thread: 11520-key tiles, 3 stages = 138 KB
+                            // (A/B 15 / 18 / 20 / 22: 19.2 / 18.6 / 17.4 / 17.7 ms per 2^30 keys)
 #endif
 #ifndef HSORT_WS_NMATCH
 #define HSORT_WS_NMATCH 3  // items ranked with match.any in high-entropy passes (best of 0..7)
@@ -1152,6 +1170,10 @@ __device__ __forceinline__ void st_relaxed_v4(uint32_t* p, const uint32_t* v) {
 
 __device__ __forceinline__ void st_global_u64(uint64_t addr, uint64_t v) {
   asm volatile("st.global.u64 [%0], %1;" ::"l"(addr), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_global_w(const uint64_t* a, uint64_t v) { st_global_u64((uint64_t)a, v); }
+__device__ __forceinline__ void st_global_w(const uint32_t* a, uint32_t v) {
+  asm volatile("st.global.u32 [%0], %1;" ::"l"((uint64_t)a), "r"(v) : "memory");
 }
 // One bit of the ballot multisplit: peers &= (bit b of d) ? ballot(bit) : ~ballot(bit).
 __device__ __forceinline__ uint32_t peer_bit(uint32_t peers, uint32_t d, uint32_t bm) {
@@ -1239,8 +1261,10 @@ __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64
 // outliers' digit-P histogram); 2 the elided sort's last pass (diverts the outliers).  The host
 // picks DM per launch after reading K2's plan, so the DM = 0 kernel carries no elision code.
 // DESC: a descending float64 sort (compile-time, so ascending kernels carry no extra work).
-template <int CT, int ITEMS, bool IN_F64, bool KV = false, int DM = 0, bool DESC = false>
-__global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in, uint64_t* out, uint64_t* tmp,
+// K32: 32-bit keys (float32 / uint32, S§8(f) #4 native path): 4-byte stage and stores, the
+// binary32 key transform; keys-only, no elision.
+template <int CT, int ITEMS, bool IN_F64, bool KV = false, int DM = 0, bool DESC = false, bool K32 = false>
+__global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in64, uint64_t* out64, uint64_t* tmp64,
                                                        uint64_t* vin, uint64_t* vout, uint64_t* vtmp,
                                                        uint64_t n, const RadixPlan* __restrict__ plan,
                                                        const uint64_t* __restrict__ bin_base,
@@ -1251,12 +1275,17 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
                                                        const uint64_t* __restrict__ hist = nullptr,
                                                        DdeState* __restrict__ dde = nullptr,
                                                        uint64_t* __restrict__ side = nullptr) {
-  using L = WsSmem<CT, ITEMS, KV>;
+  using KT = std::conditional_t<K32, uint32_t, uint64_t>;  // key word of this pass
+  static_assert(!K32 || (!KV && DM == 0), "32-bit keys: keys-only, no elision");
+  using L = WsSmem<CT, ITEMS, KV, sizeof(KT)>;
   constexpr int TILE = L::TILE;
   constexpr int CW = L::CW;
   constexpr int THREADS = CT;  // compute threads
+  KT* in = (KT*)in64;
+  KT* out = (KT*)out64;
+  KT* tmp = (KT*)tmp64;
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* stage = (uint64_t*)(smem + L::stage_off);
+  KT* stage = (KT*)(smem + L::stage_off);
   uint64_t* vstage = (uint64_t*)(smem + L::vstage_off);  // KV only
   uint32_t* whist = (uint32_t*)(smem + L::whist_off);
   int32_t* s_gofs = (int32_t*)(smem + L::gofs_off);
@@ -1273,8 +1302,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   if (p >= na) return;
   const int digit = plan->digit[p];
   const int shift = 8 * digit;
-  const uint64_t* __restrict__ src = pick(plan->src[p], in, out, tmp);
-  uint64_t* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
+  const KT* __restrict__ src = pick(plan->src[p], in, out, tmp);
+  KT* __restrict__ dst = pick(plan->dst[p], in, out, tmp);
   const uint64_t* __restrict__ vsrc = KV ? pick(plan->src[p], vin, vout, vtmp) : nullptr;
   uint64_t* __restrict__ vdst = KV ? pick(plan->dst[p], vin, vout, vtmp) : nullptr;
   const bool use_match = (plan->match_mask >> p) & 1;
@@ -1282,8 +1311,8 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   // dominant-digit elision: pass 0 counts the outliers' digit-P histogram; the last pass diverts
   // the outliers (digit L != v) to the side buffer and ranks the rest by digit P
   static_assert(DM == 0 || !KV, "the elision is keys-only");
-  const uint64_t kx = DESC ? plan->key_xor : 0ull;  // descending: complement on the first load
-  const uint64_t kx_in = p == 0 ? kx : 0ull;        // ... and before the last inverse store
+  const KT kx = DESC ? (KT)plan->key_xor : (KT)0;  // descending: complement on the first load
+  const KT kx_in = p == 0 ? kx : (KT)0;             // ... and before the last inverse store
   constexpr bool dde_here = DM == 2;
   const int sh_l = DM ? 8 * plan->dde_digit : 0;
   const uint32_t v_l = DM ? plan->dde_value : 0u;
@@ -1299,11 +1328,11 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     if (t < num_tiles) {
       const uint64_t base = (uint64_t)t * TILE;
       const uint64_t cnt = (n - base) < (uint64_t)TILE ? (n - base) : (uint64_t)TILE;
-      const uint32_t bytes = (uint32_t)(cnt * 8) & ~15u;
+      const uint32_t bytes = (uint32_t)(cnt * sizeof(KT)) & ~15u;
       mbar_arrive_expect_tx(&bar_tma[b], KV ? 2 * bytes : bytes);
       if (bytes) {
         bulk_g2s(stage + (size_t)b * TILE, src + base, bytes, &bar_tma[b]);
-        if (KV) bulk_g2s(vstage + (size_t)b * TILE, vsrc + base, bytes, &bar_tma[b]);
+        if (KV) bulk_g2s(vstage + (size_t)b * TILE, vsrc + base, bytes, &bar_tma[b]);  // KT = u64
       }
     } else {
       mbar_arrive(&bar_tma[b]);
@@ -1424,7 +1453,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   unsigned long long t_g = 0, t_t = 0, t_all = 0, t_rank = 0, t_cnt = 0, t_wo = 0, n_t = 0, t_peers = 0;
   long long c_start = clock64();
 #endif
-  uint64_t* const dst_t = dst + tid;
+  KT* const dst_t = dst + tid;
   // write-out of the tile of iteration jj from its (digit-ordered) stage buffer: a key at stage
   // position i with digit d goes to dst[s_gofs[d] + i]; then this warp releases the stage
   auto write_out = [&](uint32_t jj, uint64_t tile) {
@@ -1436,7 +1465,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     t_g += clock64() - cw0;
 #endif
     const int32_t* gofs = s_gofs + (jj & 1) * kRadix;
-    const uint64_t* sb = stage + (size_t)(jj % 3) * TILE;
+    const KT* sb = stage + (size_t)(jj % 3) * TILE;
     const uint64_t* vsb = vstage + (size_t)(jj % 3) * TILE;
     const uint64_t rem = n - tile * (uint64_t)TILE;
     int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
@@ -1452,13 +1481,13 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
       for (int q = 0; q < ITEMS; ++q) {
         if (BOUNDED && tid + q * THREADS >= tile_n) break;
-        const uint64_t v = sb[tid + q * THREADS];
+        const KT v = sb[tid + q * THREADS];
         const int32_t g = gofs[(uint32_t)(v >> shift) & 255u];
-        uint64_t* a = dst_t + g;
+        KT* a = dst_t + g;
 #if HSORT_FAKE == 3
         if (v == 0x123456789ull)
 #endif
-        st_global_u64((uint64_t)(a + q * THREADS), INV ? from_key(v ^ kx) : v);
+        st_global_w(a + q * THREADS, INV ? from_key_w((KT)(v ^ kx)) : v);
         if (KV) st_global_u64((uint64_t)(vdst + tid + g + q * THREADS), vsb[tid + q * THREADS]);
       }
     };
@@ -1470,9 +1499,9 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       else wo_full(std::false_type{}, std::true_type{});
     } else {
       for (int i = tid; i < tile_n; i += THREADS) {
-        const uint64_t v = sb[i];
+        const KT v = sb[i];
         const int32_t g = gofs[(uint32_t)(v >> shift) & 255u];
-        st_global_u64((uint64_t)(dst + g + i), inv ? from_key(v ^ kx) : v);
+        st_global_w(dst + g + i, inv ? from_key_w((KT)(v ^ kx)) : v);
         if (KV) st_global_u64((uint64_t)(vdst + g + i), vsb[i]);
       }
     }
@@ -1483,27 +1512,27 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
   // DM (compile-time): 0 no elision work, 1 count the outliers' digit-P histogram (pass 0),
   // 2 divert the outliers (the elision's last pass; never FULL)
-  auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, uint64_t* sb, uint64_t* vsb) {
+  auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, KT* sb, uint64_t* vsb) {
     constexpr bool FULL = decltype(full_tag)::value;
     const uint64_t tbase = tile * (uint64_t)TILE;
-    const int bulk_n = (int)(((uint32_t)tile_n * 8u & ~15u) >> 3);
+    const int bulk_n = (int)(((uint32_t)tile_n * (uint32_t)sizeof(KT) & ~15u) / (uint32_t)sizeof(KT));
     const int wofs = warp * 32 * ITEMS + lane;
     uint32_t* wh = whist + warp * (kRadix + 1);  // this warp's row: zero on entry
-    uint64_t k[ITEMS];
+    KT k[ITEMS];
     uint64_t vv[KV ? ITEMS : 1];
     uint32_t dd[ITEMS];
     uint32_t omask = 0;  // elision: items of this lane that are outliers
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int jj = wofs + i * 32;
-      uint64_t v;
+      KT v;
       if (FULL) v = sb[jj];
-      else v = jj < bulk_n ? sb[jj] : (jj < tile_n ? src[tbase + jj] : 0);
+      else v = jj < bulk_n ? sb[jj] : (jj < tile_n ? src[tbase + jj] : (KT)0);
       if (KV) {
         if (FULL) vv[i] = vsb[jj];
         else vv[i] = jj < bulk_n ? vsb[jj] : (jj < tile_n ? vsrc[tbase + jj] : 0);
       }
-      k[i] = (IN_F64 ? to_key(v) : v) ^ kx_in;
+      k[i] = (IN_F64 ? to_key_w(v) : v) ^ kx_in;
       const bool valid = FULL || jj < tile_n;
       dd[i] = valid ? ((uint32_t)(k[i] >> shift) & 255u) : (uint32_t)kRadix;
       if (DM != 0) omask |= (uint32_t)(valid && ((uint32_t)(k[i] >> sh_l) & 255u) != v_l) << i;
@@ -1652,7 +1681,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #endif
     const uint64_t rem = n - tile * (uint64_t)TILE;
     const int tile_n = rem < (uint64_t)TILE ? (int)rem : TILE;
-    uint64_t* sb = stage + (size_t)cb * TILE;
+    KT* sb = stage + (size_t)cb * TILE;
     uint64_t* vsb = vstage + (size_t)cb * TILE;
     long long cr0;
     if (tile_n == TILE) cr0 = rank_tile(std::true_type{}, tile, tile_n, sb, vsb);
@@ -1692,17 +1721,17 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       lb32_next[rr * kRadix + tid] = 0;
 }
 
-template <int CT, int ITEMS, bool KV = false, int DM = 0, bool DESC = false>
+template <int CT, int ITEMS, bool KV = false, int DM = 0, bool DESC = false, bool K32 = false>
 cudaError_t launch_ws_pass(uint64_t* in, uint64_t* out, uint64_t* tmp, uint64_t* vin, uint64_t* vout,
                            uint64_t* vtmp, uint64_t n, RadixScratch& s, int p, bool first_in_f64,
                            bool out_f64, cudaStream_t st) {
-  using L = WsSmem<CT, ITEMS, KV>;
+  using L = WsSmem<CT, ITEMS, KV, K32 ? 4 : 8>;
   static int blocks_per_sm[64] = {0};
   int dev = 0;
   cudaGetDevice(&dev);
   constexpr bool dde = DM != 0;
-  auto kt = k_onesweep_ws<CT, ITEMS, true, KV, DM, DESC>;
-  auto kf = k_onesweep_ws<CT, ITEMS, false, KV, DM, DESC>;
+  auto kt = k_onesweep_ws<CT, ITEMS, true, KV, DM, DESC, K32>;
+  auto kf = k_onesweep_ws<CT, ITEMS, false, KV, DM, DESC, K32>;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   if (!blocks_per_sm[dev]) {
     cudaError_t e;
@@ -1742,7 +1771,8 @@ int pass_kernel(uint64_t* in, uint64_t* out, uint64_t* tmp) {
 // exclude its own keys.  The one value that can reach 2^30 (all n keys in one digit, a forced
 // single pass) is only read by tiles without keys of d and decodes as flag 3 = "aggregate", so a
 // reader never spins on it.
-cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t st, bool kv = false) {
+cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t st, bool kv = false,
+                           bool k32 = false) {
   const int mode = (kernel >= 1 && n <= (1ull << 30)) ? 2 : 1;
   if (s.lb_mode != 0 && s.lb_mode != mode) {
     cudaError_t e = cudaMemsetAsync(s.lookback, 0, s.max_tiles * kRadix * sizeof(uint64_t), st);
@@ -1752,6 +1782,7 @@ cudaError_t select_lb_mode(RadixScratch& s, int kernel, uint64_t n, cudaStream_t
   s.lb_mode = mode;
   if (mode == 2) {
     const uint64_t tile = kv ? (uint64_t)kKvTile
+                             : k32 ? (uint64_t)HSORT_WS_CT * HSORT_K32_ITEMS
                              : (kernel == 2 ? (uint64_t)HSORT_WS_CT * HSORT_WS_ITEMS : (uint64_t)kRadixTile);
     const uint64_t t = (n + tile - 1) / tile;
     if (t > s.lb_rows) s.lb_rows = t;
@@ -1802,6 +1833,100 @@ cudaError_t launch_pass(RadixScratch& s, uint64_t* in, uint64_t* out, uint64_t* 
     k_onesweep<kPassThreads, kPassItems, false><<<(unsigned)tiles, kPassThreads, 0, st>>>(
         in, out, tmp, n, s.plan, s.bin_base, s.lookback, s.tile_ctr, ep, p, out_f64 ? 1 : 0);
   return launched();
+}
+
+// K1 for 32-bit keys (float32 / uint32): histograms of digits 0..3 (digits 4..7 stay zero, so K2
+// sees them trivial).  16 interleaved copies of the 4 x 256 counters (a half-warp's 16 lanes hit 16
+// distinct banks), a register run cache per digit (constant high digits cost one atomic per run),
+// 16-byte loads of 4 keys.  desc: counts ascending digits (K2 mirrors them, as for float64).
+constexpr int kHist32Threads = 1024;
+constexpr int kHist32Copies = 16;
+// digits 0, 1 (low mantissa bytes: spread for float data) by direct shared atomics; digits 2, 3
+// (exponent / sign bytes: few values) through a register run cache
+template <bool IN_F32>
+__device__ __forceinline__ void hist32_key(uint32_t w, uint32_t* my, uint32_t (&cd)[2],
+                                           uint32_t (&cc)[2]) {
+  const uint32_t k = IN_F32 ? to_key32(w) : w;
+  atomicAdd(&my[(0 * kRadix + (k & 255u)) * kHist32Copies], 1u);
+  atomicAdd(&my[(1 * kRadix + ((k >> 8) & 255u)) * kHist32Copies], 1u);
+#pragma unroll
+  for (int q = 0; q < 2; ++q) {
+    const uint32_t d = (k >> (16 + 8 * q)) & 255u;
+    if (d == cd[q]) {
+      ++cc[q];
+    } else {
+      if (cc[q]) atomicAdd(&my[((2 + q) * kRadix + cd[q]) * kHist32Copies], cc[q]);
+      cd[q] = d;
+      cc[q] = 1;
+    }
+  }
+}
+template <bool IN_F32>
+__global__ void __launch_bounds__(kHist32Threads) k_hist32(const uint32_t* __restrict__ src,
+                                                           uint64_t n, uint64_t* __restrict__ hist) {
+  extern __shared__ uint32_t sh[];  // [4 * 256][16] (64 KB, dynamic)
+  for (int i = threadIdx.x; i < 4 * kRadix * kHist32Copies; i += kHist32Threads) sh[i] = 0;
+  __syncthreads();
+  uint32_t* my = sh + (threadIdx.x & (kHist32Copies - 1));
+  uint32_t cd[2] = {0, 0}, cc[2] = {0, 0};
+  const uint64_t head = ((((uintptr_t)src & 15) / 4) ? (4 - ((uintptr_t)src & 15) / 4) : 0);
+  const uint64_t h = head < n ? head : n;
+  if (blockIdx.x == 0 && threadIdx.x < h) hist32_key<IN_F32>(src[threadIdx.x], my, cd, cc);
+  const uint4* b4 = (const uint4*)(src + h);
+  const uint64_t m = n - h, quads = m / 4;
+  const uint64_t stride = (uint64_t)gridDim.x * kHist32Threads;
+  uint64_t i = (uint64_t)blockIdx.x * kHist32Threads + threadIdx.x;
+  for (; i + 3 * stride < quads; i += 4 * stride) {  // 4 independent 16-byte loads in flight
+    uint4 v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) v[u] = __ldcs(b4 + i + u * stride);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      hist32_key<IN_F32>(v[u].x, my, cd, cc);
+      hist32_key<IN_F32>(v[u].y, my, cd, cc);
+      hist32_key<IN_F32>(v[u].z, my, cd, cc);
+      hist32_key<IN_F32>(v[u].w, my, cd, cc);
+    }
+  }
+  for (; i < quads; i += stride) {
+    const uint4 v = __ldcs(b4 + i);
+    hist32_key<IN_F32>(v.x, my, cd, cc);
+    hist32_key<IN_F32>(v.y, my, cd, cc);
+    hist32_key<IN_F32>(v.z, my, cd, cc);
+    hist32_key<IN_F32>(v.w, my, cd, cc);
+  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (m & 3))
+    hist32_key<IN_F32>(src[h + quads * 4 + threadIdx.x], my, cd, cc);
+#pragma unroll
+  for (int q = 0; q < 2; ++q)
+    if (cc[q]) atomicAdd(&my[((2 + q) * kRadix + cd[q]) * kHist32Copies], cc[q]);
+  __syncthreads();
+  for (int j = threadIdx.x; j < 4 * kRadix; j += kHist32Threads) {
+    uint32_t c = 0;
+#pragma unroll
+    for (int q = 0; q < kHist32Copies; q += 4) {
+      const uint4 a = *(const uint4*)&sh[j * kHist32Copies + q];
+      c += a.x + a.y + a.z + a.w;
+    }
+    if (c) atomicAdd((unsigned long long*)&hist[j], (unsigned long long)c);
+  }
+}
+
+// final copy of a 32-bit sort (odd pass count in place, or every digit trivial): plan flags
+// copy_in_f64 / copy_out_f64 mean float32 bits here
+__global__ void k_final_copy32(uint32_t* in, uint32_t* out, uint32_t* tmp, uint64_t n,
+                               const RadixPlan* __restrict__ plan) {
+  const int cs = plan->copy_src;
+  if (cs < 0) return;
+  const uint32_t* s = pick(cs, in, out, tmp);
+  const bool fin = plan->copy_in_f64, fout = plan->copy_out_f64;
+  const uint32_t kx = (uint32_t)plan->key_xor;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t v = s[i];
+    if (fin != fout) v = fin ? to_key32(v) ^ kx : from_key32(v ^ kx);
+    out[i] = v;
+  }
 }
 
 }  // namespace
@@ -2000,6 +2125,64 @@ cudaError_t radix_sort_impl(RadixScratch& s, const uint64_t* in_c, uint64_t* out
 cudaError_t radix_sort(RadixScratch& s, const uint64_t* in_c, uint64_t* out, uint64_t* tmp,
                        uint64_t n, bool in_f64, bool out_f64, cudaStream_t st) {
   return radix_sort_impl(s, in_c, out, tmp, n, in_f64, out_f64, st, true);
+}
+
+cudaError_t radix_sort32(RadixScratch& s, const uint32_t* in_c, uint32_t* out, uint32_t* tmp,
+                         uint64_t n, bool in_f32, bool out_f32, bool desc, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  uint32_t* in = const_cast<uint32_t*>(in_c);
+  if (n > (1ull << 30) || ((((uintptr_t)in) | ((uintptr_t)out) | ((uintptr_t)tmp)) & 15) ||
+      pass_variant() != 2 || (desc && (!in_f32 || !out_f32)))
+    return cudaErrorNotSupported;  // the caller takes the 64-bit codec path
+  cudaError_t e = radix_scratch_reserve(s, n);
+  if (e != cudaSuccess) return e;
+  auto mark = [&](int i) -> cudaError_t {
+    return s.timing ? cudaEventRecord(s.ev[i], st) : cudaSuccess;
+  };
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if ((e = cudaMemsetAsync(s.small, 0, s.small_zero_bytes, st)) != cudaSuccess) return e;
+  if ((e = mark(0)) != cudaSuccess) return e;
+  {
+    const uint64_t want = (n / 4 + kHist32Threads * 4 - 1) / (kHist32Threads * 4);
+    const uint64_t cap = (uint64_t)num_sms(dev);
+    const unsigned grid = (unsigned)(want < 1 ? 1 : (want > cap ? cap : want));
+    constexpr int smem = 4 * kRadix * kHist32Copies * 4;
+    static bool attr[64] = {false};
+    if (dev >= 0 && dev < 64 && !attr[dev]) {
+      if ((e = cudaFuncSetAttribute(k_hist32<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      if ((e = cudaFuncSetAttribute(k_hist32<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+      attr[dev] = true;
+    }
+    if (in_f32) k_hist32<true><<<grid, kHist32Threads, smem, st>>>(in, n, s.hist);
+    else k_hist32<false><<<grid, kHist32Threads, smem, st>>>(in, n, s.hist);
+    if ((e = launched()) != cudaSuccess) return e;
+  }
+  if ((e = mark(1)) != cudaSuccess) return e;
+  if ((e = select_lb_mode(s, 2, n, st, false, true)) != cudaSuccess) return e;
+  k_scan_plan<<<1, 256, 0, st>>>(s.hist, s.bin_base, s.plan, n, in == out ? 1 : 0, in_f32 ? 1 : 0,
+                                 out_f32 ? 1 : 0, s.lb_state, 0, nullptr, desc ? 1 : 0);
+  if ((e = launched()) != cudaSuccess) return e;
+  if ((e = mark(2)) != cudaSuccess) return e;
+  constexpr int CT = HSORT_WS_CT, IT = HSORT_K32_ITEMS;
+  for (int p = 0; p < 4; ++p) {  // digits 4..7 of a 32-bit key are always trivial
+    uint64_t* i64 = (uint64_t*)in;
+    uint64_t* o64 = (uint64_t*)out;
+    uint64_t* t64 = (uint64_t*)tmp;
+    const bool f = p == 0 && in_f32;
+    e = desc ? launch_ws_pass<CT, IT, false, 0, true, true>(i64, o64, t64, nullptr, nullptr, nullptr, n, s,
+                                                           p, f, out_f32, st)
+             : launch_ws_pass<CT, IT, false, 0, false, true>(i64, o64, t64, nullptr, nullptr, nullptr, n,
+                                                            s, p, f, out_f32, st);
+    if (e != cudaSuccess) return e;
+    if ((e = mark(3 + p)) != cudaSuccess) return e;
+  }
+  for (int p = 4; p < kDigits; ++p)
+    if ((e = mark(3 + p)) != cudaSuccess) return e;
+  k_final_copy32<<<num_sms(dev) * 2, 512, 0, st>>>(in, out, tmp, n, s.plan);
+  if ((e = launched()) != cudaSuccess) return e;
+  if ((e = mark(11)) != cudaSuccess) return e;
+  return cudaMemcpyAsync(s.h_plan, s.plan, sizeof(RadixPlan), cudaMemcpyDeviceToHost, st);
 }
 
 cudaError_t radix_sort_desc_f64(RadixScratch& s, const uint64_t* in, uint64_t* out, uint64_t* tmp,

@@ -84,3 +84,37 @@ def test_device_f64_descending_fused(hs_gpu, oracle_mod, inputs_mod, dist, n):
     assert np.array_equal(out.cpu().numpy().view(np.uint64), want)
     if dist == "uniform":
         assert hs_gpu.hsort_get_last_plan()["elided"]
+
+
+@pytest.mark.parametrize("desc", [False, True])
+@pytest.mark.parametrize("dist", ["uniform", "special32", "all_equal", "few_distinct"])
+@pytest.mark.parametrize("n", [1, 3, 4, 7, 8641, 17_283, (1 << 22) + 3])
+def test_device_f32_native_in_place_and_launches(hs_gpu, oracle_mod, inputs_mod, desc, dist, n):
+    """The native 32-bit GPUSort (4-byte keys; K1 over 4 digits, <= 4 warp-specialised passes with
+    the binary32 transform fused into the first and last pass): 7 launches (K1, K2,
+    4 pass launches, final copy) instead of the codec path's encode/decode around a 64-bit sort;
+    in place (odd active-pass counts end with the final copy) and all-equal keys (no active
+    digit) included."""
+    import torch
+    A = _f32(inputs_mod, dist, n, seed=n % 1013)
+    want = oracle_mod.sort_f32(A, desc).view(np.uint32)
+    d = torch.from_numpy(A.view(np.int32).copy()).cuda().view(torch.float32)
+    out = torch.empty_like(d)
+    L0 = hs_gpu.hsort_get_launch_count()
+    hs_gpu.hsort_sort_device_typed(d, out, desc)
+    torch.cuda.synchronize()
+    assert hs_gpu.hsort_get_launch_count() - L0 == 7
+    assert np.array_equal(out.view(torch.int32).cpu().numpy().view(np.uint32), want)
+    assert hs_gpu.hsort_get_last_plan()["num_active"] <= 4
+    hs_gpu.hsort_sort_device_typed(d, d, desc)  # in place
+    torch.cuda.synchronize()
+    assert np.array_equal(d.view(torch.int32).cpu().numpy().view(np.uint32), want)
+
+
+def test_device_typed_requires_16_byte_alignment(hs_gpu):
+    """hsort_sort_device_typed's contract: 16-byte aligned device buffers (TMA tile loads)."""
+    import torch
+    buf = torch.zeros(1001, dtype=torch.float32, device="cuda")
+    with pytest.raises(hs_gpu.HsortError) as e:
+        hs_gpu.hsort_sort_device_typed(buf[1:], buf[1:].clone(), False)
+    assert e.value.code == -1

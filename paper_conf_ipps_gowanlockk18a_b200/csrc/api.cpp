@@ -1064,12 +1064,16 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
   std::vector<uint64_t> hoff(2 * (size_t)(k + 1));
   Acc acc;
   CK(cudaEventRecord(em.a, g.s_h2d));
-  for (uint64_t ch = 0; ch < nch; ++ch) {
+  // Chunk ch+1's HtoD + K4/K5 are enqueued before chunk ch's (possibly staged, blocking) DtoH, so
+  // the two link directions overlap (duplex); two slots per buffer.
+  std::vector<uint64_t> totals(nch, 0);
+  auto enqueue = [&](uint64_t ch) {
     const int s = (int)(ch & 1);
     const uint64_t* r0 = &cr[(size_t)ch * k];
     const uint64_t* r1 = &cr[(size_t)(ch + 1) * k];
     uint64_t* din = g.min.u64() + (uint64_t)s * C;
     uint64_t* ho = &hoff[(size_t)s * (k + 1)];
+    if (ch >= 2) CK(cudaEventSynchronize(in_ready[s]));  // chunk ch-2's offsets copy read ho
     ho[0] = 0;
     CK(cudaStreamWaitEvent(g.s_h2d, in_free[s], 0));
     for (int j = 0; j < k; ++j) {
@@ -1081,6 +1085,7 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
     CK(cudaMemcpyAsync(doff, ho, (k + 1) * 8, cudaMemcpyHostToDevice, g.s_h2d));
     CK(cudaEventRecord(in_ready[s], g.s_h2d));
     const uint64_t total = ho[k];
+    totals[ch] = total;
     const uint64_t tiles = (total + kMergeTile - 1) / kMergeTile;
     uint64_t* rk = g.ranks.u64() + (uint64_t)s * (tiles_c + 1) * k;
     uint64_t* dout = g.mout.u64() + (uint64_t)s * C;
@@ -1090,12 +1095,16 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
     CK(merge_tiles(din, nullptr, doff, k, total, rk, 0, 0, tiles, dout, 0, c.f64, g.s_comp));
     CK(cudaEventRecord(in_free[s], g.s_comp));
     CK(cudaEventRecord(merged[s], g.s_comp));
+  };
+  if (nch) enqueue(0);
+  for (uint64_t ch = 0; ch < nch; ++ch) {
+    const int s = (int)(ch & 1);
+    if (ch + 1 < nch) enqueue(ch + 1);
     CK(cudaStreamWaitEvent(g.s_d2h, merged[s], 0));
     const uint64_t p0 = o_lo + ch * C;
-    download(g, (uint64_t*)c.B + p0, dout, total * 8, g.s_d2h, c.direct_out, c.mc_threads, acc);
+    download(g, (uint64_t*)c.B + p0, g.mout.u64() + (uint64_t)s * C, totals[ch] * 8, g.s_d2h,
+             c.direct_out, c.mc_threads, acc);
     CK(cudaEventRecord(out_free[s], g.s_d2h));
-    // the pageable host offsets of the other slot are rewritten next iteration: its copy must be done
-    if (ch + 1 < nch) CK(cudaEventSynchronize(in_ready[s ^ 1]));
   }
   CK(cudaEventRecord(em.b, g.s_d2h));
   CK(cudaStreamSynchronize(g.s_d2h));

@@ -434,6 +434,37 @@ def skewed_rows(hs, torch, A_h, B_h, d_in, d_out, stream, peak, n):
     return rows
 
 
+def pairs_e2e(hs, torch, A_h, B_h, n):
+    """Key/value host->host (S§8(f) #3, the [5] workload of keys with 64-bit values): 2^30
+    (uniform key, index) pairs through hsort_sort_pairs on pinned buffers -- the RESIDENT
+    key/value plan (stable batch sorts in HBM + the key/value merge); 32 B/pair cross the link."""
+    import hsort_inputs
+    hsort_inputs.generate("uniform", n, seed=SEED, out=A_h.numpy())
+    V = torch.arange(n, dtype=torch.int64).pin_memory()
+    VB = torch.empty(n, dtype=torch.int64, pin_memory=True)
+    Vn, VBn = V.numpy().view(np.uint64), VB.numpy().view(np.uint64)
+    hs.hsort_sort_pairs(A_h.numpy(), Vn, B_h.numpy(), VBn)  # warm
+    ts = []
+    for _ in range(3):
+        t = time.perf_counter()
+        hs.hsort_sort_pairs(A_h.numpy(), Vn, B_h.numpy(), VBn)
+        ts.append(time.perf_counter() - t)
+    st = hs.hsort_get_stats()
+    Bv = B_h.numpy()
+    assert is_sorted(Bv), "pairs: keys not sorted"
+    assert multiset_sig(A_h.numpy()) == multiset_sig(Bv), "pairs: keys not a permutation"
+    # values: the stable argsort of A; spot-check the pairing on a sample (full pairing is pinned
+    # against the oracle in tests/test_gpu_pairs.py)
+    idx = np.random.default_rng(0).integers(0, n, size=1 << 16)
+    assert np.array_equal(A_h.numpy()[VBn[idx].astype(np.int64)].view(np.uint64), Bv[idx].view(np.uint64))
+    dt = statistics.median(ts)
+    del V, VB
+    return {"what": "hsort_sort_pairs(A, V = 0..n-1, B, VB) pinned, 2^30 pairs, RESIDENT key/value plan",
+            "pairs_per_s": n / dt, "ms": 1e3 * dt, "mode": st["mode_name"], "n_b": st["n_b"],
+            "t_h2d_s": st["t_h2d"], "t_d2h_s": st["t_d2h"], "t_gpu_sort_s": st["t_gpu_sort"],
+            "t_merge_gpu_s": st["t_merge_gpu"], "link_bytes_per_pair": 32}
+
+
 def out_of_core(hs, torch, bw, host_bw):
     """The paper's out-of-core workflow (STREAM: batches -> HtoD -> GPUSort -> DtoH -> W, then the
     CPU/GPU merge split W -> B, configs C3/C5) at the largest n this host fits with
@@ -730,6 +761,7 @@ def main():
                                  avg_pass_ms, stream)
         line["stages"] = stages
         line["skewed"] = skewed_rows(hs, torch, A_h, B_h, d_in, d_out, stream, peak, n_gpu)
+        line["pairs_e2e"] = pairs_e2e(hs, torch, A_h, B_h, n_gpu)
     del d_in, d_out
     torch.cuda.empty_cache()
     host_bw = None

@@ -158,9 +158,10 @@ int hsort_sort_typed(const void* A_host, void* B_host, uint64_t n, int key_type,
  * Key/value sort (the [5] workload of 64-bit keys with 64-bit values,
  * P:743-761).  B/VB = the pairs (A[i], V[i]) ordered by A under IEEE totalOrder, STABLY: pairs
  * with equal keys keep their input order, so the result is unique (V = 0..n-1 gives the stable
- * argsort).  Values are opaque 64-bit payloads, never transformed.  One GPU, one batch (BLINE):
- * 1 <= n <= 2^30 pairs and 32 B/pair + 0.5 B/pair of HBM; larger n -> HSORT_ERR_INVALID (a merge
- * that carries values is not built).  B == A and VB == V allowed together or separately; any
+ * argsort).  Values are opaque 64-bit payloads, never transformed.  n < 2^24 (option
+ * "auto_pipeline_min"): one GPU, one batch (BLINE; 32.5 B/pair of HBM); larger n: the RESIDENT
+ * key/value plan of hsort_sort_pairs_ex on GPU 0 (runs in HBM, key/value merge; n beyond one GPU's
+ * HBM -> HSORT_ERR_INVALID).  B == A and VB == V allowed together or separately; any
  * other overlap among A, V, B, VB -> HSORT_ERR_INVALID.  Synchronous; retains no pointer.
  * ------------------------------------------------------------------------------------------- */
 int hsort_sort_pairs(const double* A_host, const uint64_t* V_host, double* B_host, uint64_t* VB_host,
@@ -168,6 +169,16 @@ int hsort_sort_pairs(const double* A_host, const uint64_t* V_host, double* B_hos
 /* Same with raw uint64 keys (ascending unsigned). */
 int hsort_sort_pairs_u64(const uint64_t* A_host, const uint64_t* V_host, uint64_t* B_host,
                          uint64_t* VB_host, uint64_t n);
+/* Key/value sort with the batch size and GPU count of hsort_sort (keys_f64: 1 float64 keys under
+ * totalOrder, 0 raw uint64 keys).  batch_elems = 0 and n < option "auto_pipeline_min" (2^24):
+ * one batch on one GPU as above; otherwise (or batch_elems < n, n_gpus > 1, n > 2^30) the RESIDENT
+ * plan: GPU g stably sorts the batches of its shard of the pairs in HBM (key/value GPUSort) and
+ * merges one range of B/VB from all GPUs' runs (K4 on the keys, the key/value K5, equal keys in run
+ * order), so the result is the same unique stable sort.  The runs must fit in HBM (16 B/pair per
+ * shard + one batch of scratch), else HSORT_ERR_INVALID; a streamed (W) key/value merge is not
+ * built.  Aliasing and errors as hsort_sort_pairs. */
+int hsort_sort_pairs_ex(const void* A_host, const uint64_t* V_host, void* B_host, uint64_t* VB_host,
+                        uint64_t n, uint64_t batch_elems, int n_gpus, int keys_f64);
 
 /* ---------------------------------------------------------------------------------------------
  * Options, statistics, errors

@@ -80,6 +80,7 @@ SIGNATURES = {
     "hsort_sort_device_typed": ([_P, _P, _U64, _I, _I, _P], _I),
     "hsort_sort_pairs": ([_P, _P, _P, _P, _U64], _I),
     "hsort_sort_pairs_u64": ([_P, _P, _P, _P, _U64], _I),
+    "hsort_sort_pairs_ex": ([_P, _P, _P, _P, _U64, _U64, _I, _I], _I),
     "hsort_sort_device_pairs": ([_P, _P, _P, _P, _U64, _I, _P], _I),
     "hsort_set_option": ([ctypes.c_char_p, ctypes.c_int64], _I),
     "hsort_get_option": ([ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64)], _I),
@@ -269,6 +270,25 @@ def hsort_sort_pairs_u64(A, V, B=None, VB=None):
     if not (n == nv == nb == nvb):
         raise ValueError("A, V, B, VB must have the same length")
     _check(lib().hsort_sort_pairs_u64(a, v, b, vb, n))
+    return B, VB
+
+
+def hsort_sort_pairs_ex(A, V, B=None, VB=None, batch_elems: int = 0, n_gpus: int = 1):
+    """Key/value sort with hsort_sort's batch size and GPU count (RESIDENT key/value plan: stable
+    batch sorts in HBM + the key/value K4/K5 merge).  A float64 or uint64, V uint64 payloads."""
+    f64 = A.dtype == np.float64 if isinstance(A, np.ndarray) else A.dtype.is_floating_point
+    dt = np.float64 if f64 else np.uint64
+    a, n = _host_ptr(A, dt)
+    v, nv = _host_ptr(V, np.uint64)
+    if B is None:
+        B = np.empty(n, dtype=dt)
+    if VB is None:
+        VB = np.empty(n, dtype=np.uint64)
+    b, nb = _host_ptr(B, dt)
+    vb, nvb = _host_ptr(VB, np.uint64)
+    if not (n == nv == nb == nvb):
+        raise ValueError("A, V, B, VB must have the same length")
+    _check(lib().hsort_sort_pairs_ex(a, v, b, vb, n, batch_elems, n_gpus, int(f64)))
     return B, VB
 
 

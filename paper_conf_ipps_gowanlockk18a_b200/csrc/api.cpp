@@ -157,6 +157,7 @@ struct GpuCtx {
   DevBuf part, bcnt, btot, bspl, bseg;  // MSD-first split: partitioned batches, tile counts,
                                         // batch bucket totals, splitters, gather segment table
   DevBuf vruns, valt;  // key/value sorts: values and their ping-pong scratch
+  DevBuf vmout, vrptr; // key/value merge: merged value chunks, value run-pointer table
   DevBuf tmp3;         // typed sorts: third key buffer, so the GPUSort runs out of place (elision)
   std::vector<char*> ring_in, ring_out;
   uint64_t ring_bytes = 0;
@@ -542,6 +543,10 @@ struct CallCtx {
   bool direct_in, direct_out;
   int mc_threads, merge_threads;
   hsort_stats* st;
+  // key/value calls (S§8(f) #3): the values V (host, n) and VB; nullptr for keys-only calls
+  const uint64_t* V = nullptr;
+  uint64_t* VB = nullptr;
+  bool direct_vin = false, direct_vout = false;
 };
 
 void sort_bline(GpuCtx& g, CallCtx& c) {
@@ -646,7 +651,9 @@ void corank_on(GpuCtx& g, const uint64_t* keys, const uint64_t* const* rp, const
 // into K4/K5's loads.
 void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_keys, const uint64_t* const* d_rp,
                        const uint64_t* d_off, int k, uint64_t total, uint64_t o_lo, uint64_t o_hi,
-                       PhaseTimes& pt) {
+                       PhaseTimes& pt, const uint64_t* d_vkeys = nullptr,
+                       const uint64_t* const* d_vrp = nullptr) {
+  const bool kv = c.VB != nullptr;
   if (o_hi <= o_lo) return;
   Nvtx nv("GPU merge -> B");
   const uint64_t t_lo = o_lo / kMergeTile;
@@ -657,6 +664,7 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_keys, const uint
   const uint64_t nch = (tiles + ctiles - 1) / ctiles;
   const uint64_t slots = nch > 1 ? 2 : 1;
   g.mout.reserve(slots * chunk * 8);
+  if (kv) g.vmout.reserve(slots * chunk * 8);
   g.ranks.reserve(slots * (ctiles + 1) * (uint64_t)k * 8);
   std::vector<cudaEvent_t> ev_done(slots), ev_free(slots);
   std::vector<EvPair> em(nch), ed(nch);
@@ -678,7 +686,8 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_keys, const uint
     CK(cudaEventRecord(em[ch].a, g.s_comp));
     corank_on(g, d_keys, d_rp, d_off, k, total, kMergeTile, tb, tc + 1, rk, g.s_comp);
     CK(merge_tiles(d_keys, d_rp, d_off, k, total, rk, tb, tb, tc, g.mout.u64() + s * chunk,
-                   tb * kMergeTile, c.f64, g.s_comp));
+                   tb * kMergeTile, c.f64, g.s_comp, d_vkeys, d_vrp,
+                   kv ? g.vmout.u64() + s * chunk : nullptr));
     CK(cudaEventRecord(em[ch].b, g.s_comp));
     CK(cudaEventRecord(ev_done[s], g.s_comp));
   };
@@ -691,6 +700,9 @@ void gpu_merge_to_host(GpuCtx& g, CallCtx& c, const uint64_t* d_keys, const uint
     CK(cudaEventRecord(ed[ch].a, g.s_d2h));
     download(g, B + o * 8, g.mout.u64() + s * chunk, len * 8, g.s_d2h, c.direct_out, c.mc_threads,
              pt.acc);
+    if (kv)
+      download(g, c.VB + o, g.vmout.u64() + s * chunk, len * 8, g.s_d2h, c.direct_vout, c.mc_threads,
+               pt.acc);
     CK(cudaEventRecord(ed[ch].b, g.s_d2h));
     CK(cudaEventRecord(ev_free[s], g.s_d2h));
   }
@@ -719,8 +731,13 @@ void resident_sort_phase(GpuCtx& g, CallCtx& c, uint64_t a0, const std::vector<u
   Nvtx nv("sort phase (resident)");
   uint64_t bmax = 0;
   for (uint64_t i = 0; i < nb; ++i) bmax = std::max(bmax, h_off[i + 1] - h_off[i]);
+  const bool kv = c.V != nullptr;
   g.runs.reserve(shard * 8);
   g.alt.reserve(bmax * 8);
+  if (kv) {
+    g.vruns.reserve(shard * 8);
+    g.valt.reserve(bmax * 8);
+  }
   std::vector<EvPair> eh(nb), es(nb);
   for (auto& e : eh) e.make();
   for (auto& e : es) e.make();
@@ -729,10 +746,16 @@ void resident_sort_phase(GpuCtx& g, CallCtx& c, uint64_t a0, const std::vector<u
     CK(cudaEventRecord(eh[i].a, g.s_h2d));
     upload(g, g.runs.u64() + o, (const char*)c.A + (a0 + o) * 8, len * 8, g.s_h2d, c.direct_in,
            c.mc_threads, pt.acc);
+    if (kv)
+      upload(g, g.vruns.u64() + o, c.V + a0 + o, len * 8, g.s_h2d, c.direct_vin, c.mc_threads, pt.acc);
     CK(cudaEventRecord(eh[i].b, g.s_h2d));
     CK(cudaStreamWaitEvent(g.s_comp, eh[i].b, 0));
     CK(cudaEventRecord(es[i].a, g.s_comp));
-    CK(radix_sort(g.rs, g.runs.u64() + o, g.runs.u64() + o, g.alt.u64(), len, c.f64, false, g.s_comp));
+    if (kv)  // stable key/value GPUSort of the batch, in place; keys stay transformed for the merge
+      CK(radix_sort_pairs(g.rs, g.runs.u64() + o, g.vruns.u64() + o, g.runs.u64() + o,
+                          g.vruns.u64() + o, g.alt.u64(), g.valt.u64(), len, c.f64, false, g.s_comp));
+    else
+      CK(radix_sort(g.rs, g.runs.u64() + o, g.runs.u64() + o, g.alt.u64(), len, c.f64, false, g.s_comp));
     CK(cudaEventRecord(es[i].b, g.s_comp));
   }
   CK(cudaStreamSynchronize(g.s_comp));
@@ -768,11 +791,12 @@ void sort_resident(std::vector<GpuCtx*>& gs, CallCtx& c) {
   run_per_gpu(N, [&](size_t g) { resident_sort_phase(*gs[g], c, shard[g], h_off[g], pt[g]); });
   c.st->t_sort_phase = secs_since(t0);
   // the global run table (run order: GPU-major, then batch): device pointers and offsets
-  std::vector<const uint64_t*> rp;
+  std::vector<const uint64_t*> rp, vrp;
   std::vector<uint64_t> goff{0};
   for (size_t g = 0; g < N; ++g)
     for (size_t i = 0; i + 1 < h_off[g].size(); ++i) {
       rp.push_back(gs[g]->runs.u64() + h_off[g][i]);
+      if (c.V) vrp.push_back(gs[g]->vruns.u64() + h_off[g][i]);
       goff.push_back(goff.back() + h_off[g][i + 1] - h_off[g][i]);
     }
   const int k = (int)rp.size();
@@ -784,12 +808,19 @@ void sort_resident(std::vector<GpuCtx*>& gs, CallCtx& c) {
     g.off.reserve((k + 1) * 8);
     CK(cudaMemcpyAsync(g.off.p, goff.data(), (k + 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
     if (N == 1) {
-      gpu_merge_to_host(g, c, g.runs.u64(), nullptr, g.off.u64(), k, n, 0, n, pt[gi]);
+      gpu_merge_to_host(g, c, g.runs.u64(), nullptr, g.off.u64(), k, n, 0, n, pt[gi],
+                        c.V ? g.vruns.u64() : nullptr, nullptr);
     } else {
       g.rptr.reserve(k * sizeof(void*));
       CK(cudaMemcpyAsync(g.rptr.p, rp.data(), k * sizeof(void*), cudaMemcpyHostToDevice, g.s_comp));
+      const uint64_t* const* d_vrp = nullptr;
+      if (c.V) {
+        g.vrptr.reserve(k * sizeof(void*));
+        CK(cudaMemcpyAsync(g.vrptr.p, vrp.data(), k * sizeof(void*), cudaMemcpyHostToDevice, g.s_comp));
+        d_vrp = (const uint64_t* const*)g.vrptr.p;
+      }
       gpu_merge_to_host(g, c, nullptr, (const uint64_t* const*)g.rptr.p, g.off.u64(), k, n,
-                        orng[gi], orng[gi + 1], pt[gi]);
+                        orng[gi], orng[gi + 1], pt[gi], nullptr, d_vrp);
     }
   });
   c.st->t_merge_phase = secs_since(t1);
@@ -1513,6 +1544,8 @@ void ctx_destroy(GpuCtx& g) {
   g.tmp3.release();
   g.vruns.release();
   g.valt.release();
+  g.vmout.release();
+  g.vrptr.release();
   g.mout.release();
   g.min.release();
   g.ranks.release();
@@ -1693,7 +1726,8 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
 // Key/value host->host sort (S§8(f) #3, the [5] workload of P:743-761): BLINE on one GPU --
 // HtoD of keys and values, the key/value GPUSort in place, DtoH of both.  Out-of-core pairs (a
 // merge that carries values) are not built: n must fit one GPU (32 B/pair + look-back).
-int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint64_t n, bool f64) {
+int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint64_t n, bool f64,
+                  uint64_t batch_elems = 0, int n_gpus = 1) {
   int rc = check_ready();
   if (rc) return rc;
   BusyGuard busy;
@@ -1724,9 +1758,89 @@ int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint6
     g_err = "key and value arrays must not overlap (B == A and VB == V are allowed)";
     return HSORT_ERR_INVALID;
   }
-  if (n > (1ull << 30)) {
-    g_err = "key/value sort: n <= 2^30 pairs (one GPU, no out-of-core merge of pairs)";
+  const int vis = (int)S().gpus.size();
+  if (n_gpus < 0 || n_gpus > vis) {
+    g_err = "n_gpus must be in [0, " + std::to_string(vis) + "]";
     return HSORT_ERR_INVALID;
+  }
+  if (n_gpus == 0) n_gpus = vis;
+  if (!S().peer_ok) n_gpus = 1;
+  const uint64_t auto_min = (uint64_t)std::max<int64_t>(0, S().opt.get("auto_pipeline_min"));
+  const bool batched = (batch_elems > 0 && batch_elems < n) || n_gpus > 1 || n > (1ull << 30) ||
+                       (batch_elems == 0 && auto_min && n >= auto_min);
+  if (batched) {
+    // RESIDENT key/value plan over n_gpus GPUs (S§8(f) #3 widened out of core): every batch of a
+    // GPU's shard is sorted stably in HBM, then each GPU merges one range of B/VB from all runs
+    // with K4 + the key/value K5 (ties in run order = input order, so the result is the unique
+    // stable sort).  The runs must fit in HBM (16 B/pair); a streamed pair merge is not built.
+    return guarded([&]() -> int {
+      Nvtx nv("hsort_sort_pairs (resident)");
+      auto t0 = Clock::now();
+      const int N = n_gpus;
+      const std::vector<uint64_t> sh = shard_bounds(n, N, kRadixTile);
+      uint64_t smax = 0;
+      for (int g = 0; g < N; ++g) smax = std::max(smax, sh[g + 1] - sh[g]);
+      uint64_t b;
+      int schedule;
+      if (batch_elems > 0 && batch_elems < n) {
+        b = std::min<uint64_t>(batch_elems, 1ull << 30);
+        b += b & 1;  // 16-byte aligned batch starts (TMA tile loads of the pair sort)
+        schedule = 0;
+      } else {
+        b = std::min<uint64_t>(1ull << 27, std::max<uint64_t>(smax / 8, kRadixTile));
+        b -= b % kRadixTile;
+        schedule = 1;
+      }
+      const uint64_t runs = resident_runs(n, N, b, schedule, nullptr);
+      if (runs > (uint64_t)kMaxMergeRuns)
+        throw HsortError(HSORT_ERR_INVALID, "key/value sort: more than 1024 runs; use larger batches");
+      const uint64_t need = smax * 16 + b * (16 + (uint64_t)kLookbackBytesPerKey + 1) +
+                            4 * (uint64_t)S().opt.get("merge_chunk") * 8 +
+                            ((uint64_t)S().opt.get("device_reserve_mb") << 20);
+      if (need > device_budget(N))
+        throw HsortError(HSORT_ERR_INVALID,
+                         "key/value sort: the runs do not fit in HBM (16 B/pair per GPU shard); "
+                         "a streamed key/value merge is not built");
+      hsort_stats st{};
+      st.n = n;
+      st.b_s = b;
+      st.n_b = runs;
+      st.n_gpus = N;
+      st.n_s = 1;
+      st.mode = HSORT_MODE_RESIDENT;
+      st.merge_k = (int)runs;
+      st.t_init = S().t_init;
+      CallCtx c;
+      c.A = A;
+      c.B = B;
+      c.n = n;
+      c.f64 = f64;
+      c.plan = hsort_plan_t{};
+      c.plan.n = n;
+      c.plan.b_s = b;
+      c.plan.n_b = runs;
+      c.plan.n_gpus = N;
+      c.plan.schedule = schedule;
+      c.plan.mode = HSORT_MODE_RESIDENT;
+      c.direct_in = is_pinned(A, bytes);
+      c.direct_out = is_pinned(B, bytes);
+      c.V = V;
+      c.VB = VB;
+      c.direct_vin = is_pinned(V, bytes);
+      c.direct_vout = is_pinned(VB, bytes);
+      c.mc_threads = (int)S().opt.get("memcpy_threads");
+      c.merge_threads = (int)S().opt.get("merge_threads");
+      c.st = &st;
+      st.direct_in = c.direct_in && c.direct_vin;
+      st.direct_out = c.direct_out && c.direct_vout;
+      st.t_setup = secs_since(t0);
+      std::vector<GpuCtx*> gs;
+      for (int i = 0; i < N; ++i) gs.push_back(&S().gpus[i]);
+      sort_resident(gs, c);
+      st.t_total = secs_since(t0);
+      S().last = st;
+      return HSORT_OK;
+    });
   }
   return guarded([&]() -> int {
     auto t0 = Clock::now();
@@ -1999,6 +2113,11 @@ int hsort_sort_pairs(const double* A_host, const uint64_t* V_host, double* B_hos
 int hsort_sort_pairs_u64(const uint64_t* A_host, const uint64_t* V_host, uint64_t* B_host,
                          uint64_t* VB_host, uint64_t n) {
   return do_sort_pairs(A_host, V_host, B_host, VB_host, n, false);
+}
+
+int hsort_sort_pairs_ex(const void* A_host, const uint64_t* V_host, void* B_host, uint64_t* VB_host,
+                        uint64_t n, uint64_t batch_elems, int n_gpus, int keys_f64) {
+  return do_sort_pairs(A_host, V_host, B_host, VB_host, n, keys_f64 != 0, batch_elems, n_gpus);
 }
 
 int hsort_set_option(const char* key, int64_t value) {

@@ -155,10 +155,14 @@ cudaError_t merge_corank(const uint64_t* keys, const uint64_t* const* rp, const 
 // K5: merge tiles [tile_begin, tile_begin + tile_count) (tile t = output [t*kMergeTile, ...)),
 // given co-ranks of boundaries t = rank_tile0, rank_tile0 + 1, ... (row t - rank_tile0 of
 // `ranks`, step kMergeTile); writes out[o - out_origin].
+// With vout != nullptr the runs carry 64-bit values (vkeys + d_off[j] or vrp[j], same offsets),
+// moved with their keys into vout (key/value merge: stable given stably sorted runs).
 cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
                         int k, uint64_t total, const uint64_t* ranks, uint64_t rank_tile0,
                         uint64_t tile_begin, uint64_t tile_count, uint64_t* out,
-                        uint64_t out_origin, bool out_f64, cudaStream_t st);
+                        uint64_t out_origin, bool out_f64, cudaStream_t st,
+                        const uint64_t* vkeys = nullptr, const uint64_t* const* vrp = nullptr,
+                        uint64_t* vout = nullptr);
 
 // ---- MSD-first split (msd.cu, S§8(f) #2) ---------------------------------------------------------
 constexpr int kMaxBuckets = 1024;

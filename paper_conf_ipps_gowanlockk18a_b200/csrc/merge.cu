@@ -312,20 +312,28 @@ __device__ __forceinline__ int advance_run(const uint32_t* bnd, int a, int cnt, 
   return a;
 }
 
-template <int T>
+// KV (S§8(f) #3, the out-of-core key/value sort): every key carries a 64-bit value; values sit in
+// their own shared buffers and move with their keys (the merge compares keys only, ties in run
+// order, so the merge of stably sorted runs is the stable sort of the pairs).
+template <int T, bool KV = false>
 __global__ void __launch_bounds__(T) k_merge_tile(
     const uint64_t* __restrict__ keys, const uint64_t* const* __restrict__ rp,
     const uint64_t* __restrict__ off, int k, uint64_t total,
     const uint64_t* __restrict__ ranks, uint64_t rank_tile0, uint64_t tile_begin,
-    uint64_t* __restrict__ out, uint64_t out_origin, int out_f64) {
+    uint64_t* __restrict__ out, uint64_t out_origin, int out_f64,
+    const uint64_t* __restrict__ vkeys = nullptr, const uint64_t* const* __restrict__ vrp = nullptr,
+    uint64_t* __restrict__ vout = nullptr) {
   using Cfg = MergeCfg<T>;
   constexpr int IPT = Cfg::IPT;
   extern __shared__ __align__(16) unsigned char smem[];
   uint64_t* buf0 = (uint64_t*)smem;
   uint64_t* buf1 = buf0 + Cfg::BUF;
+  uint64_t* vbuf0 = buf1 + Cfg::BUF;                   // KV only
+  uint64_t* vbuf1 = vbuf0 + Cfg::BUF;
   // [k] address of slice j's first key minus bnd[j] keys (slices may sit in peer GPUs' HBM)
-  const uint64_t** s_src = (const uint64_t**)(buf1 + Cfg::BUF);
-  uint32_t* bnd = (uint32_t*)(s_src + k);       // [k + 1] tile-local slice starts
+  const uint64_t** s_src = (const uint64_t**)(buf1 + Cfg::BUF * (KV ? 3 : 1));
+  const uint64_t** s_vsrc = s_src + k;                 // KV only: the values' slices
+  uint32_t* bnd = (uint32_t*)(s_src + k * (KV ? 2 : 1));  // [k + 1] tile-local slice starts
   __shared__ uint32_t s_w[T / 32];
 
   const uint64_t t = tile_begin + blockIdx.x;
@@ -343,10 +351,12 @@ __global__ void __launch_bounds__(T) k_merge_tile(
     const int j = c0 + tid;
     uint32_t len = 0;
     const uint64_t* srcj = nullptr;
+    const uint64_t* vsrcj = nullptr;
     if (j < k) {
       const uint64_t a = r0[j];
       len = (uint32_t)(r1[j] - a);
       srcj = (rp ? rp[j] : keys + off[j]) + a;
+      if (KV) vsrcj = (vrp ? vrp[j] : vkeys + off[j]) + a;
     }
     uint32_t x = len;
 #pragma unroll
@@ -358,6 +368,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
       if (j < k) {
         bnd[j] = x - len;
         s_src[j] = srcj - (x - len);
+        if (KV) s_vsrc[j] = vsrcj - (x - len);
       }
       break;
     }
@@ -374,6 +385,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
       const uint32_t bj = carry + pre + x - len;
       bnd[j] = bj;
       s_src[j] = srcj - bj;
+      if (KV) s_vsrc[j] = vsrcj - bj;
     }
     carry += tot;
     __syncthreads();
@@ -388,6 +400,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   //    advances it (usually zero steps: slices are longer than 32 keys).
   constexpr int C = 32 * IPT;
   uint64_t v[IPT];
+  uint64_t vv[KV ? IPT : 1];
   {
     const int e0 = w * C + lane;
     int a = (k > 1 && e0 < L) ? advance_run(bnd, 0, k, (uint32_t)e0) : 0;
@@ -397,21 +410,29 @@ __global__ void __launch_bounds__(T) k_merge_tile(
       if (e < L) {
         while (a + 1 < k && bnd[a + 1] <= (uint32_t)e) ++a;
         v[q] = ld_stream_u64(s_src[a] + e);
+        if (KV) vv[q] = ld_stream_u64(s_vsrc[a] + e);
       }
     }
   }
+  uint64_t* vo = KV ? vout + (o0 - out_origin) : nullptr;
   if (k == 1) {
 #pragma unroll
     for (int q = 0; q < IPT; ++q) {
       const int e = w * C + lane + 32 * q;
-      if (e < L) o[e] = out_f64 ? from_key(v[q]) : v[q];
+      if (e < L) {
+        o[e] = out_f64 ? from_key(v[q]) : v[q];
+        if (KV) vo[e] = vv[q];
+      }
     }
     return;
   }
 #pragma unroll
   for (int q = 0; q < IPT; ++q) {
     const int e = w * C + lane + 32 * q;
-    if (e < L) buf0[Cfg::pp(e)] = v[q];
+    if (e < L) {
+      buf0[Cfg::pp(e)] = v[q];
+      if (KV) vbuf0[Cfg::pp(e)] = vv[q];
+    }
   }
   const int p0 = tid * IPT;
   const int pend = p0 + IPT < L ? p0 + IPT : L;
@@ -421,6 +442,8 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   // 3. pairwise merge-path rounds
   uint64_t* src = buf0;
   uint64_t* dst = buf1;
+  uint64_t* vsrc = vbuf0;
+  uint64_t* vdst = vbuf1;
   for (int sh = 0; (1 << sh) < k; ++sh) {
     int p = p0;
     int m = j0 >> (sh + 1);
@@ -451,10 +474,12 @@ __global__ void __launch_bounds__(T) k_merge_tile(
         // whole output range inside one pair (the common case): fully unrolled, output slots at
         // constant offsets from pp(p0) (p0 = IPT tid: no pad inside a thread's range)
         uint64_t* d = dst + Cfg::pp(p);
+        uint64_t* dv = vdst + Cfg::pp(p);
 #pragma unroll
         for (int q = 0; q < IPT; ++q) {
           const bool ta = jb >= lenB || (i < lenA && a <= b);
           d[q] = ta ? a : b;
+          if (KV) dv[q] = vsrc[Cfg::pp(ta ? s0 + i : s1 + jb)];
           i += ta;
           jb += !ta;
           int nx = ta ? s0 + i : s1 + jb;
@@ -469,6 +494,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
         const bool ta = jb >= lenB || (i < lenA && a <= b);
         const uint64_t x = ta ? a : b;
         dst[Cfg::pp(p)] = x;
+        if (KV) vdst[Cfg::pp(p)] = vsrc[Cfg::pp(ta ? s0 + i : s1 + jb)];
         i += ta;
         jb += !ta;
         int nx = ta ? s0 + i : s1 + jb;
@@ -483,6 +509,9 @@ __global__ void __launch_bounds__(T) k_merge_tile(
     uint64_t* tsw = src;
     src = dst;
     dst = tsw;
+    tsw = vsrc;
+    vsrc = vdst;
+    vdst = tsw;
   }
 
   // 4. coalesced store of the tile (src holds the merged, transformed keys)
@@ -497,6 +526,13 @@ __global__ void __launch_bounds__(T) k_merge_tile(
     for (int q = 0; q < IPT; ++q) {
       const int p = q * T + tid;
       if (p < L) __stcs(o + p, src[Cfg::pp(p)]);
+    }
+  }
+  if (KV) {
+#pragma unroll
+    for (int q = 0; q < IPT; ++q) {
+      const int p = q * T + tid;
+      if (p < L) __stcs(vo + p, vsrc[Cfg::pp(p)]);
     }
   }
 }
@@ -515,8 +551,9 @@ __global__ void k_upper_bounds(const uint64_t* __restrict__ keys, uint64_t n,
 #endif
 constexpr int kMergeThreads = HSORT_MERGE_THREADS;
 
-size_t merge_smem_bytes(int k) {
-  return 2 * MergeCfg<kMergeThreads>::BUF * sizeof(uint64_t) + (size_t)k * sizeof(void*) +
+size_t merge_smem_bytes(int k, bool kv = false) {
+  return (kv ? 4 : 2) * MergeCfg<kMergeThreads>::BUF * sizeof(uint64_t) +
+         (size_t)k * sizeof(void*) * (kv ? 2 : 1) +
          ((size_t)k + 1) * sizeof(uint32_t);
 }
 
@@ -623,21 +660,32 @@ cudaError_t merge_tiles(const uint64_t* keys, const uint64_t* const* rp, const u
                         int k, uint64_t total,
                         const uint64_t* ranks, uint64_t rank_tile0, uint64_t tile_begin,
                         uint64_t tile_count, uint64_t* out, uint64_t out_origin, bool out_f64,
-                        cudaStream_t st) {
+                        cudaStream_t st, const uint64_t* vkeys, const uint64_t* const* vrp,
+                        uint64_t* vout) {
   if (tile_count == 0) return cudaSuccess;
   static bool attr_set[64] = {false};
+  static bool attr_kv[64] = {false};
   int dev = 0;
   cudaGetDevice(&dev);
-  const size_t smem = merge_smem_bytes(k);
-  if (dev >= 0 && dev < 64 && !attr_set[dev]) {
-    cudaError_t e = cudaFuncSetAttribute(k_merge_tile<kMergeThreads>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)merge_smem_bytes(kMaxMergeRuns));
+  const bool kv = vout != nullptr;
+  const size_t smem = merge_smem_bytes(k, kv);
+  if (dev >= 0 && dev < 64 && !(kv ? attr_kv : attr_set)[dev]) {
+    cudaError_t e = kv ? cudaFuncSetAttribute(k_merge_tile<kMergeThreads, true>,
+                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)merge_smem_bytes(kMaxMergeRuns, true))
+                       : cudaFuncSetAttribute(k_merge_tile<kMergeThreads>,
+                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)merge_smem_bytes(kMaxMergeRuns));
     if (e != cudaSuccess) return e;
-    attr_set[dev] = true;
+    (kv ? attr_kv : attr_set)[dev] = true;
   }
-  k_merge_tile<kMergeThreads><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(keys, rp, d_off, k, total, ranks,
-                                                                  rank_tile0, tile_begin, out,
-                                                                  out_origin, out_f64 ? 1 : 0);
+  if (kv)
+    k_merge_tile<kMergeThreads, true><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(
+        keys, rp, d_off, k, total, ranks, rank_tile0, tile_begin, out, out_origin, out_f64 ? 1 : 0,
+        vkeys, vrp, vout);
+  else
+    k_merge_tile<kMergeThreads><<<(unsigned)tile_count, kMergeThreads, smem, st>>>(
+        keys, rp, d_off, k, total, ranks, rank_tile0, tile_begin, out, out_origin, out_f64 ? 1 : 0);
   return launched();
 }
 

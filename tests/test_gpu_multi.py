@@ -199,3 +199,18 @@ def test_msd_split_tiny(hv, oracle_mod, inputs_mod, n, b):
     want = _bits(oracle_mod.sort_f64(A))
     B = _with(hv, {"msd": 1}, lambda: hv.hsort_sort(A, batch_elems=b, n_gpus=4))
     assert np.array_equal(_bits(B), want)
+
+
+@pytest.mark.parametrize("N", [2, 3])
+@pytest.mark.parametrize("dist", ["few_distinct", "uniform", "zipf_dup"])
+def test_multi_pairs_resident(hv, oracle_mod, inputs_mod, N, dist):
+    """Key/value RESIDENT plan over N GPUs: per-GPU stable batch sorts, then each GPU merges its
+    range of B/VB from all GPUs' key and value runs (two run-pointer tables)."""
+    n = 900_001
+    A = inputs_mod.generate(dist, n, seed=N + len(dist))
+    V = np.arange(n, dtype=np.uint64)[::-1].copy()
+    wantB, wantV = oracle_mod.sort_pairs_f64(A, V)
+    B, VB = _with(hv, {"merge_chunk": 1 << 17}, lambda: hv.hsort_sort_pairs_ex(A, V, batch_elems=65_536, n_gpus=N))
+    st = hv.hsort_get_stats()
+    assert st["mode_name"] == "RESIDENT" and st["n_gpus"] == N
+    assert np.array_equal(_bits(B), _bits(wantB)) and np.array_equal(VB, wantV)

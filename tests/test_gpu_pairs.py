@@ -101,3 +101,49 @@ def test_device_pairs_full_size_properties(hs_gpu, inputs_mod):
     eq = dB[1:] == dB[:-1]
     assert bool((dVB[1:][eq] > dVB[:-1][eq]).all())                       # stable
     assert bool((torch.bincount(dVB, minlength=n) == 1).all())            # a permutation
+
+
+# ---- out-of-core key/value: the RESIDENT plan (batches sorted stably in HBM + key/value merge) ----
+@pytest.mark.parametrize("dist", ["few_distinct", "zipf_dup", "all_equal", "special", "salted", "uniform"])
+@pytest.mark.parametrize("pinned", [False, True])
+def test_host_pairs_resident_batches(hs_gpu, oracle_mod, inputs_mod, dist, pinned):
+    """hsort_sort_pairs_ex with b_s < n: each batch stably sorted by the key/value GPUSort, then
+    K4 + the key/value K5 merge the runs with equal keys in run (= input) order: the unique stable
+    sort, bit-exact on keys and values.  Heavy ties cross batch boundaries (few_distinct, all_equal)."""
+    import torch
+    n, b = 1_000_003, 100_000
+    A = inputs_mod.generate(dist, n, seed=len(dist) + 3)
+    V = np.arange(n, dtype=np.uint64)
+    wantB, wantV = oracle_mod.sort_pairs_f64(A, V)
+    if pinned:
+        A = torch.from_numpy(A).pin_memory().numpy()
+        V = torch.from_numpy(V.view(np.int64)).pin_memory().numpy().view(np.uint64)
+    old = hs_gpu.hsort_get_option("merge_chunk")
+    hs_gpu.hsort_set_option("merge_chunk", 1 << 17)  # several merge chunks
+    try:
+        B, VB = hs_gpu.hsort_sort_pairs_ex(A, V, batch_elems=b)
+    finally:
+        hs_gpu.hsort_set_option("merge_chunk", old)
+    st = hs_gpu.hsort_get_stats()
+    assert st["mode_name"] == "RESIDENT" and st["n_b"] == -(-n // b)
+    assert np.array_equal(_bits(B), _bits(wantB))
+    assert np.array_equal(VB, wantV)
+
+
+def test_host_pairs_resident_auto_u64_in_place(hs_gpu, oracle_mod, inputs_mod):
+    """The auto plan of hsort_sort_pairs from n >= auto_pipeline_min (lowered here): pipelined
+    batches + halving tail; raw uint64 keys with duplicates; in place (B == A, VB == V)."""
+    n = 3_000_017
+    K = _bits(inputs_mod.generate("random_bits", n, seed=8)).copy()
+    K[::5] = K[7]
+    V = np.random.default_rng(1).integers(0, 2**64, size=n, dtype=np.uint64)
+    wantB, wantV = oracle_mod.sort_pairs_u64(K, V)
+    old = hs_gpu.hsort_get_option("auto_pipeline_min")
+    hs_gpu.hsort_set_option("auto_pipeline_min", 1 << 20)
+    try:
+        hs_gpu.hsort_sort_pairs_u64(K, V, K, V)
+        st = hs_gpu.hsort_get_stats()
+    finally:
+        hs_gpu.hsort_set_option("auto_pipeline_min", old)
+    assert st["mode_name"] == "RESIDENT" and st["n_b"] > 8
+    assert np.array_equal(K, wantB) and np.array_equal(V, wantV)

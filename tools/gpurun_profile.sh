@@ -15,7 +15,7 @@ timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/${tag}_bench.json
 echo "bench exit $?" >> gpurun_out/${tag}_bench.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 5000 --csv --log-file gpurun_out/${tag}_launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-extras > gpurun_out/${tag}_ncu_list.log 2>&1
 K="--set full --clock-control none --import-source on --kernel-name-base demangled"
-timeout 900 ncu $K -k "regex:k_onesweep_ws<576, 15, false, false, 0" -s 8 -c 1 -o gpurun_out/${tag}_onesweep_full python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-extras --device-only > gpurun_out/${tag}_ncu_full1.log 2>&1
+timeout 900 ncu $K -k "regex:k_onesweep_ws<\(int\)576, \(int\)15, \(bool\)0, \(bool\)0, \(int\)0" -s 10 -c 1 -o gpurun_out/${tag}_onesweep_full python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-extras --device-only --no-dde > gpurun_out/${tag}_ncu_full1.log 2>&1
 timeout 900 ncu $K -k "regex:k_merge_tile" -s 20 -c 1 -o gpurun_out/${tag}_merge_full python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-extras > gpurun_out/${tag}_ncu_full2.log 2>&1
 timeout 900 ncu $K -k "regex:k_hist3" -s 2 -c 1 -o gpurun_out/${tag}_hist_full python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-extras --device-only > gpurun_out/${tag}_ncu_full3.log 2>&1
 ls -la gpurun_out/${tag}_* | tail -20

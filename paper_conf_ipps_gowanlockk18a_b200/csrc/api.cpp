@@ -885,11 +885,19 @@ void sort_msd(std::vector<GpuCtx*>& gs, CallCtx& c) {
   std::mutex spl_m;
   std::condition_variable spl_cv;
   bool spl_ready = false;
+  bool spl_failed = false;
   std::thread sampler([&] {
-    std::vector<uint64_t> v = sample_splitters(c.A, n, c.f64, R);
+    std::vector<uint64_t> v;
+    bool ok = true;
+    try {
+      v = sample_splitters(c.A, n, c.f64, R);
+    } catch (...) {
+      ok = false;
+    }
     {
       std::lock_guard<std::mutex> lk(spl_m);
       spl = std::move(v);
+      spl_failed = !ok;
       spl_ready = true;
     }
     spl_cv.notify_all();
@@ -928,6 +936,7 @@ void sort_msd(std::vector<GpuCtx*>& gs, CallCtx& c) {
       if (i == 0) {  // the splitters are sampled while the first batch uploads
         std::unique_lock<std::mutex> lk(spl_m);
         spl_cv.wait(lk, [&] { return spl_ready; });
+        if (spl_failed) throw HsortError(HSORT_ERR_HOST_OOM, "splitter sampling failed");
         if (R > 1)
           CK(cudaMemcpyAsync(g.bspl.p, spl.data(), (R - 1) * 8, cudaMemcpyHostToDevice, g.s_comp));
       }

@@ -465,6 +465,44 @@ def pairs_e2e(hs, torch, A_h, B_h, n):
             "t_merge_gpu_s": st["t_merge_gpu"], "link_bytes_per_pair": 32}
 
 
+def lanes_row(hs, torch, A_h, B_h, n, sorts_per_lane=3):
+    """Serving throughput: two host threads sort their own pinned 2^30-key arrays at the same time
+    on lanes 0 and 1 (two GPU contexts of the same B200, hsort_sort_lane).  One sort cannot overlap
+    its HtoD with its DtoH (its first output key depends on its last input key); two concurrent
+    sorts use both link directions.  Not the headline: `value` is one sort at a time."""
+    import hsort_inputs
+    hsort_inputs.generate("uniform", n, seed=SEED, out=A_h.numpy())
+    A2 = torch.empty(n, dtype=torch.float64, pin_memory=True)
+    B2 = torch.empty(n, dtype=torch.float64, pin_memory=True)
+    hsort_inputs.generate("uniform", n, seed=SEED + 1, out=A2.numpy())
+    pairs = [(A_h, B_h), (A2, B2)]
+    for lane in (0, 1):
+        hs.hsort_sort_lane(lane, *pairs[lane])  # warm: the lane's buffers
+    bar = threading.Barrier(3)
+    ends = []
+
+    def work(lane):
+        bar.wait()
+        for _ in range(sorts_per_lane):
+            hs.hsort_sort_lane(lane, *pairs[lane])
+        ends.append(time.perf_counter())
+    th = [threading.Thread(target=work, args=(lane,)) for lane in (0, 1)]
+    for t in th:
+        t.start()
+    bar.wait()
+    t0 = time.perf_counter()
+    for t in th:
+        t.join()
+    dt = max(ends) - t0
+    for a, b in pairs:
+        guard(a.numpy(), b.numpy(), "lanes")
+    del A2, B2
+    return {"what": "2 concurrent hsort_sort_lane calls (lanes 0/1 = 2 GPU contexts of one B200), "
+                    f"{sorts_per_lane} sorts of 2^30 pinned keys each",
+            "keys_per_s": 2 * sorts_per_lane * n / dt, "ms_per_sort_per_lane": 1e3 * dt / sorts_per_lane,
+            "vs_one_at_a_time": None}
+
+
 def out_of_core(hs, torch, bw, host_bw):
     """The paper's out-of-core workflow (STREAM: batches -> HtoD -> GPUSort -> DtoH -> W, then the
     CPU/GPU merge split W -> B, configs C3/C5) at the largest n this host fits with
@@ -616,6 +654,8 @@ def main():
         n_gpu //= 2
     n = N * n_gpu
     hs.hsort_set_option("kernel_timing", 1)
+    if N == 1 and not args.no_extras:
+        hs.hsort_set_option("virtual_gpus", 2)  # a second GPU context on the device: the lanes row
     if args.no_dde:
         hs.hsort_set_option("dde", 0)
     t0 = time.perf_counter()
@@ -768,6 +808,8 @@ def main():
         line["stages"] = stages
         line["skewed"] = skewed_rows(hs, torch, A_h, B_h, d_in, d_out, stream, peak, n_gpu)
         line["pairs_e2e"] = pairs_e2e(hs, torch, A_h, B_h, n_gpu)
+        line["lanes"] = lanes_row(hs, torch, A_h, B_h, n_gpu)
+        line["lanes"]["vs_one_at_a_time"] = line["lanes"]["keys_per_s"] / value
     del d_in, d_out
     torch.cuda.empty_cache()
     host_bw = None

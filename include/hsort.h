@@ -19,7 +19,8 @@
  *  - After a CUDA error the library is poisoned: later calls return HSORT_ERR_CUDA until
  *    hsort_finalize().  B's contents are unspecified after an error; A is never written
  *    unless B == A.
- *  - The library is not re-entrant: a concurrent hsort_sort returns HSORT_ERR_BUSY.
+ *  - The library is not re-entrant: a concurrent hsort_sort returns HSORT_ERR_BUSY (except
+ *    hsort_sort_lane calls on different lanes, which may run concurrently).
  *  - "host" pointers may be pageable or pinned (cudaHostAlloc / cudaHostRegister); pinned
  *    buffers are DMA'd directly, pageable ones go through the pinned staging ring (Stage, MCpy).
  *  - "device" pointers are CUDA global memory on the CURRENT device; "stream" is a cudaStream_t
@@ -138,6 +139,16 @@ int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_
 int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_t batch_elems,
                    int n_gpus);
 
+/* Concurrent sorts (serving): hsort_sort on GPU context `lane` alone (0 <= lane < contexts: the
+ * visible devices, or option "virtual_gpus").  Calls on different lanes may run at the same time
+ * from different host threads -- on one GPU their HtoD and DtoH overlap, which one sort cannot do
+ * (its first output key depends on its last input key).  The runs must fit in the lane's HBM
+ * (RESIDENT or BLINE plans; a STREAM plan -> HSORT_ERR_INVALID).  A call on a busy lane, or while
+ * an hsort_sort/hsort_sort_pairs/hsort_sort_typed call runs, -> HSORT_ERR_BUSY (and vice versa).
+ * Arguments as hsort_sort. */
+int hsort_sort_lane(int lane, const double* A_host, double* B_host, uint64_t n,
+                    uint64_t batch_elems);
+
 /* ---------------------------------------------------------------------------------------------
  * Other key types and orders.  key_type HSORT_KEY_F64 (8-byte float64) or
  * HSORT_KEY_F32 (4-byte float32); descending != 0 sorts by the reverse of IEEE totalOrder (the
@@ -203,7 +214,7 @@ int hsort_sort_pairs_ex(const void* A_host, const uint64_t* V_host, void* B_host
  * ------------------------------------------------------------------------------------------- */
 int hsort_set_option(const char* key, int64_t value);
 int hsort_get_option(const char* key, int64_t* value);
-int hsort_get_stats(hsort_stats* out);      /* stats of the last successful hsort_sort */
+int hsort_get_stats(hsort_stats* out);      /* stats of the calling thread's last successful sort */
 const char* hsort_last_error(void);          /* thread-local; never NULL */
 const char* hsort_version(void);
 

@@ -76,6 +76,7 @@ SIGNATURES = {
     "hsort_finalize": ([], _I),
     "hsort_sort": ([_P, _P, _U64, _U64, _I], _I),
     "hsort_sort_u64": ([_P, _P, _U64, _U64, _I], _I),
+    "hsort_sort_lane": ([_I, _P, _P, _U64, _U64], _I),
     "hsort_sort_typed": ([_P, _P, _U64, _I, _I], _I),
     "hsort_sort_device_typed": ([_P, _P, _U64, _I, _I, _P], _I),
     "hsort_sort_pairs": ([_P, _P, _P, _P, _U64], _I),
@@ -210,6 +211,19 @@ def hsort_sort(A, B=None, batch_elems: int = 0, n_gpus: int = 0):
     if nb != n:
         raise ValueError("A and B must have the same length")
     _check(lib().hsort_sort(a, b, n, batch_elems, n_gpus))
+    return B
+
+
+def hsort_sort_lane(lane: int, A, B=None, batch_elems: int = 0):
+    """hsort_sort on GPU context `lane` alone; calls on different lanes may run concurrently
+    (the ctypes call releases the GIL)."""
+    a, n = _host_ptr(A, np.float64)
+    if B is None:
+        B = np.empty(n, dtype=np.float64)
+    b, nb = _host_ptr(B, np.float64)
+    if nb != n:
+        raise ValueError("A and B must have the same length")
+    _check(lib().hsort_sort_lane(lane, a, b, n, batch_elems))
     return B
 
 

@@ -169,10 +169,8 @@ struct State {
   std::mutex m;
   bool inited = false;
   bool poisoned = false;
-  std::atomic<bool> busy{false};
   std::vector<GpuCtx> gpus;
   Options opt;
-  hsort_stats last{};
   double t_init = 0;
   // pinned working memory W (STREAM mode), allocated once and reused: pinning is expensive
   // so it is cached like the staging ring
@@ -185,11 +183,20 @@ struct State {
   // query behind the plan (cudaMemGetInfo) measured 0.1-62 ms on the B200 box
   // (profiles/r02l_setup.txt), which made repeated calls jitter by tens of ms
   uint64_t opt_version = 0;
-  bool plan_valid = false;
-  uint64_t plan_n = 0, plan_b = 0;
-  int plan_ng = -1;
-  uint64_t plan_opt = 0;
-  hsort_plan_t plan_cached{};
+  struct PlanCache {
+    bool valid = false;
+    uint64_t n = 0, b = 0;
+    int ng = -1;
+    uint64_t opt = 0;
+    hsort_plan_t plan{};
+  };
+  PlanCache pc[65];  // [0]: calls over GPUs [0, n_gpus); [1 + l]: calls on lane l
+  // concurrency: a regular call owns every GPU context; lane calls (hsort_sort_lane) own one
+  // context each and may run concurrently on different lanes
+  std::mutex busy_m;
+  bool global_busy = false;
+  int lanes_active = 0;
+  bool lane_busy[64] = {};
   int n_physical = 0;      // visible CUDA devices
 };
 State& S() {
@@ -197,11 +204,34 @@ State& S() {
   return s;
 }
 
+// stats of the calling thread's last successful sort (lanes sort concurrently)
+thread_local hsort_stats t_last{};
+
 struct BusyGuard {
-  bool ok;
-  BusyGuard() { ok = !S().busy.exchange(true); }
+  bool ok = false;
+  int lane;
+  explicit BusyGuard(int l = -1) : lane(l) {
+    std::lock_guard<std::mutex> g(S().busy_m);
+    if (lane < 0) {
+      ok = !S().global_busy && S().lanes_active == 0;
+      if (ok) S().global_busy = true;
+    } else {
+      ok = !S().global_busy && !S().lane_busy[lane];
+      if (ok) {
+        S().lane_busy[lane] = true;
+        ++S().lanes_active;
+      }
+    }
+  }
   ~BusyGuard() {
-    if (ok) S().busy.store(false);
+    if (!ok) return;
+    std::lock_guard<std::mutex> g(S().busy_m);
+    if (lane < 0) {
+      S().global_busy = false;
+    } else {
+      S().lane_busy[lane] = false;
+      --S().lanes_active;
+    }
   }
 };
 
@@ -1576,10 +1606,10 @@ void ctx_destroy(GpuCtx& g) {
 // Usable HBM per GPU context for a call on the first n_gpus contexts: free memory of its device
 // shared by the call's contexts on that device (virtual GPUs, option "virtual_gpus"), plus what
 // the context already holds; the minimum over the contexts.
-uint64_t device_budget(int n_gpus) {
+uint64_t device_budget(const std::vector<int>& ctx) {
   uint64_t best = ~0ull;
   std::map<int, int> per_dev;
-  for (int i = 0; i < n_gpus; ++i) per_dev[S().gpus[i].dev]++;
+  for (int i : ctx) per_dev[S().gpus[i].dev]++;
   std::map<int, uint64_t> free_of;
   for (auto& kv : per_dev) {
     CK(cudaSetDevice(kv.first));
@@ -1587,12 +1617,17 @@ uint64_t device_budget(int n_gpus) {
     CK(cudaMemGetInfo(&fr, &tot));
     free_of[kv.first] = fr;
   }
-  for (int i = 0; i < n_gpus; ++i) {
+  for (int i : ctx) {
     const GpuCtx& g = S().gpus[i];
     const uint64_t held = g.runs.cap + g.alt.cap + g.mout.cap + g.ranks.cap + g.min.cap + g.coarse.cap;
     best = std::min<uint64_t>(best, free_of[g.dev] / per_dev[g.dev] + held);
   }
   return best == ~0ull ? 0 : best;
+}
+uint64_t device_budget(int n_gpus) {
+  std::vector<int> ctx;
+  for (int i = 0; i < n_gpus; ++i) ctx.push_back(i);
+  return device_budget(ctx);
 }
 
 GpuCtx& current_ctx() {
@@ -1615,16 +1650,21 @@ int check_ready() {
   return HSORT_OK;
 }
 
-int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus, bool f64) {
+int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus, bool f64,
+            int lane = -1) {
   int rc = check_ready();
   if (rc) return rc;
-  BusyGuard busy;
+  if (lane >= (int)S().gpus.size() || lane >= 64) {
+    g_err = "lane must be in [0, GPU contexts)";
+    return HSORT_ERR_INVALID;
+  }
+  BusyGuard busy(lane);
   if (!busy.ok) {
     g_err = "hsort_sort already running";
     return HSORT_ERR_BUSY;
   }
   if (n == 0) {
-    S().last = hsort_stats{};
+    t_last = hsort_stats{};
     return HSORT_OK;
   }
   if (!A || !B) {
@@ -1646,19 +1686,27 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
     return HSORT_ERR_INVALID;
   }
   if (n_gpus == 0) n_gpus = vis;
+  if (lane >= 0) n_gpus = 1;
   return guarded([&]() -> int {
     Nvtx nv("hsort_sort");
     auto t0 = Clock::now();
-    GpuCtx& g0 = S().gpus[0];
+    std::vector<int> ctx;  // the GPU contexts this call owns
+    if (lane >= 0) ctx.push_back(lane);
+    else
+      for (int i = 0; i < n_gpus; ++i) ctx.push_back(i);
+    GpuCtx& g0 = S().gpus[ctx[0]];
+    State::PlanCache& pc = S().pc[lane + 1];
     hsort_plan_t plan;
-    if (S().plan_valid && S().plan_n == n && S().plan_b == batch_elems && S().plan_ng == n_gpus &&
-        S().plan_opt == S().opt_version) {
-      plan = S().plan_cached;  // the buffers it needs are already held
+    if (pc.valid && pc.n == n && pc.b == batch_elems && pc.ng == n_gpus && pc.opt == S().opt_version) {
+      plan = pc.plan;  // the buffers it needs are already held
     } else {
-      const uint64_t budget = device_budget(n_gpus);
+      const uint64_t budget = device_budget(ctx);
       plan = make_plan(n, batch_elems, n_gpus, budget, S().opt, S().peer_ok);
-      S().plan_valid = false;
+      pc.valid = false;
     }
+    if (lane >= 0 && plan.mode == HSORT_MODE_STREAM)
+      throw HsortError(HSORT_ERR_INVALID, "lane sorts keep their runs in HBM (RESIDENT/BLINE); "
+                                          "STREAM (host working memory W) is not per lane");
     CK(cudaSetDevice(g0.dev));
     hsort_stats st{};
     st.n = n;
@@ -1711,7 +1759,7 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
       sort_bline(g0, c);
     } else if (plan.mode == HSORT_MODE_RESIDENT) {
       std::vector<GpuCtx*> gs;
-      for (int i = 0; i < plan.n_gpus; ++i) gs.push_back(&S().gpus[i]);
+      for (int i = 0; i < plan.n_gpus; ++i) gs.push_back(&S().gpus[ctx[i]]);
       if (S().opt.get("msd") == 1) sort_msd(gs, c);
       else sort_resident(gs, c);
     } else {
@@ -1721,13 +1769,13 @@ int do_sort(const void* A, void* B, uint64_t n, uint64_t batch_elems, int n_gpus
       sort_stream(gs, c);
     }
     st.t_total = secs_since(t0);
-    S().last = st;
-    S().plan_cached = plan;  // succeeded: its buffers are allocated
-    S().plan_n = n;
-    S().plan_b = batch_elems;
-    S().plan_ng = n_gpus;
-    S().plan_opt = S().opt_version;
-    S().plan_valid = true;
+    t_last = st;
+    pc.plan = plan;  // succeeded: its buffers are allocated
+    pc.n = n;
+    pc.b = batch_elems;
+    pc.ng = n_gpus;
+    pc.opt = S().opt_version;
+    pc.valid = true;
     return HSORT_OK;
   });
 }
@@ -1745,7 +1793,7 @@ int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint6
     return HSORT_ERR_BUSY;
   }
   if (n == 0) {
-    S().last = hsort_stats{};
+    t_last = hsort_stats{};
     return HSORT_OK;
   }
   if (!A || !B || !V || !VB) {
@@ -1847,7 +1895,7 @@ int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint6
       for (int i = 0; i < N; ++i) gs.push_back(&S().gpus[i]);
       sort_resident(gs, c);
       st.t_total = secs_since(t0);
-      S().last = st;
+      t_last = st;
       return HSORT_OK;
     });
   }
@@ -1906,7 +1954,7 @@ int do_sort_pairs(const void* A, const uint64_t* V, void* B, uint64_t* VB, uint6
     es.destroy();
     ed.destroy();
     st.t_total = secs_since(t0);
-    S().last = st;
+    t_last = st;
     return HSORT_OK;
   });
 }
@@ -1926,7 +1974,7 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     return HSORT_ERR_BUSY;
   }
   if (n == 0) {
-    S().last = hsort_stats{};
+    t_last = hsort_stats{};
     return HSORT_OK;
   }
   const uint64_t es = key_type == HSORT_KEY_F64 ? 8 : 4;
@@ -2013,7 +2061,7 @@ int do_sort_typed(const void* A, void* B, uint64_t n, int key_type, int desc) {
     es_.destroy();
     ed.destroy();
     st.t_total = secs_since(t0);
-    S().last = st;
+    t_last = st;
     return HSORT_OK;
   });
 }
@@ -2093,7 +2141,7 @@ int hsort_init(void) {
 int hsort_finalize(void) {
   std::lock_guard<std::mutex> lk(S().m);
   release_w();
-  S().plan_valid = false;
+  for (auto& p : S().pc) p.valid = false;
   for (auto& g : S().gpus) ctx_destroy(g);
   S().gpus.clear();
   S().inited = false;
@@ -2108,6 +2156,12 @@ int hsort_sort(const double* A_host, double* B_host, uint64_t n, uint64_t batch_
 int hsort_sort_u64(const uint64_t* A_host, uint64_t* B_host, uint64_t n, uint64_t batch_elems,
                    int n_gpus) {
   return do_sort(A_host, B_host, n, batch_elems, n_gpus, false);
+}
+
+int hsort_sort_lane(int lane, const double* A_host, double* B_host, uint64_t n,
+                    uint64_t batch_elems) {
+  if (lane < 0) return g_err = "lane must be >= 0", HSORT_ERR_INVALID;
+  return do_sort(A_host, B_host, n, batch_elems, 1, true, lane);
 }
 
 int hsort_sort_typed(const void* A_host, void* B_host, uint64_t n, int key_type, int descending) {
@@ -2199,7 +2253,7 @@ int hsort_get_option(const char* key, int64_t* value) {
 
 int hsort_get_stats(hsort_stats* out) {
   if (!out) return HSORT_ERR_INVALID;
-  *out = S().last;
+  *out = t_last;
   return HSORT_OK;
 }
 

@@ -214,3 +214,43 @@ def test_multi_pairs_resident(hv, oracle_mod, inputs_mod, N, dist):
     st = hv.hsort_get_stats()
     assert st["mode_name"] == "RESIDENT" and st["n_gpus"] == N
     assert np.array_equal(_bits(B), _bits(wantB)) and np.array_equal(VB, wantV)
+
+
+# ---- lanes: concurrent sorts on one GPU (hsort_sort_lane) -------------------------------------------
+def test_lanes_concurrent_sorts(hv, oracle_mod, inputs_mod):
+    """Two host threads sort different arrays at the same time on lanes 0 and 1 (two GPU contexts
+    of the same device): every output bit-exact; a regular call meanwhile gets HSORT_ERR_BUSY."""
+    import threading
+    arrays = [inputs_mod.generate(d, 1_500_001 + i, seed=i) for i, d in enumerate(["uniform", "zipf_dup"])]
+    wants = [_bits(oracle_mod.sort_f64(a)) for a in arrays]
+    errors, busy_seen = [], []
+    start = threading.Barrier(2)
+
+    def worker(lane):
+        try:
+            start.wait()
+            for rep in range(4):
+                B = hv.hsort_sort_lane(lane, arrays[lane], batch_elems=200_000 if rep % 2 else 0)
+                if not np.array_equal(_bits(B), wants[lane]):
+                    errors.append((lane, rep))
+                st = hv.hsort_get_stats()
+                if st["n"] != arrays[lane].size:  # per-thread stats
+                    errors.append(("stats", lane))
+        except Exception as e:  # noqa: BLE001
+            errors.append(repr(e))
+
+    th = [threading.Thread(target=worker, args=(l,)) for l in (0, 1)]
+    for t in th:
+        t.start()
+    try:
+        hv.hsort_sort(arrays[0])
+    except hv.HsortError as e:
+        busy_seen.append(e.code)
+    for t in th:
+        t.join()
+    assert not errors, errors
+    assert all(c == -7 for c in busy_seen)
+    with pytest.raises(hv.HsortError):
+        hv.hsort_sort_lane(99, arrays[0])
+    with pytest.raises(hv.HsortError):  # a STREAM plan is not per lane
+        _with(hv, {"resident": 0}, lambda: hv.hsort_sort_lane(0, arrays[0], batch_elems=100_000))

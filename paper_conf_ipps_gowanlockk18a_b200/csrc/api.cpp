@@ -133,6 +133,8 @@ struct Options {
       {"pin_w", -1},                 // STREAM W: 1 page-locked, 0 pageable, -1 locked if <= pin_w_max_mb
       {"pin_w_max_mb", 1ll << 20},   // auto page-locking limit of W (MB)
       {"w_cache", 1},                // keep W (allocated, prefaulted, locked) across calls
+      {"merge_stage_threads", 8},    // STREAM merge: host threads per GPU reserved for staging the
+                                     // GPU share's DtoH into a pageable B
 
       {"virtual_gpus", 0},           // > 0 (set before hsort_init): that many GPU contexts mapped
                                      // round-robin onto the visible devices (multi-GPU scheduler,
@@ -1173,7 +1175,7 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
     CK(cudaStreamWaitEvent(g.s_d2h, merged[s], 0));
     const uint64_t p0 = o_lo + ch * C;
     download(g, (uint64_t*)c.B + p0, g.mout.u64() + (uint64_t)s * C, totals[ch] * 8, g.s_d2h,
-             c.direct_out, c.mc_threads, acc);
+             c.direct_out, (int)S().opt.get("merge_stage_threads"), acc);
     CK(cudaEventRecord(out_free[s], g.s_d2h));
   }
   CK(cudaEventRecord(em.b, g.s_d2h));
@@ -1509,8 +1511,13 @@ void sort_stream(std::vector<GpuCtx*>& gs, CallCtx& c) {
     try {
       Nvtx nv("CPU merge W -> B");
       auto tc = Clock::now();
-      host_merge_runs_range(run.data(), rlen.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64,
-                            c.merge_threads, nullptr);
+      // the CPU share runs on its own pool; while the GPU share stages DtoH chunks into a
+      // pageable B it keeps `merge_stage_threads` cores free for that staging
+      int mt = c.merge_threads > 0 ? c.merge_threads : host_threads();
+      if (o_f > 0 && !c.direct_out)
+        mt = std::max<int>(1, mt - (int)S().opt.get("merge_stage_threads") * (int)gs.size());
+      host_merge_runs_range(run.data(), rlen.data(), k, o_f, n, (uint64_t*)c.B + o_f, c.f64, mt,
+                            &merge_pool());
       t_cpu = secs_since(tc);
     } catch (const std::exception& e) {
       cpu_code = HSORT_ERR_INTERNAL;

@@ -80,6 +80,11 @@ ThreadPool& host_pool() {
   return pool;
 }
 
+ThreadPool& merge_pool() {
+  static ThreadPool pool(std::max(1, host_threads() - 1));
+  return pool;
+}
+
 ThreadPool& pipe_pool() {
   static ThreadPool pool(std::max(1, host_threads() / 2 - 1));
   return pool;

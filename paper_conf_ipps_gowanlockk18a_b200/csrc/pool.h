@@ -48,6 +48,9 @@ ThreadPool& host_pool();
 // Second pool for the PIPEMERGE pair merges that run during the sort phase, so they never queue
 // ahead of the PARMEMCPY staging jobs on host_pool() (half the hardware threads).
 ThreadPool& pipe_pool();
+// Pool of the STREAM merge phase's CPU share, so its loser-tree tasks never queue ahead of the
+// GPU share's staging copies on host_pool() (they ran FIFO on one pool in round 1).
+ThreadPool& merge_pool();
 int host_threads();
 
 // PARMEMCPY: dst <- src (bytes) split over `threads` workers (0 = all host threads).

@@ -1264,7 +1264,7 @@ __device__ __forceinline__ void lookback8(const uint32_t* __restrict__ lb, int64
 // K32: 32-bit keys (float32 / uint32, S§8(f) #4 native path): 4-byte stage and stores, the
 // binary32 key transform; keys-only, no elision.
 template <int CT, int ITEMS, bool IN_F64, bool KV = false, int DM = 0, bool DESC = false, bool K32 = false>
-__global__ void __launch_bounds__(CT + 32, (CT <= 288 ? 2 : 1)) k_onesweep_ws(uint64_t* in64, uint64_t* out64, uint64_t* tmp64,
+__global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(uint64_t* in64, uint64_t* out64, uint64_t* tmp64,
                                                        uint64_t* vin, uint64_t* vout, uint64_t* vtmp,
                                                        uint64_t n, const RadixPlan* __restrict__ plan,
                                                        const uint64_t* __restrict__ bin_base,

@@ -78,3 +78,45 @@ def test_large_multi_gpu_auto_plan_matches_oracle(hs_gpu, oracle_mod, inputs_mod
         hs_gpu.hsort_finalize()
         hs_gpu.hsort_set_option("virtual_gpus", 0)
         hs_gpu.hsort_init()
+
+
+def test_fullsize_host_pairs_properties(hs_gpu, full):
+    """The bench's pairs_e2e call at 2^30 (RESIDENT key/value plan, pinned): keys equal the oracle's
+    key sort; every (key, value) pair of the input is preserved (A[VB] == B); equal keys keep input
+    order (VB increasing inside runs of equal keys) -- with V = 0..n-1 these fix the unique stable
+    answer."""
+    import torch
+    A, want = full
+    n = A.size
+    At = torch.from_numpy(A).pin_memory()
+    V = torch.arange(n, dtype=torch.int64).pin_memory()
+    Bt = torch.empty(n, dtype=torch.float64).pin_memory()
+    VBt = torch.empty(n, dtype=torch.int64).pin_memory()
+    hs_gpu.hsort_sort_pairs(At.numpy(), V.numpy().view(np.uint64), Bt.numpy(), VBt.numpy().view(np.uint64))
+    st = hs_gpu.hsort_get_stats()
+    assert st["mode_name"] == "RESIDENT" and st["n_b"] == 12
+    B = Bt.numpy().view(np.uint64)
+    VB = VBt.numpy()
+    assert _first_diff(B, want) is None
+    assert np.array_equal(A.view(np.uint64)[VB], B)
+    eq = B[1:] == B[:-1]
+    assert bool(np.all(VB[1:][eq] > VB[:-1][eq]))
+
+
+def test_large_stream_out_of_core_matches_oracle(hs_gpu, oracle_mod, inputs_mod):
+    """The paper's out-of-core workflow (STREAM: runs to page-locked W, CPU/GPU merge split with
+    the auto f, pageable A/B) at 2^27 + ragged keys in 2^24-key batches, element by element."""
+    n = (1 << 27) + 4321
+    A = inputs_mod.generate("normal", n, seed=21)
+    want = oracle_mod.sort_f64(A).view(np.uint64)
+    old = {k: hs_gpu.hsort_get_option(k) for k in ("resident", "pin_w")}
+    hs_gpu.hsort_set_option("resident", 0)
+    hs_gpu.hsort_set_option("pin_w", 1)
+    try:
+        B = hs_gpu.hsort_sort(A, batch_elems=1 << 24)
+        st = hs_gpu.hsort_get_stats()
+    finally:
+        for k, v in old.items():
+            hs_gpu.hsort_set_option(k, v)
+    assert st["mode_name"] == "STREAM" and st["n_b"] == 9 and 0 < st["merge_gpu_fraction"] < 1
+    assert _first_diff(B.view(np.uint64), want) is None

@@ -2,7 +2,8 @@
 synccheck / initcheck): K1/K2/K3 (f64, u64, elision with a lowered threshold; the elision's K1
 outlier count on normal data), key/value, typed float32 descending, K4 two-level + K5, host
 RESIDENT and STREAM modes, and (round 2) the multi-GPU RESIDENT merge through the run-pointer
-table, the MSD-first split (K6a-d) and multi-GPU STREAM on 3 virtual GPUs.  Checks results against
+table, the MSD-first split (K6a-d), multi-GPU STREAM on 3 virtual GPUs, the key/value RESIDENT
+plan (key/value K5), the native float32 GPUSort and two concurrent lanes.  Checks results against
 the oracle so a silent corruption also fails."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -64,5 +65,23 @@ hs.hsort_set_option("msd", 0)
 hs.hsort_set_option("resident", 0)
 hs.hsort_set_option("merge_gpu_permille", 500)
 assert np.array_equal(bits(hs.hsort_sort(A, batch_elems=20_000, n_gpus=3)), want), "multi STREAM"
+hs.hsort_set_option("resident", -1)
+# key/value RESIDENT plan over 2 GPU contexts (key/value K5, value run-pointer tables)
+Vp = np.arange(A.size, dtype=np.uint64)
+wB, wV = oracle.sort_pairs_f64(A, Vp)
+B2, VB2 = hs.hsort_sort_pairs_ex(A, Vp, batch_elems=20_000, n_gpus=2)
+assert np.array_equal(bits(B2), bits(wB)) and np.array_equal(VB2, wV), "pairs RESIDENT multi"
+# native float32 GPUSort
+F = A.astype(np.float32)
+assert np.array_equal(hs.hsort_sort_typed(F).view(np.uint32), oracle.sort_f32(F, False).view(np.uint32)), "f32 native"
+# two lanes at once
+import threading
+res = {}
+def lane(l):
+    res[l] = hs.hsort_sort_lane(l, A, batch_elems=30_000 if l else 0)
+th = [threading.Thread(target=lane, args=(l,)) for l in (0, 1)]
+for t in th: t.start()
+for t in th: t.join()
+assert all(np.array_equal(bits(res[l]), want) for l in (0, 1)), "lanes"
 hs.hsort_finalize()
 print("sanitize_run ok")

@@ -1130,7 +1130,8 @@ struct WsSmem {
   static constexpr size_t bar_off = cnt_off + 2 * kRadix * 4;                 // [12] u64
   static constexpr size_t swarp_off = bar_off + 12 * 8;                       // [8] u32 (+pad)
   static constexpr size_t tile_off = swarp_off + 64;                          // [4] u32
-  static constexpr size_t bytes = tile_off + 16;
+  static constexpr size_t dummy_off = tile_off + 16;                          // [32] u32 (+pad)
+  static constexpr size_t bytes = dummy_off + 32 * 4;
 };
 
 #ifndef HSORT_WS_CT
@@ -1147,10 +1148,20 @@ struct WsSmem {
                             // (A/B 15 / 18 / 20 / 22: 19.2 / 18.6 / 17.4 / 17.7 ms per 2^30 keys)
 #endif
 #ifndef HSORT_WS_NMATCH
-#define HSORT_WS_NMATCH 3  // items ranked with match.any in high-entropy passes (best of 0..7)
+#define HSORT_WS_NMATCH 4  // items ranked with match.any in high-entropy passes (A/B over 2..7)
 #endif
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
+#endif
+#ifndef HSORT_WS_PATOM
+#define HSORT_WS_PATOM 3  // leader atomics: 0 branch per item, 1 predicated PTX, 2 every lane adds to
+                          // the digit slot (0 unless leader), 3 non-leaders add to a word of their own
+#endif
+#ifndef HSORT_WS_IL_DM2
+#define HSORT_WS_IL_DM2 0  // ... also in the elision's diverting pass (A/B: slower, spills)
+#endif
+#ifndef HSORT_WS_IL
+#define HSORT_WS_IL 1  // write-out of tile j-1 interleaved with the ranking of tile j (full tiles)
 #endif
 // key/value pass: HSORT_KV_CT compute threads x HSORT_KV_ITEMS pairs (internal.h: 10 warps x 13)
 constexpr int kKvCT = HSORT_KV_CT;
@@ -1174,6 +1185,16 @@ __device__ __forceinline__ void st_global_u64(uint64_t addr, uint64_t v) {
 __device__ __forceinline__ void st_global_w(const uint64_t* a, uint64_t v) { st_global_u64((uint64_t)a, v); }
 __device__ __forceinline__ void st_global_w(const uint32_t* a, uint32_t v) {
   asm volatile("st.global.u32 [%0], %1;" ::"l"((uint64_t)a), "r"(v) : "memory");
+}
+// The group leader's shared atomic as one predicated instruction (no branch per item); the
+// result is defined in the leader lane only (the others read it by shuffle)
+__device__ __forceinline__ uint32_t atom_add_if_leader(uint32_t* a, uint32_t v, int lane, int leader) {
+  uint32_t r;
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.eq.s32 q, %1, %2;\n\t@q atom.shared.add.u32 %0, [%3], %4;\n\t}"
+               : "=r"(r)
+               : "r"(lane), "r"(leader), "r"(smem_u32(a)), "r"(v)
+               : "memory");
+  return r;
 }
 // One bit of the ballot multisplit: peers &= (bit b of d) ? ballot(bit) : ~ballot(bit).
 __device__ __forceinline__ uint32_t peer_bit(uint32_t peers, uint32_t d, uint32_t bm) {
@@ -1293,6 +1314,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   uint64_t* bars = (uint64_t*)(smem + L::bar_off);
   uint32_t* s_warp = (uint32_t*)(smem + L::swarp_off);
   uint32_t* s_tile = (uint32_t*)(smem + L::tile_off);
+  uint32_t* s_dummy = (uint32_t*)(smem + L::dummy_off);  // leader atomics: non-leaders' targets
   uint64_t* bar_tma = bars;       // [3] stage s holds its tile (TMA done, or "no tile")
   uint64_t* bar_a = bars + 3;     // [2] tile j counted, A published, counts in s_cnt
   uint64_t* bar_g = bars + 5;     // [2] offsets of tile j in s_gofs
@@ -1512,8 +1534,12 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
   // DM (compile-time): 0 no elision work, 1 count the outliers' digit-P histogram (pass 0),
   // 2 divert the outliers (the elision's last pass; never FULL)
-  auto rank_tile = [&](auto full_tag, uint64_t tile, int tile_n, KT* sb, uint64_t* vsb) {
+  // WO (compile-time): 0 = no write-out here; 1 / 2 = write tile j-1 out (2: with the inverse
+  // transform) interleaved with this tile's ranking, so its shared loads and global stores issue
+  // beside the ballots (ALU) instead of in a memory-only phase of their own
+  auto rank_tile = [&](auto full_tag, auto wo_tag, uint64_t tile, int tile_n, KT* sb, uint64_t* vsb) {
     constexpr bool FULL = decltype(full_tag)::value;
+    constexpr int WO = decltype(wo_tag)::value;
     const uint64_t tbase = tile * (uint64_t)TILE;
     const int bulk_n = (int)(((uint32_t)tile_n * (uint32_t)sizeof(KT) & ~15u) / (uint32_t)sizeof(KT));
     const int wofs = warp * 32 * ITEMS + lane;
@@ -1598,13 +1624,29 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #ifdef HSORT_PHASE_TIMING
     long long cr0 = clock64();
 #endif
+    const uint32_t jp = j - 1;  // WO: the previous tile (every warp scattered it before barrier 1)
+    const int32_t* pgofs = s_gofs + (jp & 1) * kRadix;
+    const KT* psb = stage + (size_t)(jp % 3) * TILE;
+    const uint64_t* pvsb = vstage + (size_t)(jp % 3) * TILE;
+    if (WO) mbar_wait(&bar_g[jp & 1], (jp >> 1) & 1u);
+    auto wo_item = [&](int q) {
+      if (WO && q < ITEMS) {
+        const KT v = psb[tid + q * THREADS];
+        const int32_t g = pgofs[(uint32_t)(v >> shift) & 255u];
+        st_global_w(dst_t + g + q * THREADS, WO == 2 ? from_key_w((KT)(v ^ kx)) : v);
+        if (KV) st_global_u64((uint64_t)(vdst + tid + g + q * THREADS), pvsb[tid + q * THREADS]);
+      }
+    };
 
     // rank: peers = lanes of this item with the same digit; the leader's atomic on the warp's
     // base returns the group's first slot.
     uint32_t peers[ITEMS];
     if (use_match) {
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+      for (int i = 0; i < ITEMS; ++i) {
+        peers[i] = __match_any_sync(0xffffffffu, dd[i]);
+        wo_item(i);
+      }
     } else {
       // high-entropy digits: an 8-ballot multisplit (4 instructions per bit: test -> predicate,
       // vote, select, and) for most items; the first NM items use match.any, which runs on another
@@ -1619,11 +1661,21 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       for (int b = 0; b < (FULL ? 8 : 9); ++b) {
 #pragma unroll
         for (int i = NM; i < ITEMS; ++i) peers[i] = peer_bit(peers[i], dd[i], 1u << b);
+        if (b < 8) {
+          wo_item(2 * b);
+          wo_item(2 * b + 1);
+        }
       }
       if (FULL && DM == 2 && w_out) {  // diverted items carry digit 256: separate them (bit 8)
 #pragma unroll
         for (int i = NM; i < ITEMS; ++i) peers[i] = peer_bit(peers[i], dd[i], 1u << 8);
       }
+#pragma unroll
+      for (int q = 16; q < ITEMS; ++q) wo_item(q);
+    }
+    if (WO) {  // tile j-1 is written out: release its stage to the next TMA
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bar_free[jp % 3]);
     }
 #if HSORT_FAKE == 2
 #pragma unroll
@@ -1642,9 +1694,17 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
-      rr[i] = (lane == leader && ((FULL && (DM != 2 || !w_out)) || dd[i] < kRadix))
-                  ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i]))
-                  : 0u;
+      if (HSORT_WS_PATOM == 1 && FULL && DM != 2)
+        rr[i] = atom_add_if_leader(&wh[dd[i]], (uint32_t)__popc(peers[i]), lane, leader);
+      else if (HSORT_WS_PATOM == 2 && FULL && DM != 2)  // every lane adds (0 unless leader)
+        rr[i] = atomicAdd(&wh[dd[i]], lane == leader ? (uint32_t)__popc(peers[i]) : 0u);
+      else if (HSORT_WS_PATOM == 3 && FULL && DM != 2)  // every lane adds; a non-leader to its own
+        // word of s_dummy, so large groups (duplicate-heavy data) do not serialise on one address
+        rr[i] = atomicAdd(lane == leader ? &wh[dd[i]] : s_dummy + lane, (uint32_t)__popc(peers[i]));
+      else
+        rr[i] = (lane == leader && ((FULL && (DM != 2 || !w_out)) || dd[i] < kRadix))
+                    ? atomicAdd(&wh[dd[i]], (uint32_t)__popc(peers[i]))
+                    : 0u;
     }
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -1684,8 +1744,25 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     KT* sb = stage + (size_t)cb * TILE;
     uint64_t* vsb = vstage + (size_t)cb * TILE;
     long long cr0;
-    if (tile_n == TILE) cr0 = rank_tile(std::true_type{}, tile, tile_n, sb, vsb);
-    else cr0 = rank_tile(std::false_type{}, tile, tile_n, sb, vsb);
+    using WO0 = std::integral_constant<int, 0>;
+    // interleaved write-out (WO): this tile and the previous one are full (only the last tile is
+    // ragged; in the elision's diverting pass a tile that lost outliers is written out separately)
+    constexpr bool IL = HSORT_WS_IL && (DM != 2 || HSORT_WS_IL_DM2);
+    bool il = IL && j >= 1 && tile_n == TILE;
+    if (DM == 2 && il) {  // the elision's diverting pass: only if tile j-1 lost no outliers
+      const uint32_t c = s_cnt[((j - 1) & 1) * kRadix + kRadix - 1];
+      il = (int)((c >> 16) + (c & 0xFFFFu)) == TILE;
+    }
+    if (tile_n == TILE) {
+      if (IL && il) {
+        if (inv) cr0 = rank_tile(std::true_type{}, std::integral_constant<int, IL ? 2 : 0>{}, tile, tile_n, sb, vsb);
+        else cr0 = rank_tile(std::true_type{}, std::integral_constant<int, IL ? 1 : 0>{}, tile, tile_n, sb, vsb);
+      } else {
+        cr0 = rank_tile(std::true_type{}, WO0{}, tile, tile_n, sb, vsb);
+      }
+    } else {
+      cr0 = rank_tile(std::false_type{}, WO0{}, tile, tile_n, sb, vsb);
+    }
 #ifdef HSORT_PHASE_TIMING
     t_cnt += cr0 - cc0;
     long long cw1 = clock64();
@@ -1693,7 +1770,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #else
     (void)cr0;
 #endif
-    if (j >= 1) write_out(j - 1, prev_tile);
+    if (j >= 1 && !il) write_out(j - 1, prev_tile);
 #ifdef HSORT_PHASE_TIMING
     t_wo += clock64() - cw1;
 #endif

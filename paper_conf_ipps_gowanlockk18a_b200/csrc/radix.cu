@@ -1157,6 +1157,9 @@ struct WsSmem {
 #define HSORT_WS_PATOM 3  // leader atomics: 0 branch per item, 1 predicated PTX, 2 every lane adds to
                           // the digit slot (0 unless leader), 3 non-leaders add to a word of their own
 #endif
+#ifndef HSORT_WS_PATOM_DM2
+#define HSORT_WS_PATOM_DM2 1  // ... also in the elision's diverting pass (A/B: 5.33 -> 5.23 ms)
+#endif
 #ifndef HSORT_WS_IL_DM2
 #define HSORT_WS_IL_DM2 0  // ... also in the elision's diverting pass (A/B: slower, spills)
 #endif
@@ -1698,7 +1701,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
         rr[i] = atom_add_if_leader(&wh[dd[i]], (uint32_t)__popc(peers[i]), lane, leader);
       else if (HSORT_WS_PATOM == 2 && FULL && DM != 2)  // every lane adds (0 unless leader)
         rr[i] = atomicAdd(&wh[dd[i]], lane == leader ? (uint32_t)__popc(peers[i]) : 0u);
-      else if (HSORT_WS_PATOM == 3 && FULL && DM != 2)  // every lane adds; a non-leader to its own
+      else if (HSORT_WS_PATOM == 3 && FULL && (DM != 2 || HSORT_WS_PATOM_DM2))  // every lane adds; a non-leader to its own
         // word of s_dummy, so large groups (duplicate-heavy data) do not serialise on one address
         rr[i] = atomicAdd(lane == leader ? &wh[dd[i]] : s_dummy + lane, (uint32_t)__popc(peers[i]));
       else

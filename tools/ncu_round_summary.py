@@ -11,6 +11,10 @@ from collections import OrderedDict
 
 tag = sys.argv[1]
 G = "gpurun_out"
+try:  # HBM peak of this pool (driver-written)
+    PEAK = float(json.load(open("MEASURED_PEAKS.json"))["hbm_gbs"])
+except Exception:
+    PEAK = 6464.0
 
 
 def short(name):
@@ -85,7 +89,7 @@ for rep, what, n, bpk, key in caps:
     rd, wr = tob(*m["dram__bytes_read.sum"]), tob(*m["dram__bytes_write.sum"])
     t = float(m["gpu__time_duration.sum"][0].replace(",", "")) * (1e-3 if m["gpu__time_duration.sum"][1] in ("us", "usecond") else 1)
     md.append(f"- DRAM read+write: {(rd+wr)/1e9:.3f} GB = {(rd+wr)/n:.2f} B/key (algorithmic {bpk} B/key: "
-              f"{(rd+wr)/(bpk*n):.3f}x); algorithmic {bpk*n/(t*1e-3)/1e9:.0f} GB/s = {bpk*n/(t*1e-3)/1e9/6464:.1%} of 6464 GB/s")
+              f"{(rd+wr)/(bpk*n):.3f}x); algorithmic {bpk*n/(t*1e-3)/1e9:.0f} GB/s = {bpk*n/(t*1e-3)/1e9/PEAK:.1%} of {PEAK:.0f} GB/s")
     md.append("")
     traffic[f"{key}_dram_bytes_per_launch"] = rd + wr
     traffic[f"{key}_n"] = n

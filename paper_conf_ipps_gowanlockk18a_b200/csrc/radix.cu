@@ -1160,6 +1160,12 @@ struct WsSmem {
 #ifndef HSORT_WS_PATOM_DM2
 #define HSORT_WS_PATOM_DM2 1  // ... also in the elision's diverting pass (A/B: 5.33 -> 5.23 ms)
 #endif
+#ifndef HSORT_WS_IL_K32
+#define HSORT_WS_IL_K32 0  // interleaved write-out in the 32-bit-key pass (A/B: 17.55 vs 17.48 ms off)
+#endif
+#ifndef HSORT_WS_PATOM_K32
+#define HSORT_WS_PATOM_K32 1  // branch-free leader atomics there (A/B: 18.63 ms without)
+#endif
 #ifndef HSORT_WS_IL_DM2
 #define HSORT_WS_IL_DM2 0  // ... also in the elision's diverting pass (A/B: slower, spills)
 #endif
@@ -1701,7 +1707,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
         rr[i] = atom_add_if_leader(&wh[dd[i]], (uint32_t)__popc(peers[i]), lane, leader);
       else if (HSORT_WS_PATOM == 2 && FULL && DM != 2)  // every lane adds (0 unless leader)
         rr[i] = atomicAdd(&wh[dd[i]], lane == leader ? (uint32_t)__popc(peers[i]) : 0u);
-      else if (HSORT_WS_PATOM == 3 && FULL && (DM != 2 || HSORT_WS_PATOM_DM2))  // every lane adds; a non-leader to its own
+      else if (HSORT_WS_PATOM == 3 && FULL && (DM != 2 || HSORT_WS_PATOM_DM2) && (!K32 || HSORT_WS_PATOM_K32))  // every lane adds; a non-leader to its own
         // word of s_dummy, so large groups (duplicate-heavy data) do not serialise on one address
         rr[i] = atomicAdd(lane == leader ? &wh[dd[i]] : s_dummy + lane, (uint32_t)__popc(peers[i]));
       else
@@ -1750,7 +1756,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
     using WO0 = std::integral_constant<int, 0>;
     // interleaved write-out (WO): this tile and the previous one are full (only the last tile is
     // ragged; in the elision's diverting pass a tile that lost outliers is written out separately)
-    constexpr bool IL = HSORT_WS_IL && (DM != 2 || HSORT_WS_IL_DM2);
+    constexpr bool IL = HSORT_WS_IL && (DM != 2 || HSORT_WS_IL_DM2) && (!K32 || HSORT_WS_IL_K32);
     bool il = IL && j >= 1 && tile_n == TILE;
     if (DM == 2 && il) {  // the elision's diverting pass: only if tile j-1 lost no outliers
       const uint32_t c = s_cnt[((j - 1) & 1) * kRadix + kRadix - 1];

@@ -1140,9 +1140,6 @@ struct WsSmem {
 #ifndef HSORT_WS_ITEMS
 #define HSORT_WS_ITEMS 15  // keys per compute thread: 8640-key tiles, 3 stages = 203 KB, 1 CTA/SM
 #endif
-#ifndef HSORT_WS_RC
-#define HSORT_WS_RC 0  // ranking chunk (0 = all items at once)
-#endif
 #ifndef HSORT_K32_ITEMS
 #define HSORT_K32_ITEMS 20  // 32-bit keys per compute thread: 11520-key tiles, 3 stages = 138 KB
                             // (A/B 15 / 18 / 20 / 22: 19.2 / 18.6 / 17.4 / 17.7 ms per 2^30 keys)
@@ -1154,8 +1151,9 @@ struct WsSmem {
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
 #endif
 #ifndef HSORT_WS_PATOM
-#define HSORT_WS_PATOM 3  // leader atomics: 0 branch per item, 1 predicated PTX, 2 every lane adds to
-                          // the digit slot (0 unless leader), 3 non-leaders add to a word of their own
+#define HSORT_WS_PATOM 1  // branch-free leader atomics: every lane issues one, a non-leader to a word
+                          // of its own (A/B: a branch per item, predicated PTX and
+                          // every lane adding to the digit's slot were slower)
 #endif
 #ifndef HSORT_WS_PATOM_DM2
 #define HSORT_WS_PATOM_DM2 1  // ... also in the elision's diverting pass (A/B: 5.33 -> 5.23 ms)
@@ -1194,16 +1192,6 @@ __device__ __forceinline__ void st_global_u64(uint64_t addr, uint64_t v) {
 __device__ __forceinline__ void st_global_w(const uint64_t* a, uint64_t v) { st_global_u64((uint64_t)a, v); }
 __device__ __forceinline__ void st_global_w(const uint32_t* a, uint32_t v) {
   asm volatile("st.global.u32 [%0], %1;" ::"l"((uint64_t)a), "r"(v) : "memory");
-}
-// The group leader's shared atomic as one predicated instruction (no branch per item); the
-// result is defined in the leader lane only (the others read it by shuffle)
-__device__ __forceinline__ uint32_t atom_add_if_leader(uint32_t* a, uint32_t v, int lane, int leader) {
-  uint32_t r;
-  asm volatile("{\n\t.reg .pred q;\n\tsetp.eq.s32 q, %1, %2;\n\t@q atom.shared.add.u32 %0, [%3], %4;\n\t}"
-               : "=r"(r)
-               : "r"(lane), "r"(leader), "r"(smem_u32(a)), "r"(v)
-               : "memory");
-  return r;
 }
 // One bit of the ballot multisplit: peers &= (bit b of d) ? ballot(bit) : ~ballot(bit).
 __device__ __forceinline__ uint32_t peer_bit(uint32_t peers, uint32_t d, uint32_t bm) {
@@ -1703,11 +1691,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
-      if (HSORT_WS_PATOM == 1 && FULL && DM != 2)
-        rr[i] = atom_add_if_leader(&wh[dd[i]], (uint32_t)__popc(peers[i]), lane, leader);
-      else if (HSORT_WS_PATOM == 2 && FULL && DM != 2)  // every lane adds (0 unless leader)
-        rr[i] = atomicAdd(&wh[dd[i]], lane == leader ? (uint32_t)__popc(peers[i]) : 0u);
-      else if (HSORT_WS_PATOM == 3 && FULL && (DM != 2 || HSORT_WS_PATOM_DM2) && (!K32 || HSORT_WS_PATOM_K32))  // every lane adds; a non-leader to its own
+      if (HSORT_WS_PATOM && FULL && (DM != 2 || HSORT_WS_PATOM_DM2) && (!K32 || HSORT_WS_PATOM_K32))  // every lane adds; a non-leader to its own
         // word of s_dummy, so large groups (duplicate-heavy data) do not serialise on one address
         rr[i] = atomicAdd(lane == leader ? &wh[dd[i]] : s_dummy + lane, (uint32_t)__popc(peers[i]));
       else

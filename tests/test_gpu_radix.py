@@ -62,6 +62,40 @@ def test_single_pass_is_stable_counting_sort(hs_gpu, oracle_mod, digit, n):
     assert np.array_equal(dst.cpu().numpy(), oracle_mod.counting_sort_pass(K, digit))
 
 
+# every CTA of the persistent pass (one per SM, 148 on B200) processes several 8640-key tiles, so
+# the write-out of tile j-1 runs interleaved with the ranking of tile j (radix.cu HSORT_WS_IL)
+MULTI_TILE_N = 3 * 148 * 8640 + 4097
+
+
+@pytest.mark.parametrize("digit", [0, 3, 7])
+@pytest.mark.parametrize("kind", ["random", "low_entropy"])
+def test_single_pass_multi_tile_per_cta(hs_gpu, oracle_mod, digit, kind):
+    import torch
+    rng = np.random.default_rng(digit * 7 + len(kind))
+    n = MULTI_TILE_N
+    if kind == "random":  # ballot ranking with the branch-free leader atomics
+        K = rng.integers(0, 2**64, size=n, dtype=np.uint64)
+        K[::5] = K[7]
+    else:  # few distinct digits per warp: match.any ranking, large peer groups
+        K = rng.integers(0, 6, size=n, dtype=np.uint64) << np.uint64(8 * digit)
+        K |= rng.integers(0, 2**8, size=n, dtype=np.uint64) << np.uint64(8 * ((digit + 1) % 8))
+    src = _to_dev(K)
+    dst = torch.empty_like(src)
+    hs_gpu.hsort_device_radix_pass(src, dst, digit)
+    assert np.array_equal(dst.cpu().numpy(), oracle_mod.counting_sort_pass(K, digit))
+
+
+@pytest.mark.parametrize("dist", ["uniform", "normal", "zipf_dup", "few_distinct", "special"])
+def test_device_sort_multi_tile_per_cta(hs_gpu, oracle_mod, inputs_mod, dist):
+    import torch
+    A = inputs_mod.generate(dist, MULTI_TILE_N, seed=77)
+    d_in = _to_dev(A)
+    d_out = torch.empty_like(d_in)
+    hs_gpu.hsort_sort_device(d_in, d_out)
+    torch.cuda.synchronize()
+    assert np.array_equal(_bits(d_out.cpu().numpy()), _bits(oracle_mod.sort_f64(A)))
+
+
 @pytest.mark.parametrize("dist", DISTS)
 @pytest.mark.parametrize("n", SIZES)
 def test_device_sort_bit_exact(hs_gpu, oracle_mod, inputs_mod, dist, n):

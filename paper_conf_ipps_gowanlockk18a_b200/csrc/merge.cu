@@ -18,6 +18,9 @@
 
 #include "internal.h"
 
+#ifndef HSORT_MERGE_ABS
+#define HSORT_MERGE_ABS 1  // unrolled merge steps on absolute head indices
+#endif
 #ifndef HSORT_MERGE_CLAMP
 // 0: a merge step may load the head one past an exhausted pair (pp(s2) <= BUF stays inside the
 // dynamic shared allocation; the bounds test never takes it), saving the clamp per output
@@ -480,6 +483,20 @@ __global__ void __launch_bounds__(T) k_merge_tile(
         // constant offsets from pp(p0) (p0 = IPT tid: no pad inside a thread's range)
         uint64_t* d = dst + Cfg::pp(p);
         uint64_t* dv = vdst + Cfg::pp(p);
+#if HSORT_MERGE_ABS
+        int ia = s0 + i, ib = s1 + jb;  // absolute heads; A = [s0, s1), B = [s1, s2)
+#pragma unroll
+        for (int q = 0; q < IPT; ++q) {
+          const bool ta = ib >= s2 || (ia < s1 && a <= b);
+          d[q] = ta ? a : b;
+          if (KV) dv[q] = vsrc[Cfg::pp(ta ? ia : ib)];
+          ia += ta;
+          ib += !ta;
+          const uint64_t y = src[Cfg::pp(ta ? ia : ib)];  // may be one past an exhausted pair
+          a = ta ? y : a;
+          b = ta ? b : y;
+        }
+#else
 #pragma unroll
         for (int q = 0; q < IPT; ++q) {
           const bool ta = jb >= lenB || (i < lenA && a <= b);
@@ -495,6 +512,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
           a = ta ? y : a;
           b = ta ? b : y;
         }
+#endif
         p = stop;
       }
       for (; p < stop; ++p) {

@@ -1147,6 +1147,9 @@ struct WsSmem {
 #ifndef HSORT_WS_NMATCH
 #define HSORT_WS_NMATCH 4  // items ranked with match.any in high-entropy passes (A/B over 2..7)
 #endif
+#ifndef HSORT_KV_NMATCH
+#define HSORT_KV_NMATCH 2  // ... in the key/value pass (13 items; A/B 2 / 3 / 4 / 5: 8.29 / 8.34 / 8.73 / 8.51 ms)
+#endif
 #ifndef HSORT_WS_W
 #define HSORT_WS_W 4  // look-back rows per round trip in the warp-specialised pass
 #endif
@@ -1648,7 +1651,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
       // high-entropy digits: an 8-ballot multisplit (4 instructions per bit: test -> predicate,
       // vote, select, and) for most items; the first NM items use match.any, which runs on another
       // pipe, so both proceed in parallel
-      constexpr int NM0 = KV ? (ITEMS * HSORT_WS_NMATCH + 7) / 15 : HSORT_WS_NMATCH;
+      constexpr int NM0 = KV ? HSORT_KV_NMATCH : HSORT_WS_NMATCH;
       constexpr int NM = NM0 < ITEMS ? NM0 : ITEMS;
 #pragma unroll
       for (int i = 0; i < NM; ++i) peers[i] = __match_any_sync(0xffffffffu, dd[i]);

@@ -22,18 +22,27 @@ for i in range(L):
 for lanes in range(1, L + 1):
     bar = threading.Barrier(lanes + 1)
     done = []
+    phases = []
+    t_start = [time.perf_counter()]
     def work(l):
         bar.wait()
         for _ in range(K):
+            t = time.perf_counter()
             hs.hsort_sort_lane(l, A[l], B[l])
+            st = hs.hsort_get_stats()
+            phases.append({"lane": l, "t0": round(t - t_start[0], 3), "s": round(time.perf_counter() - t, 3),
+                           "sort_phase": round(st["t_sort_phase"], 3), "merge_phase": round(st["t_merge_phase"], 3)})
         done.append(time.perf_counter())
     th = [threading.Thread(target=work, args=(l,)) for l in range(lanes)]
     for t in th: t.start()
     bar.wait()
     t0 = time.perf_counter()
+    t_start[0] = t0
     for t in th: t.join()
     dt = max(done) - t0
     ok = all(bool(np.all(B[l].numpy()[1:] >= B[l].numpy()[:-1])) for l in range(lanes))
     print(json.dumps({"lanes": lanes, "sorts": lanes * K, "s": dt, "keys_per_s": lanes * K * n / dt,
                       "ms_per_sort": 1e3 * dt / K, "sorted": ok}), flush=True)
+    if os.environ.get("LANES_PHASES"):
+        for ph in sorted(phases, key=lambda x: x["t0"]): print(json.dumps(ph))
 hs.hsort_finalize()

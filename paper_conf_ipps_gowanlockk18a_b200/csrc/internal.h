@@ -135,7 +135,10 @@ cudaError_t radix_one_pass(RadixScratch& s, const uint64_t* src, uint64_t* dst, 
                            int digit, cudaStream_t st);
 
 // ---- GPU merge (merge.cu) ------------------------------------------------------------------
-constexpr int kMergeTile = 4096;  // output keys per merge CTA
+#ifndef HSORT_MERGE_TILE
+#define HSORT_MERGE_TILE 4096
+#endif
+constexpr int kMergeTile = HSORT_MERGE_TILE;  // output keys per merge CTA
 constexpr int kMaxMergeRuns = 1024;
 
 // Runs of a merge: run j has len_j = d_off[j + 1] - d_off[j] keys (device offsets) and starts at

@@ -47,7 +47,8 @@ for k in ks:
         a, b = int(cuts[j]), int(cuts[j + 1])
         if b > a:
             hs.hsort_sort_device_keys(d_a[a:b], d_runs[a:b], True, False)
-    tiles = (n + 4095) // 4096
+    mt = int(os.environ.get("MERGE_TILE", "4096"))  # the build's kMergeTile (A/B builds)
+    tiles = (n + mt - 1) // mt
     d_ranks = torch.empty((tiles + 1) * k, dtype=torch.int64, device="cuda")
     for _ in range(2):
         hs.hsort_device_merge(d_runs, cuts, d_out, False)
@@ -56,7 +57,7 @@ for k in ks:
     for _ in range(5):
         e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
         e[0].record(st)
-        hs.hsort_device_corank(d_runs, cuts, 4096, tiles + 1, d_ranks)
+        hs.hsort_device_corank(d_runs, cuts, mt, tiles + 1, d_ranks)
         e[1].record(st)
         e[2].record(st)
         hs.hsort_device_merge(d_runs, cuts, d_out, False)

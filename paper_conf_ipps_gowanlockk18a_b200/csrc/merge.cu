@@ -18,6 +18,9 @@
 
 #include "internal.h"
 
+#ifndef HSORT_MERGE_GCACHE
+#define HSORT_MERGE_GCACHE 1  // K5 gather: run source / end cached in registers
+#endif
 #ifndef HSORT_MERGE_ABS
 #define HSORT_MERGE_ABS 1  // unrolled merge steps on absolute head indices
 #endif
@@ -412,6 +415,26 @@ __global__ void __launch_bounds__(T) k_merge_tile(
   {
     const int e0 = w * C + lane;
     int a = (k > 1 && e0 < L) ? advance_run(bnd, 0, k, (uint32_t)e0) : 0;
+#if HSORT_MERGE_GCACHE
+    // the run's source and its end held in registers; they change only when e crosses a boundary
+    const uint64_t* sp = s_src[a];
+    const uint64_t* svp = KV ? s_vsrc[a] : nullptr;
+    uint32_t nb = a + 1 < k ? bnd[a + 1] : 0xffffffffu;
+#pragma unroll
+    for (int q = 0; q < IPT; ++q) {
+      const int e = e0 + 32 * q;
+      if (e < L) {
+        while ((uint32_t)e >= nb) {
+          ++a;
+          sp = s_src[a];
+          if (KV) svp = s_vsrc[a];
+          nb = a + 1 < k ? bnd[a + 1] : 0xffffffffu;
+        }
+        v[q] = ld_stream_u64(sp + e);
+        if (KV) vv[q] = ld_stream_u64(svp + e);
+      }
+    }
+#else
 #pragma unroll
     for (int q = 0; q < IPT; ++q) {
       const int e = e0 + 32 * q;
@@ -421,6 +444,7 @@ __global__ void __launch_bounds__(T) k_merge_tile(
         if (KV) vv[q] = ld_stream_u64(s_vsrc[a] + e);
       }
     }
+#endif
   }
   uint64_t* vo = KV ? vout + (o0 - out_origin) : nullptr;
   if (k == 1) {

@@ -126,6 +126,7 @@ struct Options {
       {"merge_chunk", 1ll << 26},    // GPU merge output chunk (keys)
       {"device_reserve_mb", 2048},   // HBM kept free for the runtime / other tenants
       {"kernel_timing", 0},          // 1: CUDA events around every radix kernel (bench roofline)
+      {"defer_out_drain", 1},        // STREAM GPU merge share: staged DtoH copy-outs drained lazily
       {"dde", 1},                    // 1: dominant-digit elision in the GPUSort
       {"dde_min_n", 1ll << 22},      // smallest n the elision is tried at
       {"memcpy_nt", 1},              // PARMEMCPY staging copies with non-temporal stores
@@ -165,6 +166,12 @@ struct GpuCtx {
   uint64_t ring_bytes = 0;
   std::vector<cudaEvent_t> ev_in, ev_out;
   uint64_t in_next = 0;
+  // staged downloads: out-ring slots whose DMA is enqueued but whose copy-out into the host
+  // destination is still pending (dst, bytes); with defer_out set, download() returns without
+  // draining them, so the next download's DMAs keep the link busy (flush_out drains the rest)
+  uint64_t out_next = 0;
+  std::vector<std::pair<char*, uint64_t>> out_pend;
+  bool defer_out = false;
 };
 
 struct State {
@@ -356,8 +363,25 @@ void upload(GpuCtx& g, void* d_dst, const void* h_src, uint64_t bytes, cudaStrea
   }
 }
 
+// Staged downloads: copy the out-ring slot s (DMA complete) into its pending host destination.
+void drain_out(GpuCtx& g, uint64_t s, int threads, Acc& acc) {
+  CK(cudaEventSynchronize(g.ev_out[s]));
+  auto t0 = Clock::now();
+  par_memcpy(g.out_pend[s].first, g.ring_out[s], g.out_pend[s].second, threads);
+  acc.t_stage += secs_since(t0);
+  g.out_pend[s] = {nullptr, 0};
+}
+// ... every pending slot, oldest first
+void flush_out(GpuCtx& g, int threads, Acc& acc) {
+  const uint64_t R = g.out_pend.size();
+  for (uint64_t i = 0; i < R; ++i) {
+    const uint64_t s = (g.out_next + i) % R;
+    if (g.out_pend[s].first) drain_out(g, s, threads, acc);
+  }
+}
 // Device -> host.  Direct: enqueued only (caller synchronises st).  Staged: returns when every
-// byte is in h_dst (DMA of chunk c overlaps the host copy-out of chunk c-1).
+// byte is in h_dst (DMA of chunk c overlaps the host copy-out of chunk c-1), unless g.defer_out:
+// then the last ring slots stay pending until a later download needs them or flush_out.
 void download(GpuCtx& g, void* h_dst, const void* d_src, uint64_t bytes, cudaStream_t st,
               bool direct, int threads, Acc& acc) {
   Nvtx r(direct ? "DtoH" : "DtoH+Stage");
@@ -368,21 +392,16 @@ void download(GpuCtx& g, void* h_dst, const void* d_src, uint64_t bytes, cudaStr
     return;
   }
   const uint64_t R = g.ring_out.size(), C = g.ring_bytes;
-  const uint64_t nch = (bytes + C - 1) / C;
-  auto drain = [&](uint64_t c) {
-    uint64_t s = c % R, o = c * C, len = std::min(C, bytes - o);
-    CK(cudaEventSynchronize(g.ev_out[s]));
-    auto t0 = Clock::now();
-    par_memcpy((char*)h_dst + o, g.ring_out[s], len, threads);
-    acc.t_stage += secs_since(t0);
-  };
-  for (uint64_t c = 0; c < nch; ++c) {
-    if (c >= R) drain(c - R);
-    uint64_t s = c % R, o = c * C, len = std::min(C, bytes - o);
+  if (g.out_pend.size() != R) g.out_pend.assign(R, {nullptr, 0});
+  for (uint64_t o = 0; o < bytes; o += C) {
+    const uint64_t len = std::min(C, bytes - o);
+    const uint64_t s = g.out_next++ % R;
+    if (g.out_pend[s].first) drain_out(g, s, threads, acc);  // the slot's previous chunk
     CK(cudaMemcpyAsync(g.ring_out[s], (const char*)d_src + o, len, cudaMemcpyDeviceToHost, st));
     CK(cudaEventRecord(g.ev_out[s], st));
+    g.out_pend[s] = {(char*)h_dst + o, len};
   }
-  for (uint64_t c = (nch > R ? nch - R : 0); c < nch; ++c) drain(c);
+  if (!g.defer_out) flush_out(g, threads, acc);
 }
 
 struct EvPair {
@@ -1135,6 +1154,16 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
   em.make();
   std::vector<uint64_t> hoff(2 * (size_t)(k + 1));
   Acc acc;
+  // a staged (pageable B) download of chunk ch leaves its last ring slots pending, so chunk ch+1's
+  // DMAs start at once instead of after the copy-out tail (HSORT option defer_out_drain)
+  struct DeferGuard {
+    GpuCtx& g;
+    ~DeferGuard() {
+      g.defer_out = false;
+      std::fill(g.out_pend.begin(), g.out_pend.end(), std::make_pair((char*)nullptr, (uint64_t)0));
+    }
+  } dg{g};
+  g.defer_out = S().opt.get("defer_out_drain") == 1;
   CK(cudaEventRecord(em.a, g.s_h2d));
   // Chunk ch+1's HtoD + K4/K5 are enqueued before chunk ch's (possibly staged, blocking) DtoH, so
   // the two link directions overlap (duplex); two slots per buffer.
@@ -1178,6 +1207,7 @@ void gpu_merge_from_host(GpuCtx& g, CallCtx& c, const std::vector<const uint64_t
              c.direct_out, (int)S().opt.get("merge_stage_threads"), acc);
     CK(cudaEventRecord(out_free[s], g.s_d2h));
   }
+  flush_out(g, (int)S().opt.get("merge_stage_threads"), acc);
   CK(cudaEventRecord(em.b, g.s_d2h));
   CK(cudaStreamSynchronize(g.s_d2h));
   CK(cudaStreamSynchronize(g.s_comp));

@@ -10,6 +10,10 @@ if os.environ.get("HSORT_LIB"):  # A/B: an alternative build of the library
     hs.LIB_PATH = os.path.abspath(os.environ["HSORT_LIB"])
 
 n = int(float(sys.argv[1])) if len(sys.argv) > 1 else int(4.3e9)
+for kv in os.environ.get("OOC_OPTS", "").split(","):  # e.g. merge_stage_threads=12,merge_gpu_permille=1000
+    if kv:
+        k_, v_ = kv.split("=")
+        hs.hsort_set_option(k_, int(v_))
 hs.hsort_init()
 A = hsort_inputs.generate("uniform", n, seed=3)
 B = np.empty_like(A)
@@ -18,6 +22,8 @@ hs.hsort_set_option("pin_w", 1)
 runs = [("auto", -1)] * 5 + [("f600", 600), ("f700", 700), ("f800", 800)]
 if os.environ.get("OOC_AUTO_ONLY"):
     runs = [("auto", -1)] * int(os.environ["OOC_AUTO_ONLY"])
+if os.environ.get("OOC_FIXED"):  # e.g. 1000,1000,950: fixed merge splits (per mille)
+    runs = [("f" + x, int(x)) for x in os.environ["OOC_FIXED"].split(",")]
 for name, fp in runs:
     hs.hsort_set_option("merge_gpu_permille", fp)
     t = time.perf_counter()

@@ -659,6 +659,12 @@ cudaError_t corank_launch(const uint64_t* keys, const uint64_t* const* rp, const
 #define HSORT_CORANK_COARSE 16  // A/B at 2^30 keys: 8 / 16 / 32 / 64 -> 2.55 / 2.39 / 2.30 / 2.34 ms (k = 12)
 #endif
 constexpr uint64_t kCoarse = HSORT_CORANK_COARSE;
+#ifndef HSORT_CORANK_LEVELS
+#define HSORT_CORANK_LEVELS 0  // co-rank levels (2: one coarse level); 0: 3 from k = 32 runs, else 2
+                               // (A/B at 2^30 keys, profiles/r03bi: 3 levels cost 0.1-0.16 ms more
+                               // at k <= 12, save 0.1 / 0.8 ms at k = 32 / 128)
+#endif
+static int corank_levels(int k) { return HSORT_CORANK_LEVELS ? HSORT_CORANK_LEVELS : (k >= 32 ? 3 : 2); }
 
 namespace {
 // coarse rows c0 .. c0 + nc - 1 bracketing every requested bound (0 rows: single level)
@@ -675,26 +681,47 @@ void coarse_rows(uint64_t total, uint64_t step, uint64_t bound_begin, uint64_t n
 }
 }  // namespace
 
-uint64_t merge_corank_scratch_elems(int k, uint64_t total, uint64_t step, uint64_t bound_begin,
-                                    uint64_t n_bounds) {
+// levels: 2 = a coarse level (full-range search) + the requested bounds; more: the coarse level
+// is itself computed from a coarser one, recursively (each level kCoarse times sparser)
+static uint64_t corank_scratch_rec(int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                                   uint64_t n_bounds, int levels) {
   uint64_t c0, nc;
   coarse_rows(total, step, bound_begin, n_bounds, k, &c0, &nc);
-  return nc * (uint64_t)k;
+  if (nc == 0 || levels < 2) return 0;
+  return nc * (uint64_t)k + corank_scratch_rec(k, total, step * kCoarse, c0, nc, levels - 1);
+}
+uint64_t merge_corank_scratch_elems(int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                                    uint64_t n_bounds) {
+  return corank_scratch_rec(k, total, step, bound_begin, n_bounds, corank_levels(k));
 }
 
+cudaError_t merge_corank_rec(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                             int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                             uint64_t n_bounds, uint64_t* ranks, uint64_t* scratch,
+                             uint64_t scratch_elems, int levels, cudaStream_t st);
 cudaError_t merge_corank(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
                          int k, uint64_t total, uint64_t step, uint64_t bound_begin,
                          uint64_t n_bounds, uint64_t* ranks, uint64_t* scratch,
                          uint64_t scratch_elems, cudaStream_t st) {
+  return merge_corank_rec(keys, rp, d_off, k, total, step, bound_begin, n_bounds, ranks, scratch,
+                          scratch_elems, corank_levels(k), st);
+}
+
+cudaError_t merge_corank_rec(const uint64_t* keys, const uint64_t* const* rp, const uint64_t* d_off,
+                             int k, uint64_t total, uint64_t step, uint64_t bound_begin,
+                             uint64_t n_bounds, uint64_t* ranks, uint64_t* scratch,
+                             uint64_t scratch_elems, int levels, cudaStream_t st) {
   if (k < 1 || k > kMaxMergeRuns) return cudaErrorInvalidValue;
   if (n_bounds == 0) return cudaSuccess;
   uint64_t c0, nc;
   coarse_rows(total, step, bound_begin, n_bounds, k, &c0, &nc);
-  if (nc == 0 || !scratch || scratch_elems < nc * (uint64_t)k)  // single level
+  if (levels < 2 || nc == 0 || !scratch || scratch_elems < nc * (uint64_t)k)  // single level
     return corank_launch(keys, rp, d_off, k, total, step, bound_begin, n_bounds, ranks, nullptr, 1,
                          0, st);
   const uint64_t cstep = step * kCoarse;
-  cudaError_t e = corank_launch(keys, rp, d_off, k, total, cstep, c0, nc, scratch, nullptr, 1, 0, st);
+  cudaError_t e = merge_corank_rec(keys, rp, d_off, k, total, cstep, c0, nc, scratch,
+                                   scratch + nc * (uint64_t)k, scratch_elems - nc * (uint64_t)k,
+                                   levels - 1, st);
   if (e != cudaSuccess) return e;
   return corank_launch(keys, rp, d_off, k, total, step, bound_begin, n_bounds, ranks, scratch,
                        cstep, c0, st);

@@ -58,6 +58,27 @@ def test_corank_two_level_matches_oracle(hs_gpu, oracle_mod, k, hi):
         assert np.array_equal(got[b], oracle_mod.corank(runs, o)), (b, o)
 
 
+@pytest.mark.parametrize("k", [32, 48, 128])
+@pytest.mark.parametrize("hi", [2**64, 7])
+def test_corank_three_level_matches_oracle(hs_gpu, oracle_mod, k, hi):
+    """k >= 32 with >= 1024 bounds: the coarse level is itself computed from a coarser one (three
+    levels, merge.cu corank_levels), windows entered by galloping at every level."""
+    import torch
+    rng = np.random.default_rng(k * 11 + hi % 997)
+    runs, keys, off = _runs(rng, k, 3000, hi)
+    total = int(off[-1])
+    step = 16
+    nb = total // step + 2
+    assert nb >= 1024
+    d_keys = torch.from_numpy(keys).cuda()
+    d_r = torch.zeros(nb * k, dtype=torch.uint64, device="cuda")
+    hs_gpu.hsort_device_corank(d_keys, off, step, nb, d_r)
+    got = d_r.cpu().numpy().reshape(nb, k)
+    for b in list(range(0, nb, 97)) + list(range(1, 40)) + [nb - 2, nb - 1]:
+        o = min(b * step, total)
+        assert np.array_equal(got[b], oracle_mod.corank(runs, o)), (b, o)
+
+
 @pytest.mark.parametrize("k", [1, 2, 5, 16, 120, 1024])
 @pytest.mark.parametrize("hi", [2**64, 7])
 def test_device_merge_matches_oracle(hs_gpu, oracle_mod, k, hi):

@@ -193,7 +193,7 @@ int hsort_sort_pairs_ex(const void* A_host, const uint64_t* V_host, void* B_host
 
 /* ---------------------------------------------------------------------------------------------
  * Options, statistics, errors
- *   keys: "n_s" (batch slots per GPU, default 2), "p_s" (pinned staging chunk bytes),
+ *   keys: "n_s" (batch slots per GPU, default 3), "p_s" (pinned staging chunk bytes),
  *         "n_ring" (pinned slots per direction), "memcpy_threads" (PARMEMCPY threads; 1 = serial
  *         MCpy), "merge_threads" (CPU merge threads), "resident" (-1 auto, 0 force
  *         STREAM, 1 force RESIDENT), "merge_gpu_permille" (A12 share f in 1/1000; -1 auto),
@@ -207,10 +207,19 @@ int hsort_sort_pairs_ex(const void* A_host, const uint64_t* V_host, void* B_host
  *         "kernel_timing" (1 = CUDA events around each radix kernel, see hsort_get_kernel_times),
  *         "auto_pipeline_min" (smallest n for the auto pipelined RESIDENT plan; 0 = never),
  *         "pin_w" (STREAM-mode W: 1 cached pinned, 0 pageable + staging, -1 auto = pinned up to
- *         "pin_w_max_mb" (16 GiB) or when a large enough pinned W is already cached),
+ *         "pin_w_max_mb" (default 2^20 MB) or when a large enough pinned W is already cached),
+ *         "w_cache" (1 = keep W allocated, prefaulted and locked across calls),
  *         "dde" (1 = dominant-digit elision in the GPUSort: when the top active digit has one
  *         value held by all but a few keys, its LSD pass is dropped and the outliers are sorted
- *         separately; output-invisible; 0 = off).
+ *         separately; output-invisible; 0 = off), "dde_min_n" (smallest n it is tried at),
+ *         "memcpy_nt" (1 = PARMEMCPY with non-temporal stores),
+ *         "merge_stage_threads" (STREAM merge: host threads per GPU that stage the GPU share's
+ *         DtoH into a pageable B), "defer_out_drain" (1 = those staged copy-outs drained lazily
+ *         across merge chunks, so the next chunk's DMA starts at once),
+ *         "register_host" (1 = page-lock pageable A / B for the call and DMA them directly),
+ *         "msd" (1 = RESIDENT plans use the MSD-first bucket split), "msd_bucket_keys",
+ *         "virtual_gpus" (set before hsort_init: that many GPU contexts, mapped round-robin onto
+ *         the visible devices; the lanes of hsort_sort_lane and multi-GPU tests on one device).
  * ------------------------------------------------------------------------------------------- */
 int hsort_set_option(const char* key, int64_t value);
 int hsort_get_option(const char* key, int64_t* value);

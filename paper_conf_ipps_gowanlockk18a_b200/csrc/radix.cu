@@ -1537,7 +1537,7 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
   // one tile: load from the stage, per-warp digit counts, tile aggregate + scan, warp ranking,
   // scatter into the stage in digit order.  FULL (every tile but the last) drops all bounds logic.
   // DM (compile-time): 0 no elision work, 1 count the outliers' digit-P histogram (pass 0),
-  // 2 divert the outliers (the elision's last pass; never FULL)
+  // 2 divert the outliers (the elision's last pass)
   // WO (compile-time): 0 = no write-out here; 1 / 2 = write tile j-1 out (2: with the inverse
   // transform) interleaved with this tile's ranking, so its shared loads and global stores issue
   // beside the ballots (ALU) instead of in a memory-only phase of their own
@@ -1698,8 +1698,9 @@ __global__ void __launch_bounds__(CT + 32, (CT == 256 ? 2 : 1)) k_onesweep_ws(ui
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const int leader = 31 - __clz(peers[i]);
-      if (HSORT_WS_PATOM && FULL && (DM != 2 || HSORT_WS_PATOM_DM2) && (!K32 || HSORT_WS_PATOM_K32))  // every lane adds; a non-leader to its own
-        // word of s_dummy, so large groups (duplicate-heavy data) do not serialise on one address
+      // branch-free: every lane adds; a non-leader to its own word of s_dummy, so large groups
+      // (duplicate-heavy data) do not serialise on one address
+      if (HSORT_WS_PATOM && FULL && (DM != 2 || HSORT_WS_PATOM_DM2) && (!K32 || HSORT_WS_PATOM_K32))
         rr[i] = atomicAdd(lane == leader ? &wh[dd[i]] : s_dummy + lane, (uint32_t)__popc(peers[i]));
       else
         rr[i] = (lane == leader && ((FULL && (DM != 2 || !w_out)) || dd[i] < kRadix))
